@@ -1,0 +1,187 @@
+/*
+ * somier.h -- the Somier time step spread over devices: C ABI of libsomier.so.
+ *
+ * Paper (§V "Use case: Somier mini-app", 319-344):
+ * a 3-D grid of springs; each time step runs the kernels forces (a stencil over
+ * the neighbour cells), accelerations, velocities, positions, and a "centers"
+ * reduction over the positions. Four variables x three
+ * 3-D fp64 grids. The step is spread over devices along the
+ * outermost dimension with halos "between chunks in the outermost dimension"
+ * (PAPER.md:328), i.e. `target spread` over the i-loop with
+ * map(to: X[omp_spread_start-1 : omp_spread_size+2]).
+ * Where the paper is silent the readings of DESIGN.md §3
+ * apply: central Hooke springs to the 6 face neighbours, six fixed faces,
+ * semi-implicit Euler with double-buffered (Jacobi) positions, centre of mass
+ * over all nodes by an exact int128 fixed-point sum, vmax = max |v|.
+ *
+ * One call of somier_step = the paper's five kernels fused into ONE sm_100a
+ * kernel launch per chunk; the halo exchange is fused into the same kernel
+ * (boundary planes are stored straight into the neighbour chunk's halo slot,
+ * through NVLink P2P / CUDA IPC when the neighbour is on another GPU).
+ *
+ * Lifetime (mirrors the data directives):
+ *   somier_init        ~ target enter data spread map(to: X[start-1:size+2], V[start:size])
+ *   somier_load        ~ target update spread to(...)           (host -> device)
+ *   somier_step        ~ target spread teams distribute parallel for ... nowait
+ *   somier_sync        ~ taskgroup / taskwait
+ *   somier_stats       ~ the "centers" result of the last completed step
+ *   somier_read        ~ target exit data spread map(from: X[start:size], V[start:size])
+ *   somier_destroy     ~ end of the data region
+ *
+ * Conventions: every call returns spread_status (spread.h). Handles are
+ * library-owned, not thread-safe (one host thread per handle). CUDA errors
+ * raised by asynchronous work are sticky and reported by the next blocking
+ * call (somier_sync / somier_stats / somier_read) as SPREAD_ECUDA, with the
+ * CUDA message in spread_last_error(). A failed somier_init leaves no
+ * allocation behind.
+ */
+#ifndef PAPER_SOMIER_H
+#define PAPER_SOMIER_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#include "spread.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* K1 implementations (all compute bit-identical results). */
+typedef enum {
+    SOMIER_K1_AUTO = 0,      /* the fastest available (currently SOMIER_K1_MARCH)     */
+    SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
+    SOMIER_K1_MARCH = 2      /* plane-marching, smem-staged, 3 springs/node with reuse */
+} somier_kernel;
+
+typedef struct {
+    int64_t n[3];        /* nodes per dimension (i outermost, k contiguous); each >= 3        */
+    double spacing;      /* rest-lattice spacing                                               */
+    double rest_len;     /* spring rest length L                                               */
+    double k_spring;     /* stiffness K                                                        */
+    double mass;         /* node mass M (> 0)                                                  */
+    double dt;           /* time step h (> 0)                                                  */
+    double amplitude;    /* initial displacement amplitude a (|a| < rest_len / 2 recommended)  */
+    uint64_t seed;       /* SplitMix64 seed of the initial displacement (reading S7)           */
+    int32_t kernel;      /* somier_kernel                                                      */
+    int32_t reserved;    /* must be 0                                                          */
+} somier_params;
+
+/* Stats of one step ("centers"). The exact partial sums are
+ * exported so that per-process partials can be combined exactly. */
+typedef struct {
+    int64_t step;         /* number of completed steps                                     */
+    double centre[3];     /* (1/N) * sum over all N = n0*n1*n2 nodes of x_{t} (exact sum)  */
+    double vmax;          /* sqrt(max over nodes of v.v)                                    */
+    uint64_t sum_lo[3];   /* sum of round_half_even(x * 2^60), int128 two's complement, lo */
+    int64_t sum_hi[3];    /* ... hi                                                         */
+    uint64_t vmax2_bits;  /* IEEE-754 bits of max v.v (uint64 order == double order, >= 0)  */
+    int64_t nodes;        /* number of nodes covered by these sums                          */
+} somier_stats_t;
+
+typedef struct somier_s* somier_t;
+
+/*
+ * somier_init -- single-process mode (the paper's model: one host program drives
+ * every device of the list). Allocates every chunk of `s` on its device, generates
+ * the initial state on the devices (reading S7; bit-identical to the oracle's),
+ * enables peer access between list devices that hold neighbouring chunks.
+ *   s   spread over the i-range; must be exactly range(1 : n0-2), i.e. the loop
+ *       for(i=1; i<n0-1; i++) (coherence is checked, unlike the paper).
+ *       The descriptor is copied; `s` may be destroyed afterwards.
+ *   p   parameters (copied).
+ * Errors: EINVAL (params, range mismatch, chunk too thin: every chunk must own >= 1
+ * plane), ENODEV (device id >= cudaGetDeviceCount), ENOMEM, ECUDA.
+ */
+spread_status somier_init(spread_t s, const somier_params* p, somier_t* out);
+
+/*
+ * somier_init_local -- multi-process mode (one process per GPU): this handle owns
+ * only the chunks at list position `device_pos` of `s`, on CUDA device
+ * `cuda_device` of this process (-1: the id the list gives for that position;
+ * pass the local ordinal when each process sees its GPU under another index,
+ * e.g. with CUDA_VISIBLE_DEVICES). Chunks owned by other processes are reached
+ * after somier_ipc_export / somier_ipc_connect; until then somier_step returns
+ * ESTATE if a neighbour chunk is remote. somier_load is collective in this mode:
+ * every process must load (and the caller must barrier) before anyone steps.
+ */
+spread_status somier_init_local(spread_t s, const somier_params* p, int device_pos, int cuda_device,
+                                somier_t* out);
+
+/*
+ * somier_ipc_export -- serialise the CUDA IPC handles of this handle's halo slots
+ * and exchange flags into buf (capacity cap bytes); *len receives the size used
+ * (call with buf == NULL to query). The blob is opaque and position-independent.
+ */
+spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len);
+
+/*
+ * somier_ipc_connect -- import the blobs of all processes (including this one,
+ * which is skipped), open the handles of the remote neighbour chunks.
+ * Errors: EINVAL (malformed blob, other spread or params), ECUDA.
+ */
+spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const size_t* lens, int nblobs);
+
+/* Enqueue nsteps >= 0 time steps on every owned chunk; returns after enqueue (nowait). */
+spread_status somier_step(somier_t h, int64_t nsteps);
+
+/* Block until all enqueued work of this handle is complete (taskgroup). */
+spread_status somier_sync(somier_t h);
+
+/*
+ * somier_stats -- blocking; stats after the last completed step, combined over
+ * the chunks THIS handle owns (plus the fixed end planes it holds as halos).
+ * In single-process mode that is the whole grid. In multi-process mode combine
+ * the per-process results with somier_stats_combine.
+ */
+spread_status somier_stats(somier_t h, somier_stats_t* out);
+
+/* Exact, order-independent combination of n partial stats (sums added as int128,
+ * max of vmax2 bits); recomputes centre = sum * 2^-60 / N_total and vmax. */
+spread_status somier_stats_combine(const somier_stats_t* parts, int n, const somier_params* p,
+                                   somier_stats_t* out);
+
+/*
+ * somier_read -- exit-data semantics A[start:size]: copy the
+ * owned planes of every chunk of this handle (and the fixed planes 0 / n0-1 held
+ * as halos by the first / last chunk) into caller-owned host grids of n0*n1*n2
+ * doubles each, index (i*n1 + j)*n2 + k, three separate grids per variable
+ * (PAPER.md:342). Planes owned by other processes are left untouched. Blocking.
+ * Any of the six pointers may be NULL to skip that grid.
+ */
+spread_status somier_read(somier_t h, double* x, double* y, double* z, double* vx, double* vy, double* vz);
+
+/*
+ * somier_load -- update-to semantics: every owned chunk copies X[start-1 : size+2]
+ * (with halos) and V[start : size] from caller-owned host grids (layout as in
+ * somier_read) into device memory, and the step counter continues. Enqueued on
+ * the handle's streams (asynchronous w.r.t. the host if the host memory is
+ * pinned). All six pointers are required.
+ */
+spread_status somier_load(somier_t h, const double* x, const double* y, const double* z, const double* vx,
+                          const double* vy, const double* vz);
+
+/* Use `stream` (a cudaStream_t of the device at list position device_pos) for all
+ * work of that device. NULL restores the library's own stream. */
+spread_status somier_set_stream(somier_t h, int device_pos, void* stream);
+spread_status somier_get_stream(somier_t h, int device_pos, void** stream);
+
+/* Number of completed + enqueued steps. */
+spread_status somier_step_count(somier_t h, int64_t* steps);
+
+/* Number of chunks this handle owns, and K1 launches enqueued so far. */
+spread_status somier_local_chunks(somier_t h, int64_t* nchunks);
+spread_status somier_launch_count(somier_t h, int64_t* launches);
+
+/* Device bytes this handle allocated (all devices). */
+spread_status somier_device_bytes(somier_t h, int64_t* bytes);
+
+spread_status somier_destroy(somier_t h);
+
+/* Library version string. */
+const char* somier_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PAPER_SOMIER_H */

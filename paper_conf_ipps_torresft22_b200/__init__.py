@@ -1,0 +1,19 @@
+"""paper_conf_ipps_torresft22_b200 -- B200-native Somier "target spread" step.
+
+The data-parallel hot path of Torres, Ferrer, Teruel (IPDPSW 2022): the Somier
+spring-lattice time step (§V) spread over the GPUs of one node with a
+static round-robin schedule (§III-B). C ABI: include/spread.h and
+include/somier.h, implemented by libsomier.so (hand-written sm_100a kernels).
+This package is the Python binding (argument marshalling only).
+"""
+from . import _native
+from ._native import K1_AUTO, K1_DIRECT, K1_MARCH, SpreadError
+from .somier import Somier, SomierParams, Stats, combine_stats
+from .spread import Chunk, Spread
+
+__all__ = ["Spread", "Chunk", "Somier", "SomierParams", "Stats", "combine_stats", "SpreadError",
+           "K1_AUTO", "K1_DIRECT", "K1_MARCH", "version"]
+
+
+def version() -> str:
+    return _native.lib().somier_version().decode()

@@ -1,0 +1,126 @@
+"""ctypes binding of libsomier.so (include/spread.h, include/somier.h).
+
+Argument marshalling only: every step of the path runs in the library's CUDA
+kernels. There is no fallback -- if libsomier.so is missing or fails to load,
+import raises (build it with `python -m paper_conf_ipps_torresft22_b200.build`
+or __graft_entry__.build()).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsomier.so")
+
+# spread_status
+OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
+# spread_map_type
+MAP_ALLOC, MAP_TO, MAP_FROM, MAP_TOFROM = 0, 1, 2, 3
+# somier_kernel
+K1_AUTO, K1_DIRECT, K1_MARCH = 0, 1, 2
+
+
+class SpreadError(RuntimeError):
+    def __init__(self, status: int, where: str, message: str):
+        super().__init__("%s: %s (%s)" % (where, message, status_string(status)))
+        self.status = status
+
+
+class spread_map(ctypes.Structure):
+    _fields_ = [("type", ctypes.c_int), ("lo_halo", ctypes.c_int64), ("hi_halo", ctypes.c_int64)]
+
+
+class somier_params(ctypes.Structure):
+    _fields_ = [
+        ("n", ctypes.c_int64 * 3),
+        ("spacing", ctypes.c_double),
+        ("rest_len", ctypes.c_double),
+        ("k_spring", ctypes.c_double),
+        ("mass", ctypes.c_double),
+        ("dt", ctypes.c_double),
+        ("amplitude", ctypes.c_double),
+        ("seed", ctypes.c_uint64),
+        ("kernel", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
+    ]
+
+
+class somier_stats_t(ctypes.Structure):
+    _fields_ = [
+        ("step", ctypes.c_int64),
+        ("centre", ctypes.c_double * 3),
+        ("vmax", ctypes.c_double),
+        ("sum_lo", ctypes.c_uint64 * 3),
+        ("sum_hi", ctypes.c_int64 * 3),
+        ("vmax2_bits", ctypes.c_uint64),
+        ("nodes", ctypes.c_int64),
+    ]
+
+
+_lib = None
+
+# (name, restype, argtypes): every symbol include/*.h declares.
+_I64P = ctypes.POINTER(ctypes.c_int64)
+_IP = ctypes.POINTER(ctypes.c_int)
+_VP = ctypes.c_void_p
+_DP = ctypes.POINTER(ctypes.c_double)
+SIGNATURES = [
+    ("spread_create", ctypes.c_int, [_IP, ctypes.c_int, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_int64,
+                                     ctypes.POINTER(_VP)]),
+    ("spread_destroy", ctypes.c_int, [_VP]),
+    ("spread_num_chunks", ctypes.c_int, [_VP, _I64P]),
+    ("spread_num_devices", ctypes.c_int, [_VP, _IP]),
+    ("spread_device", ctypes.c_int, [_VP, ctypes.c_int, _IP]),
+    ("spread_chunk_size", ctypes.c_int, [_VP, _I64P]),
+    ("spread_range", ctypes.c_int, [_VP, _I64P, _I64P]),
+    ("spread_get_chunk", ctypes.c_int, [_VP, ctypes.c_int64, _IP, _IP, _I64P, _I64P]),
+    ("spread_chunk_of", ctypes.c_int, [_VP, ctypes.c_int64, _I64P]),
+    ("spread_map_extent", ctypes.c_int, [_VP, ctypes.c_int64, spread_map, ctypes.c_int64, _I64P, _I64P]),
+    ("spread_last_error", ctypes.c_char_p, []),
+    ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
+    ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),
+    ("somier_init_local", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.c_int, ctypes.c_int,
+                                         ctypes.POINTER(_VP)]),
+    ("somier_ipc_export", ctypes.c_int, [_VP, _VP, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]),
+    ("somier_ipc_connect", ctypes.c_int, [_VP, ctypes.POINTER(_VP), ctypes.POINTER(ctypes.c_size_t), ctypes.c_int]),
+    ("somier_step", ctypes.c_int, [_VP, ctypes.c_int64]),
+    ("somier_sync", ctypes.c_int, [_VP]),
+    ("somier_stats", ctypes.c_int, [_VP, ctypes.POINTER(somier_stats_t)]),
+    ("somier_stats_combine", ctypes.c_int, [ctypes.POINTER(somier_stats_t), ctypes.c_int,
+                                            ctypes.POINTER(somier_params), ctypes.POINTER(somier_stats_t)]),
+    ("somier_read", ctypes.c_int, [_VP] + [_DP] * 6),
+    ("somier_load", ctypes.c_int, [_VP] + [_DP] * 6),
+    ("somier_set_stream", ctypes.c_int, [_VP, ctypes.c_int, _VP]),
+    ("somier_get_stream", ctypes.c_int, [_VP, ctypes.c_int, ctypes.POINTER(_VP)]),
+    ("somier_step_count", ctypes.c_int, [_VP, _I64P]),
+    ("somier_local_chunks", ctypes.c_int, [_VP, _I64P]),
+    ("somier_launch_count", ctypes.c_int, [_VP, _I64P]),
+    ("somier_device_bytes", ctypes.c_int, [_VP, _I64P]),
+    ("somier_destroy", ctypes.c_int, [_VP]),
+    ("somier_version", ctypes.c_char_p, []),
+]
+
+
+def lib() -> ctypes.CDLL:
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError("libsomier.so not built at %s: run __graft_entry__.build() "
+                              "(there is no CPU fallback)" % LIB_PATH)
+        L = ctypes.CDLL(LIB_PATH)
+        for name, res, args in SIGNATURES:
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+def status_string(st: int) -> str:
+    return lib().spread_status_string(st).decode()
+
+
+def check(st: int, where: str) -> None:
+    if st != OK:
+        raise SpreadError(st, where, lib().spread_last_error().decode())

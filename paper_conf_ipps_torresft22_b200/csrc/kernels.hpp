@@ -1,0 +1,68 @@
+// kernels.hpp -- launch wrappers of the sm_100a kernels (host-callable).
+//
+// Slab layout of one chunk: positions X are two buffers (t and
+// t+1) of (size+2) planes, plane p <-> global i = start-1+p (planes 0 and
+// size+1 are the halo planes of the map A[start-1 : size+2]);
+// velocities V are `size` planes, plane p <-> global i = start+p. A plane is
+// three component-planar n1 x ld blocks (x, then y, then z), each row
+// ld >= n2 doubles (ld a multiple of 32: 256-byte aligned rows).
+#pragma once
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "stats_layout.hpp"
+
+namespace paper {
+
+struct SlabGeom {
+    int64_t n0, n1, n2;  // global grid
+    int64_t ld;          // row pitch in doubles
+    int64_t start;       // global i of the first owned plane (omp_spread_start)
+    int64_t size;        // owned planes (omp_spread_size)
+
+    __host__ __device__ int64_t comp_stride() const { return n1 * ld; }
+    __host__ __device__ int64_t plane_stride() const { return 3 * n1 * ld; }
+};
+
+struct StepArgs {
+    const double* x_cur;    // X_t slab (size+2 planes)
+    double* x_nxt;          // X_{t+1} slab (size+2 planes)
+    double* v;              // V slab (size planes), updated in place
+    double* lo_dst;         // left neighbour's hi-halo plane in ITS X_{t+1} buffer, or null
+    double* hi_dst;         // right neighbour's lo-halo plane in ITS X_{t+1} buffer, or null
+    SlabGeom g;
+    double K, L, M, dt;
+    StatsAccum* acc;        // this step's stats slot (accumulated)
+    StatsAccum* acc_clear;  // the next step's slot (zeroed by block 0)
+    // Completion signal for neighbours on other streams (fused exchange): the
+    // last CTA stores `signal_value` with release semantics at system scope
+    // into each non-null flag after every CTA's halo stores are fenced.
+    unsigned long long* signal_lo;   // left neighbour's "from_right" flag
+    unsigned long long* signal_hi;   // right neighbour's "from_left" flag
+    unsigned long long signal_value;
+    unsigned int* done_counter;      // per-chunk CTA completion counter (self-resetting)
+    // K1_MARCH: host pointers to the CUtensorMaps of x_cur and v (passed to the
+    // kernel by value as __grid_constant__ parameters).
+    const void* tmap_x_cur;
+    const void* tmap_v;
+};
+
+struct InitArgs {
+    double* x0;  // both X buffers, all size+2 planes
+    double* x1;
+    SlabGeom g;
+    double spacing, amplitude;
+    uint64_t seed;
+};
+
+enum class K1Variant { Direct = 1, March = 2 };
+
+cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cudaStream_t stream);
+cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
+// Stats of planes [p0, p0+np) of an X slab (plane index inside the slab) and,
+// if v != null, of V planes [p0-1, ...) (V has no halo planes).
+cudaError_t launch_stats(const double* x_slab, const double* v_slab, const SlabGeom& g, int64_t p0, int64_t np,
+                         StatsAccum* acc, cudaStream_t stream);
+
+}  // namespace paper

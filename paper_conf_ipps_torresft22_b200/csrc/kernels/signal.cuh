@@ -1,0 +1,37 @@
+// signal.cuh -- completion signal of the fused halo exchange. Every CTA that
+// stored into a neighbour's halo fences at system scope; the last CTA of the
+// launch to finish publishes the step number to the neighbours' flags with a
+// release store. The neighbour's stream waits on the flag (cuStreamWaitValue64,
+// no SM spinning) before its next step, which both makes the halo visible (RAW)
+// and proves this step no longer reads the neighbour's halo buffer (WAR).
+#pragma once
+#include "../kernels.hpp"
+
+namespace paper {
+
+__device__ __forceinline__ void st_release_sys_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Call once per CTA, by all threads, after the CTA's last store.
+__device__ __forceinline__ void signal_neighbours(const StepArgs& a) {
+    if (!a.signal_lo && !a.signal_hi) return;
+    __shared__ unsigned int s_last;
+    __syncthreads();
+    const bool leader = threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0;
+    if (leader) {
+        __threadfence_system();
+        const unsigned int nblocks = gridDim.x * gridDim.y * gridDim.z;
+        const unsigned int prev = atomicAdd(a.done_counter, 1u);
+        s_last = (prev == nblocks - 1) ? 1u : 0u;
+    }
+    __syncthreads();
+    if (leader && s_last) {
+        __threadfence_system();
+        *a.done_counter = 0u;  // self-reset for the next step (stream-ordered)
+        if (a.signal_lo) st_release_sys_u64(a.signal_lo, a.signal_value);
+        if (a.signal_hi) st_release_sys_u64(a.signal_hi, a.signal_value);
+    }
+}
+
+}  // namespace paper

@@ -1,0 +1,765 @@
+// somier.cpp -- the Somier driver behind include/somier.h: per-chunk slabs on
+// the devices of a spread, the step loop with the fused halo exchange, exact
+// stats combination, map-to / map-from copies, and CUDA IPC for one process per
+// GPU. PAPER.md §V (319-344) for the method; §III-B (79-243) for the clauses
+// whose semantics the calls follow (see include/somier.h).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "kernels.hpp"
+#include "somier.h"
+#include "spread_impl.hpp"
+#include "status.hpp"
+
+using paper::set_last_error;
+
+namespace {
+
+constexpr uint64_t kIpcMagic = 0x534f4d4945524950ull;  // "SOMIERIP"
+constexpr uint32_t kIpcVersion = 1;
+
+using PFN_waitValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+using PFN_encodeTiled = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                     const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                     CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+struct DevCtx {
+    int device = -1;
+    cudaStream_t own = nullptr;   // created by the library
+    cudaStream_t stream = nullptr;  // in use (own or user-provided)
+};
+
+// One chunk = one `target spread` iteration block (omp_spread_start/size).
+struct Chunk {
+    int64_t index = 0, start = 0, size = 0;
+    int pos = 0, device = 0;
+    bool local = false;
+    // local allocation: [x0 | x1 | v | acc[3] | flags[2] | counter]
+    void* base = nullptr;
+    size_t bytes = 0;
+    size_t off_x[2] = {0, 0}, off_v = 0, off_acc = 0, off_flags = 0, off_counter = 0;
+    // remote view (IPC-opened), for non-local neighbours
+    void* remote_base = nullptr;
+    // TMA descriptors of the local slabs (K1_MARCH): X buffers 0/1 and V
+    alignas(64) CUtensorMap tmap_x[2];
+    alignas(64) CUtensorMap tmap_v;
+
+    void* mem() const { return local ? base : remote_base; }
+    double* x(int parity) const { return (double*)((char*)mem() + off_x[parity]); }
+    double* v() const { return (double*)((char*)mem() + off_v); }
+    paper::StatsAccum* acc() const { return (paper::StatsAccum*)((char*)mem() + off_acc); }
+    unsigned long long* flags() const { return (unsigned long long*)((char*)mem() + off_flags); }
+    unsigned int* counter() const { return (unsigned int*)((char*)mem() + off_counter); }
+};
+
+struct IpcChunkRecord {
+    int64_t index;
+    uint64_t bytes, off_x0, off_x1, off_v, off_acc, off_flags, off_counter;
+    cudaIpcMemHandle_t handle;
+};
+
+struct IpcHeader {
+    uint64_t magic;
+    uint32_t version;
+    int32_t device_pos;
+    int64_t n[3];
+    int64_t nchunks;
+    int64_t chunk;
+    int64_t nrecords;
+};
+
+size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+}  // namespace
+
+struct somier_s {
+    somier_params p{};
+    spread_s spread;
+    paper::SlabGeom geom{};  // start/size filled per chunk
+    int64_t ld = 0;
+    int64_t step = 0;
+    int64_t launches = 0;
+    bool multi_process = false;
+    int local_pos = -1;
+    std::vector<Chunk> chunks;
+    std::vector<DevCtx> devs;  // indexed by list position
+    std::string sticky;        // first asynchronous CUDA error
+    PFN_waitValue64 wait_value64 = nullptr;
+    PFN_encodeTiled encode_tiled = nullptr;
+    bool connected = true;
+
+    bool unit_mass() const { return p.mass == 1.0; }
+    paper::K1Variant variant() const {
+        return p.kernel == SOMIER_K1_DIRECT ? paper::K1Variant::Direct : paper::K1Variant::March;
+    }
+    paper::SlabGeom geom_of(const Chunk& c) const {
+        paper::SlabGeom g = geom;
+        g.start = c.start;
+        g.size = c.size;
+        return g;
+    }
+    cudaStream_t stream_of(const Chunk& c) const { return devs[c.pos].stream; }
+    // Neighbour chunks on another stream (other device or other process) need
+    // the flag protocol; same-stream neighbours are ordered by the stream.
+    bool needs_flags(const Chunk& a, const Chunk& b) const {
+        if (!a.local || !b.local) return true;
+        return a.pos != b.pos;
+    }
+};
+
+namespace {
+
+spread_status cuda_fail(somier_t h, cudaError_t e, const char* what) {
+    std::string msg = std::string(what) + ": " + cudaGetErrorString(e);
+    if (h && h->sticky.empty()) h->sticky = msg;
+    set_last_error("%s", msg.c_str());
+    return e == cudaErrorMemoryAllocation ? SPREAD_ENOMEM : SPREAD_ECUDA;
+}
+
+#define CUDA_TRY(h, call)                                         \
+    do {                                                          \
+        cudaError_t e_ = (call);                                  \
+        if (e_ != cudaSuccess) return cuda_fail((h), e_, #call);  \
+    } while (0)
+
+spread_status check_params(const somier_params* p) {
+    if (!p) PAPER_FAIL(SPREAD_EINVAL, "somier: params is NULL");
+    for (int d = 0; d < 3; d++)
+        if (p->n[d] < 3) PAPER_FAIL(SPREAD_EINVAL, "somier: n[%d] = %lld < 3", d, (long long)p->n[d]);
+    const double vals[] = {p->spacing, p->rest_len, p->k_spring, p->mass, p->dt, p->amplitude};
+    for (double v : vals)
+        if (!std::isfinite(v)) PAPER_FAIL(SPREAD_EINVAL, "somier: non-finite parameter");
+    if (!(p->mass > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: mass must be > 0");
+    if (!(p->dt > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: dt must be > 0");
+    if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_MARCH)
+        PAPER_FAIL(SPREAD_EINVAL, "somier: unknown kernel %d", p->kernel);
+    if (p->reserved != 0) PAPER_FAIL(SPREAD_EINVAL, "somier: reserved field must be 0");
+    const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
+    if (n1 > 65535LL * 8 || n0 > 65535 + 2)
+        PAPER_FAIL(SPREAD_EINVAL, "somier: grid too large for the launch geometry");
+    (void)n2;
+    return SPREAD_OK;
+}
+
+spread_status load_driver_entry(somier_t h) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaError_t e = cudaGetDriverEntryPoint("cuStreamWaitValue64", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+        PAPER_FAIL(SPREAD_ECUDA, "somier: cuStreamWaitValue64 unavailable (%s)", cudaGetErrorString(e));
+    h->wait_value64 = (PFN_waitValue64)fn;
+    fn = nullptr;
+    e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+        PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled unavailable (%s)", cudaGetErrorString(e));
+    h->encode_tiled = (PFN_encodeTiled)fn;
+    return SPREAD_OK;
+}
+
+// 4-D fp64 tensor map over a slab: dims (n2, n1, 3 components, planes), row
+// pitch ld. Box = (box_k, box_j, 3, 1): one plane tile per TMA.
+spread_status encode_slab_map(somier_t h, CUtensorMap* map, double* base, int64_t planes, uint32_t box_k,
+                              uint32_t box_j) {
+    const cuuint64_t dims[4] = {(cuuint64_t)h->p.n[2], (cuuint64_t)h->p.n[1], 3, (cuuint64_t)planes};
+    const cuuint64_t strides[3] = {(cuuint64_t)h->ld * 8, (cuuint64_t)(h->p.n[1] * h->ld) * 8,
+                                   (cuuint64_t)(3 * h->p.n[1] * h->ld) * 8};
+    const cuuint32_t box[4] = {box_k, box_j, 3, 1};
+    const cuuint32_t estr[4] = {1, 1, 1, 1};
+    CUresult r = h->encode_tiled(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, base, dims, strides, box, estr,
+                                 CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                                 CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled failed (%d)", (int)r);
+    return SPREAD_OK;
+}
+
+void free_all(somier_t h) {
+    if (!h) return;
+    for (auto& c : h->chunks) {
+        if (c.remote_base) {
+            cudaSetDevice(h->devs[h->local_pos >= 0 ? h->local_pos : 0].device);
+            cudaIpcCloseMemHandle(c.remote_base);
+            c.remote_base = nullptr;
+        }
+    }
+    for (auto& c : h->chunks) {
+        if (c.local && c.base) {
+            cudaSetDevice(c.device);
+            cudaFree(c.base);
+            c.base = nullptr;
+        }
+    }
+    for (auto& d : h->devs) {
+        if (d.own) {
+            cudaSetDevice(d.device);
+            cudaStreamDestroy(d.own);
+            d.own = nullptr;
+        }
+    }
+}
+
+// Recompute the stats slots of a chunk from its resident state: slot (step-1)&1
+// = stats of the current state, slot step&1 zeroed, slot 2 = the fixed end
+// planes the chunk holds as halos (global i = 0 and i = n0-1).
+spread_status reset_stats(somier_t h, Chunk& c) {
+    cudaStream_t s = h->stream_of(c);
+    paper::SlabGeom g = h->geom_of(c);
+    CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 3 * sizeof(paper::StatsAccum), s));
+    const int cur = (int)(h->step & 1);
+    paper::StatsAccum* last = c.acc() + ((h->step - 1) & 1);
+    CUDA_TRY(h, paper::launch_stats(c.x(cur), c.v(), g, 1, c.size, last, s));
+    if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, 0, 1, c.acc() + 2, s));
+    if (c.start + c.size == h->p.n[0] - 1)
+        CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
+    return SPREAD_OK;
+}
+
+spread_status allocate_chunk(somier_t h, Chunk& c) {
+    const paper::SlabGeom g = h->geom_of(c);
+    const size_t plane = (size_t)g.plane_stride() * sizeof(double);
+    const size_t xb = round_up(plane * (size_t)(c.size + 2), 4096);
+    const size_t vb = round_up(plane * (size_t)c.size, 4096);
+    c.off_x[0] = 0;
+    c.off_x[1] = xb;
+    c.off_v = 2 * xb;
+    c.off_acc = c.off_v + vb;
+    c.off_flags = c.off_acc + 3 * sizeof(paper::StatsAccum);
+    c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);
+    c.bytes = round_up(c.off_counter + 64, 4096);
+    CUDA_TRY(h, cudaSetDevice(c.device));
+    CUDA_TRY(h, cudaMalloc(&c.base, c.bytes));
+    cudaStream_t s = h->stream_of(c);
+    CUDA_TRY(h, cudaMemsetAsync(c.base, 0, c.bytes, s));
+    paper::InitArgs ia;
+    ia.x0 = c.x(0);
+    ia.x1 = c.x(1);
+    ia.g = g;
+    ia.spacing = h->p.spacing;
+    ia.amplitude = h->p.amplitude;
+    ia.seed = h->p.seed;
+    CUDA_TRY(h, paper::launch_init(ia, s));
+    for (int b = 0; b < 2; b++) {
+        spread_status st = encode_slab_map(h, &c.tmap_x[b], c.x(b), c.size + 2, 34, 10);
+        if (st != SPREAD_OK) return st;
+    }
+    spread_status st = encode_slab_map(h, &c.tmap_v, c.v(), c.size, 32, 8);
+    if (st != SPREAD_OK) return st;
+    return reset_stats(h, c);
+}
+
+spread_status sync_all(somier_t h) {
+    for (auto& d : h->devs) {
+        if (!d.stream) continue;
+        cudaError_t e = cudaSetDevice(d.device);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(d.stream);
+        if (e != cudaSuccess) return cuda_fail(h, e, "somier_sync");
+    }
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    return SPREAD_OK;
+}
+
+spread_status init_common(spread_t s, const somier_params* p, int local_pos, int cuda_device, somier_t* out) {
+    if (!out) PAPER_FAIL(SPREAD_EINVAL, "somier_init: out is NULL");
+    *out = nullptr;
+    if (!s) PAPER_FAIL(SPREAD_EINVAL, "somier_init: spread is NULL");
+    spread_status st = check_params(p);
+    if (st != SPREAD_OK) return st;
+    // Coherence of the spread with the loop it is applied to (the paper leaves
+    // this to the programmer): for(i=1; i<n0-1; i++).
+    if (s->range_start != 1 || s->range_len != p->n[0] - 2)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_init: spread range (%lld:%lld) must be range(1:%lld), the i-loop [1, n0-1)",
+                   (long long)s->range_start, (long long)s->range_len, (long long)(p->n[0] - 2));
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) PAPER_FAIL(SPREAD_ENODEV, "somier_init: no CUDA device (%s)", cudaGetErrorString(e));
+    const int npos = (int)s->devices.size();
+    if (local_pos >= npos) PAPER_FAIL(SPREAD_EINVAL, "somier_init_local: position %d outside the list", local_pos);
+    for (int q = 0; q < npos; q++) {
+        if (local_pos >= 0 && q != local_pos) continue;
+        const int dev = (q == local_pos && cuda_device >= 0) ? cuda_device : s->devices[q];
+        if (dev >= ndev) PAPER_FAIL(SPREAD_ENODEV, "somier_init: device %d not present (%d visible)", dev, ndev);
+    }
+
+    somier_s* h = new (std::nothrow) somier_s;
+    if (!h) PAPER_FAIL(SPREAD_ENOMEM, "somier_init: out of host memory");
+    h->p = *p;
+    h->spread = *s;
+    h->multi_process = local_pos >= 0;
+    h->local_pos = local_pos;
+    h->ld = (int64_t)round_up((size_t)p->n[2], 32);
+    h->geom = paper::SlabGeom{p->n[0], p->n[1], p->n[2], h->ld, 0, 0};
+    h->devs.resize(npos);
+    for (int q = 0; q < npos; q++) h->devs[q].device = s->devices[q];
+    if (local_pos >= 0 && cuda_device >= 0) h->devs[local_pos].device = cuda_device;
+    h->chunks.resize(s->nchunks);
+    for (int64_t c = 0; c < s->nchunks; c++) {
+        paper::ChunkInfo ci = s->chunk_info(c);
+        Chunk& ch = h->chunks[c];
+        ch.index = c;
+        ch.start = ci.start;
+        ch.size = ci.size;
+        ch.pos = ci.pos;
+        ch.device = h->devs[ci.pos].device;
+        ch.local = (local_pos < 0) || (ci.pos == local_pos);
+    }
+    st = load_driver_entry(h);
+    if (st != SPREAD_OK) {
+        delete h;
+        return st;
+    }
+    auto fail = [&](spread_status code) {
+        std::string msg = paper::last_error();
+        free_all(h);
+        delete h;
+        set_last_error("%s", msg.c_str());
+        return code;
+    };
+    // streams for every list position that owns a local chunk
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        DevCtx& d = h->devs[c.pos];
+        if (d.own) continue;
+        if ((e = cudaSetDevice(d.device)) != cudaSuccess ||
+            (e = cudaStreamCreateWithFlags(&d.own, cudaStreamNonBlocking)) != cudaSuccess) {
+            cuda_fail(h, e, "somier_init: stream");
+            return fail(SPREAD_ECUDA);
+        }
+        d.stream = d.own;
+    }
+    // peer access between devices holding neighbouring local chunks
+    for (size_t c = 0; c + 1 < h->chunks.size(); c++) {
+        const Chunk& a = h->chunks[c];
+        const Chunk& b = h->chunks[c + 1];
+        if (!a.local || !b.local || a.device == b.device) continue;
+        for (int dir = 0; dir < 2; dir++) {
+            int from = dir ? b.device : a.device, to = dir ? a.device : b.device;
+            int can = 0;
+            cudaDeviceCanAccessPeer(&can, from, to);
+            if (!can) {
+                set_last_error("somier_init: device %d cannot access device %d (no P2P)", from, to);
+                return fail(SPREAD_ENOTSUP);
+            }
+            cudaSetDevice(from);
+            e = cudaDeviceEnablePeerAccess(to, 0);
+            if (e == cudaErrorPeerAccessAlreadyEnabled) {
+                cudaGetLastError();
+            } else if (e != cudaSuccess) {
+                cuda_fail(h, e, "somier_init: cudaDeviceEnablePeerAccess");
+                return fail(SPREAD_ECUDA);
+            }
+        }
+    }
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        st = allocate_chunk(h, c);
+        if (st != SPREAD_OK) return fail(st);
+    }
+    st = sync_all(h);
+    if (st != SPREAD_OK) return fail(st);
+    // neighbours owned by other processes must be connected before stepping
+    for (size_t c = 0; c < h->chunks.size(); c++) {
+        if (!h->chunks[c].local) continue;
+        if ((c > 0 && !h->chunks[c - 1].local) || (c + 1 < h->chunks.size() && !h->chunks[c + 1].local))
+            h->connected = false;
+    }
+    *out = h;
+    return SPREAD_OK;
+}
+
+int64_t owned_nodes(const somier_s* h, const Chunk& c) {
+    int64_t planes = c.size + (c.start == 1 ? 1 : 0) + (c.start + c.size == h->p.n[0] - 1 ? 1 : 0);
+    return planes * h->p.n[1] * h->p.n[2];
+}
+
+void finish_stats(const somier_params* p, __int128 sums[3], unsigned long long vmax2, int64_t nodes, int64_t step,
+                  somier_stats_t* out) {
+    const double N = (double)(p->n[0] * p->n[1] * p->n[2]);
+    for (int c = 0; c < 3; c++) {
+        out->sum_lo[c] = (uint64_t)(unsigned __int128)sums[c];
+        out->sum_hi[c] = (int64_t)(sums[c] >> 64);
+        out->centre[c] = std::ldexp((double)sums[c], -60) / N;
+    }
+    double v2;
+    std::memcpy(&v2, &vmax2, sizeof v2);
+    out->vmax2_bits = vmax2;
+    out->vmax = std::sqrt(v2);
+    out->nodes = nodes;
+    out->step = step;
+}
+
+// cudaMemcpy3D between a slab (planes of 3 component blocks, row pitch ld) and
+// a host grid of one component (n0 x n1 x n2, dense).
+cudaError_t copy_planes(somier_t h, double* slab, int comp, int64_t slab_plane, double* host, int64_t host_plane,
+                        int64_t nplanes, cudaMemcpyKind kind, cudaStream_t s) {
+    const int64_t n1 = h->p.n[1], n2 = h->p.n[2];
+    cudaMemcpy3DParms m;
+    std::memset(&m, 0, sizeof m);
+    cudaPitchedPtr sp = make_cudaPitchedPtr(slab + comp * n1 * h->ld, (size_t)h->ld * sizeof(double), (size_t)n2,
+                                            (size_t)(3 * n1));
+    cudaPitchedPtr hp = make_cudaPitchedPtr(host, (size_t)n2 * sizeof(double), (size_t)n2, (size_t)n1);
+    if (kind == cudaMemcpyDeviceToHost) {
+        m.srcPtr = sp;
+        m.srcPos = make_cudaPos(0, 0, (size_t)slab_plane);
+        m.dstPtr = hp;
+        m.dstPos = make_cudaPos(0, 0, (size_t)host_plane);
+    } else {
+        m.srcPtr = hp;
+        m.srcPos = make_cudaPos(0, 0, (size_t)host_plane);
+        m.dstPtr = sp;
+        m.dstPos = make_cudaPos(0, 0, (size_t)slab_plane);
+    }
+    m.extent = make_cudaExtent((size_t)n2 * sizeof(double), (size_t)n1, (size_t)nplanes);
+    m.kind = kind;
+    return cudaMemcpy3DAsync(&m, s);
+}
+
+}  // namespace
+
+extern "C" {
+
+spread_status somier_init(spread_t s, const somier_params* p, somier_t* out) {
+    return init_common(s, p, -1, -1, out);
+}
+
+spread_status somier_init_local(spread_t s, const somier_params* p, int device_pos, int cuda_device,
+                                somier_t* out) {
+    if (device_pos < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_init_local: negative device position");
+    return init_common(s, p, device_pos, cuda_device, out);
+}
+
+spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_export: NULL handle");
+    std::vector<IpcChunkRecord> recs;
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        IpcChunkRecord r;
+        std::memset(&r, 0, sizeof r);
+        r.index = c.index;
+        r.bytes = c.bytes;
+        r.off_x0 = c.off_x[0];
+        r.off_x1 = c.off_x[1];
+        r.off_v = c.off_v;
+        r.off_acc = c.off_acc;
+        r.off_flags = c.off_flags;
+        r.off_counter = c.off_counter;
+        CUDA_TRY(h, cudaSetDevice(c.device));
+        CUDA_TRY(h, cudaIpcGetMemHandle(&r.handle, c.base));
+        recs.push_back(r);
+    }
+    IpcHeader hd;
+    std::memset(&hd, 0, sizeof hd);
+    hd.magic = kIpcMagic;
+    hd.version = kIpcVersion;
+    hd.device_pos = h->local_pos;
+    for (int d = 0; d < 3; d++) hd.n[d] = h->p.n[d];
+    hd.nchunks = (int64_t)h->chunks.size();
+    hd.chunk = h->spread.chunk;
+    hd.nrecords = (int64_t)recs.size();
+    const size_t need = sizeof hd + recs.size() * sizeof(IpcChunkRecord);
+    if (len) *len = need;
+    if (!buf) return SPREAD_OK;
+    if (cap < need) PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_export: buffer of %zu bytes < %zu", cap, need);
+    std::memcpy(buf, &hd, sizeof hd);
+    if (!recs.empty()) std::memcpy((char*)buf + sizeof hd, recs.data(), recs.size() * sizeof(IpcChunkRecord));
+    return SPREAD_OK;
+}
+
+spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const size_t* lens, int nblobs) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: NULL handle");
+    if (!h->multi_process) PAPER_FAIL(SPREAD_ESTATE, "somier_ipc_connect: handle is not multi-process");
+    if (nblobs < 0 || (nblobs > 0 && (!blobs || !lens))) PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: bad blob list");
+    std::map<int64_t, IpcChunkRecord> remote;
+    for (int b = 0; b < nblobs; b++) {
+        if (!blobs[b] || lens[b] < sizeof(IpcHeader)) PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d too short", b);
+        IpcHeader hd;
+        std::memcpy(&hd, blobs[b], sizeof hd);
+        if (hd.magic != kIpcMagic || hd.version != kIpcVersion)
+            PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d is not a somier IPC blob", b);
+        if (hd.n[0] != h->p.n[0] || hd.n[1] != h->p.n[1] || hd.n[2] != h->p.n[2] ||
+            hd.nchunks != (int64_t)h->chunks.size() || hd.chunk != h->spread.chunk)
+            PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d describes another grid or spread", b);
+        if (lens[b] != sizeof hd + (size_t)hd.nrecords * sizeof(IpcChunkRecord))
+            PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d has a bad length", b);
+        if (hd.device_pos == h->local_pos) continue;
+        for (int64_t r = 0; r < hd.nrecords; r++) {
+            IpcChunkRecord rec;
+            std::memcpy(&rec, (const char*)blobs[b] + sizeof hd + r * sizeof rec, sizeof rec);
+            if (rec.index < 0 || rec.index >= (int64_t)h->chunks.size())
+                PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: chunk index out of range");
+            remote[rec.index] = rec;
+        }
+    }
+    CUDA_TRY(h, cudaSetDevice(h->devs[h->local_pos].device));
+    for (size_t c = 0; c < h->chunks.size(); c++) {
+        Chunk& me = h->chunks[c];
+        if (!me.local) continue;
+        for (int side = -1; side <= 1; side += 2) {
+            int64_t nb = (int64_t)c + side;
+            if (nb < 0 || nb >= (int64_t)h->chunks.size()) continue;
+            Chunk& o = h->chunks[nb];
+            if (o.local || o.remote_base) continue;
+            auto it = remote.find(nb);
+            if (it == remote.end())
+                PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: no process exported neighbour chunk %lld", (long long)nb);
+            const IpcChunkRecord& rec = it->second;
+            void* ptr = nullptr;
+            CUDA_TRY(h, cudaIpcOpenMemHandle(&ptr, rec.handle, cudaIpcMemLazyEnablePeerAccess));
+            o.remote_base = ptr;
+            o.bytes = rec.bytes;
+            o.off_x[0] = rec.off_x0;
+            o.off_x[1] = rec.off_x1;
+            o.off_v = rec.off_v;
+            o.off_acc = rec.off_acc;
+            o.off_flags = rec.off_flags;
+            o.off_counter = rec.off_counter;
+        }
+    }
+    h->connected = true;
+    return SPREAD_OK;
+}
+
+spread_status somier_step(somier_t h, int64_t nsteps) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_step: NULL handle");
+    if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_step: nsteps < 0");
+    if (!h->connected) PAPER_FAIL(SPREAD_ESTATE, "somier_step: remote neighbour chunks not connected (somier_ipc_connect)");
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    const int64_t nch = (int64_t)h->chunks.size();
+    int cur_dev = -1;
+    for (int64_t s = 0; s < nsteps; s++) {
+        const int64_t t = h->step;
+        const int cur = (int)(t & 1), nxt = cur ^ 1;
+        for (int64_t c = 0; c < nch; c++) {
+            Chunk& me = h->chunks[c];
+            if (!me.local) continue;
+            if (me.device != cur_dev) {
+                CUDA_TRY(h, cudaSetDevice(me.device));
+                cur_dev = me.device;
+            }
+            cudaStream_t st = h->stream_of(me);
+            const Chunk* left = c > 0 ? &h->chunks[c - 1] : nullptr;
+            const Chunk* right = c + 1 < nch ? &h->chunks[c + 1] : nullptr;
+            const bool fl = left && h->needs_flags(me, *left);
+            const bool fr = right && h->needs_flags(me, *right);
+            // wait until the neighbours finished step t-1 (their halo stores into
+            // my X_t are visible, and they no longer read the halo buffer I am
+            // about to write): flags[0] = from_left, flags[1] = from_right.
+            if (t > 0 && fl) {
+                CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[0], (cuuint64_t)t,
+                                             CU_STREAM_WAIT_VALUE_GEQ);
+                if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
+            }
+            if (t > 0 && fr) {
+                CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[1], (cuuint64_t)t,
+                                             CU_STREAM_WAIT_VALUE_GEQ);
+                if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
+            }
+            paper::StepArgs a;
+            std::memset(&a, 0, sizeof a);
+            a.x_cur = me.x(cur);
+            a.x_nxt = me.x(nxt);
+            a.v = me.v();
+            a.lo_dst = left ? left->x(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
+            a.hi_dst = right ? right->x(nxt) : nullptr;
+            a.g = h->geom_of(me);
+            a.K = h->p.k_spring;
+            a.L = h->p.rest_len;
+            a.M = h->p.mass;
+            a.dt = h->p.dt;
+            a.acc = me.acc() + cur;
+            a.acc_clear = me.acc() + nxt;
+            a.signal_lo = fl ? &left->flags()[1] : nullptr;
+            a.signal_hi = fr ? &right->flags()[0] : nullptr;
+            a.signal_value = (unsigned long long)(t + 1);
+            a.done_counter = me.counter();
+            a.tmap_x_cur = &me.tmap_x[cur];
+            a.tmap_v = &me.tmap_v;
+            CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
+            h->launches++;
+        }
+        h->step++;
+    }
+    return SPREAD_OK;
+}
+
+spread_status somier_sync(somier_t h) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_sync: NULL handle");
+    return sync_all(h);
+}
+
+spread_status somier_stats(somier_t h, somier_stats_t* out) {
+    if (!h || !out) PAPER_FAIL(SPREAD_EINVAL, "somier_stats: NULL argument");
+    spread_status st = sync_all(h);
+    if (st != SPREAD_OK) return st;
+    __int128 sums[3] = {0, 0, 0};
+    unsigned long long vmax2 = 0;
+    int64_t nodes = 0;
+    const int slot = (int)((h->step - 1) & 1);
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        paper::StatsAccum acc[3];
+        CUDA_TRY(h, cudaSetDevice(c.device));
+        CUDA_TRY(h, cudaMemcpy(acc, c.acc(), sizeof acc, cudaMemcpyDeviceToHost));
+        for (int q : {slot, 2}) {
+            for (int d = 0; d < 3; d++)
+                sums[d] += (__int128)(((unsigned __int128)acc[q].hi[d] << 64) | acc[q].lo[d]);
+            vmax2 = std::max(vmax2, (unsigned long long)acc[q].vmax2);
+        }
+        nodes += owned_nodes(h, c);
+    }
+    finish_stats(&h->p, sums, vmax2, nodes, h->step, out);
+    return SPREAD_OK;
+}
+
+spread_status somier_stats_combine(const somier_stats_t* parts, int n, const somier_params* p, somier_stats_t* out) {
+    if (!parts || n < 1 || !p || !out) PAPER_FAIL(SPREAD_EINVAL, "somier_stats_combine: bad arguments");
+    __int128 sums[3] = {0, 0, 0};
+    unsigned long long vmax2 = 0;
+    int64_t nodes = 0;
+    for (int i = 0; i < n; i++) {
+        if (parts[i].step != parts[0].step)
+            PAPER_FAIL(SPREAD_EINVAL, "somier_stats_combine: partials of different steps");
+        for (int d = 0; d < 3; d++)
+            sums[d] += (__int128)(((unsigned __int128)(uint64_t)parts[i].sum_hi[d] << 64) | parts[i].sum_lo[d]);
+        vmax2 = std::max(vmax2, (unsigned long long)parts[i].vmax2_bits);
+        nodes += parts[i].nodes;
+    }
+    finish_stats(p, sums, vmax2, nodes, parts[0].step, out);
+    return SPREAD_OK;
+}
+
+spread_status somier_read(somier_t h, double* x, double* y, double* z, double* vx, double* vy, double* vz) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_read: NULL handle");
+    spread_status st = sync_all(h);
+    if (st != SPREAD_OK) return st;
+    double* X[3] = {x, y, z};
+    double* V[3] = {vx, vy, vz};
+    const int cur = (int)(h->step & 1);
+    const int64_t n0 = h->p.n[0];
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        CUDA_TRY(h, cudaSetDevice(c.device));
+        cudaStream_t s = h->stream_of(c);
+        for (int d = 0; d < 3; d++) {
+            if (X[d]) {
+                CUDA_TRY(h, copy_planes(h, c.x(cur), d, 1, X[d], c.start, c.size, cudaMemcpyDeviceToHost, s));
+                if (c.start == 1) CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, X[d], 0, 1, cudaMemcpyDeviceToHost, s));
+                if (c.start + c.size == n0 - 1)
+                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, c.size + 1, X[d], n0 - 1, 1, cudaMemcpyDeviceToHost, s));
+            }
+            if (V[d]) {
+                CUDA_TRY(h, copy_planes(h, c.v(), d, 0, V[d], c.start, c.size, cudaMemcpyDeviceToHost, s));
+                // fixed end planes have zero velocity
+                const size_t plane = (size_t)(h->p.n[1] * h->p.n[2]);
+                if (c.start == 1) std::memset(V[d], 0, plane * sizeof(double));
+                if (c.start + c.size == n0 - 1) std::memset(V[d] + (size_t)(n0 - 1) * plane, 0, plane * sizeof(double));
+            }
+        }
+    }
+    return sync_all(h);
+}
+
+spread_status somier_load(somier_t h, const double* x, const double* y, const double* z, const double* vx,
+                          const double* vy, const double* vz) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_load: NULL handle");
+    if (!x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_load: NULL grid");
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    const double* X[3] = {x, y, z};
+    const double* V[3] = {vx, vy, vz};
+    const int cur = (int)(h->step & 1);
+    for (auto& c : h->chunks) {
+        if (!c.local) continue;
+        CUDA_TRY(h, cudaSetDevice(c.device));
+        cudaStream_t s = h->stream_of(c);
+        for (int d = 0; d < 3; d++) {
+            CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, const_cast<double*>(X[d]), c.start - 1, c.size + 2,
+                                    cudaMemcpyHostToDevice, s));
+            CUDA_TRY(h, copy_planes(h, c.v(), d, 0, const_cast<double*>(V[d]), c.start, c.size,
+                                    cudaMemcpyHostToDevice, s));
+        }
+        // the X_{t+1} buffer must hold the same fixed nodes (never written by a step)
+        CUDA_TRY(h, cudaMemcpyAsync(c.x(cur ^ 1), c.x(cur), c.off_x[1] - c.off_x[0], cudaMemcpyDeviceToDevice, s));
+        spread_status st = reset_stats(h, c);
+        if (st != SPREAD_OK) return st;
+    }
+    return SPREAD_OK;
+}
+
+spread_status somier_set_stream(somier_t h, int device_pos, void* stream) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_set_stream: NULL handle");
+    if (device_pos < 0 || device_pos >= (int)h->devs.size() || !h->devs[device_pos].own)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_set_stream: no local chunk at list position %d", device_pos);
+    DevCtx& d = h->devs[device_pos];
+    cudaStream_t next = stream ? (cudaStream_t)stream : d.own;
+    if (next != d.stream) {
+        // order the new stream after everything already enqueued on the old one
+        cudaEvent_t ev;
+        CUDA_TRY(h, cudaSetDevice(d.device));
+        CUDA_TRY(h, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        CUDA_TRY(h, cudaEventRecord(ev, d.stream));
+        CUDA_TRY(h, cudaStreamWaitEvent(next, ev, 0));
+        CUDA_TRY(h, cudaEventDestroy(ev));
+        d.stream = next;
+    }
+    return SPREAD_OK;
+}
+
+spread_status somier_get_stream(somier_t h, int device_pos, void** stream) {
+    if (!h || !stream) PAPER_FAIL(SPREAD_EINVAL, "somier_get_stream: NULL argument");
+    if (device_pos < 0 || device_pos >= (int)h->devs.size() || !h->devs[device_pos].own)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_get_stream: no local chunk at list position %d", device_pos);
+    *stream = (void*)h->devs[device_pos].stream;
+    return SPREAD_OK;
+}
+
+spread_status somier_step_count(somier_t h, int64_t* steps) {
+    if (!h || !steps) PAPER_FAIL(SPREAD_EINVAL, "somier_step_count: NULL argument");
+    *steps = h->step;
+    return SPREAD_OK;
+}
+
+spread_status somier_local_chunks(somier_t h, int64_t* nchunks) {
+    if (!h || !nchunks) PAPER_FAIL(SPREAD_EINVAL, "somier_local_chunks: NULL argument");
+    int64_t n = 0;
+    for (auto& c : h->chunks) n += c.local ? 1 : 0;
+    *nchunks = n;
+    return SPREAD_OK;
+}
+
+spread_status somier_launch_count(somier_t h, int64_t* launches) {
+    if (!h || !launches) PAPER_FAIL(SPREAD_EINVAL, "somier_launch_count: NULL argument");
+    *launches = h->launches;
+    return SPREAD_OK;
+}
+
+spread_status somier_device_bytes(somier_t h, int64_t* bytes) {
+    if (!h || !bytes) PAPER_FAIL(SPREAD_EINVAL, "somier_device_bytes: NULL argument");
+    int64_t b = 0;
+    for (auto& c : h->chunks)
+        if (c.local) b += (int64_t)c.bytes;
+    *bytes = b;
+    return SPREAD_OK;
+}
+
+spread_status somier_destroy(somier_t h) {
+    if (!h) return SPREAD_OK;
+    for (auto& d : h->devs)
+        if (d.stream) {
+            cudaSetDevice(d.device);
+            cudaStreamSynchronize(d.stream);
+        }
+    free_all(h);
+    delete h;
+    return SPREAD_OK;
+}
+
+const char* somier_version(void) { return "somier-spread 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,41 @@
+// spread_impl.hpp -- the descriptor behind the opaque spread_t.
+#pragma once
+#include <cstdint>
+#include <vector>
+
+#include "spread.h"
+
+namespace paper {
+
+struct ChunkInfo {
+    int64_t index;   // chunk number c
+    int pos;         // list position (c mod ndevices): distribution order
+    int device;      // device id at that position
+    int64_t start;   // omp_spread_start
+    int64_t size;    // omp_spread_size
+};
+
+const char* last_error();
+
+}  // namespace paper
+
+struct spread_s {
+    std::vector<int> devices;
+    int64_t range_start = 0;
+    int64_t range_len = 0;
+    int64_t chunk = 1;
+    int64_t nchunks = 0;
+
+    // Static round-robin: chunk c covers iterations
+    // [start + c*chunk, min(start + (c+1)*chunk, start + len)) on list position c mod p.
+    paper::ChunkInfo chunk_info(int64_t c) const {
+        paper::ChunkInfo ci;
+        ci.index = c;
+        ci.pos = (int)(c % (int64_t)devices.size());
+        ci.device = devices[ci.pos];
+        ci.start = range_start + c * chunk;
+        int64_t end = range_start + range_len;
+        ci.size = (ci.start + chunk <= end) ? chunk : end - ci.start;
+        return ci;
+    }
+};

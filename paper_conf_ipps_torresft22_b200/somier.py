@@ -1,0 +1,214 @@
+"""The Somier time step spread over devices (include/somier.h; §V).
+
+A thin ctypes layer: parameters in, pointers and sizes across the C ABI, and
+numpy views out. The step itself runs in libsomier.so's sm_100a kernels.
+"""
+from __future__ import annotations
+
+import ctypes
+import dataclasses
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+
+from . import _native as N
+from .spread import Spread
+
+
+@dataclasses.dataclass
+class SomierParams:
+    """Defaults are DESIGN.md §3 reading S3."""
+
+    n: Tuple[int, int, int] = (16, 16, 16)
+    spacing: float = 1.0
+    rest_len: float = 1.0
+    k_spring: float = 10.0
+    mass: float = 1.0
+    dt: float = 1e-3
+    amplitude: float = 0.05
+    seed: int = 42
+    kernel: int = N.K1_AUTO
+
+    def c(self) -> N.somier_params:
+        p = N.somier_params()
+        for d in range(3):
+            p.n[d] = int(self.n[d])
+        p.spacing, p.rest_len, p.k_spring, p.mass = self.spacing, self.rest_len, self.k_spring, self.mass
+        p.dt, p.amplitude, p.seed, p.kernel, p.reserved = self.dt, self.amplitude, int(self.seed), int(self.kernel), 0
+        return p
+
+    @property
+    def interior_nodes(self) -> int:
+        return (self.n[0] - 2) * (self.n[1] - 2) * (self.n[2] - 2)
+
+
+@dataclasses.dataclass
+class Stats:
+    step: int
+    centre: Tuple[float, float, float]
+    vmax: float
+    sums: Tuple[int, int, int]    # exact int128 fixed-point sums, units of 2^-60
+    vmax2_bits: int
+    nodes: int
+
+    @staticmethod
+    def from_c(s: N.somier_stats_t) -> "Stats":
+        sums = tuple((int(s.sum_hi[c]) << 64) | int(s.sum_lo[c]) for c in range(3))
+        return Stats(int(s.step), tuple(s.centre), float(s.vmax), sums, int(s.vmax2_bits), int(s.nodes))
+
+    def to_c(self) -> N.somier_stats_t:
+        s = N.somier_stats_t()
+        s.step = self.step
+        for c in range(3):
+            s.centre[c] = self.centre[c]
+            v = self.sums[c] & ((1 << 128) - 1)
+            s.sum_lo[c] = v & ((1 << 64) - 1)
+            hi = v >> 64
+            s.sum_hi[c] = hi - (1 << 64) if hi >= (1 << 63) else hi
+        s.vmax = self.vmax
+        s.vmax2_bits = self.vmax2_bits
+        s.nodes = self.nodes
+        return s
+
+
+def _dptr(a) -> ctypes.POINTER(ctypes.c_double):
+    """numpy float64 C-contiguous array, or an integer address (e.g. a pinned torch tensor's data_ptr())."""
+    if a is None:
+        return None
+    if isinstance(a, int):
+        return ctypes.cast(ctypes.c_void_p(a), ctypes.POINTER(ctypes.c_double))
+    if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags["C_CONTIGUOUS"]):
+        raise TypeError("expected a C-contiguous float64 numpy array or an address")
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+
+
+def combine_stats(parts: Sequence[Stats], params: SomierParams) -> Stats:
+    """Exact combination of per-process partial stats (somier_stats_combine)."""
+    arr = (N.somier_stats_t * len(parts))(*[p.to_c() for p in parts])
+    out = N.somier_stats_t()
+    pc = params.c()
+    N.check(N.lib().somier_stats_combine(arr, len(parts), ctypes.byref(pc), ctypes.byref(out)),
+            "somier_stats_combine")
+    return Stats.from_c(out)
+
+
+class Somier:
+    """A Somier grid spread over the devices of `spread`.
+
+    device_pos=None: single-process mode (all chunks, all devices of the list).
+    device_pos=q: multi-process mode, this process owns the chunks at list
+    position q; call ipc_connect() with every process's ipc_export() blob.
+    """
+
+    def __init__(self, spread: Spread, params: SomierParams, device_pos: Optional[int] = None,
+                 cuda_device: int = -1):
+        L = N.lib()
+        self.params = params
+        self.spread = spread
+        self._pc = params.c()
+        h = ctypes.c_void_p()
+        if device_pos is None:
+            N.check(L.somier_init(spread.handle, ctypes.byref(self._pc), ctypes.byref(h)), "somier_init")
+        else:
+            N.check(L.somier_init_local(spread.handle, ctypes.byref(self._pc), int(device_pos), int(cuda_device),
+                                        ctypes.byref(h)), "somier_init_local")
+        self._h = h
+        self.device_pos = device_pos
+
+    # -- lifetime ------------------------------------------------------------
+    def close(self) -> None:
+        if getattr(self, "_h", None):
+            N.lib().somier_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # -- the step ------------------------------------------------------------
+    def step(self, nsteps: int = 1) -> None:
+        N.check(N.lib().somier_step(self._h, int(nsteps)), "somier_step")
+
+    def sync(self) -> None:
+        N.check(N.lib().somier_sync(self._h), "somier_sync")
+
+    def stats(self) -> Stats:
+        out = N.somier_stats_t()
+        N.check(N.lib().somier_stats(self._h, ctypes.byref(out)), "somier_stats")
+        return Stats.from_c(out)
+
+    # -- data movement -------------------------------------------------------
+    def read(self, X=None, V=None):
+        """Copy the owned planes into host grids; returns (X, V), each (3, n0, n1, n2)."""
+        shape = (3,) + tuple(int(v) for v in self.params.n)
+        if X is None:
+            X = np.zeros(shape, np.float64)
+        if V is None:
+            V = np.zeros(shape, np.float64)
+        ptrs = [_dptr(X[c]) for c in range(3)] + [_dptr(V[c]) for c in range(3)]
+        N.check(N.lib().somier_read(self._h, *ptrs), "somier_read")
+        return X, V
+
+    def read_ptrs(self, ptrs: Sequence[int]) -> None:
+        N.check(N.lib().somier_read(self._h, *[_dptr(p) for p in ptrs]), "somier_read")
+
+    def load(self, X, V) -> None:
+        ptrs = [_dptr(np.ascontiguousarray(X[c])) for c in range(3)] + [_dptr(np.ascontiguousarray(V[c]))
+                                                                      for c in range(3)]
+        self._keep = (X, V)
+        N.check(N.lib().somier_load(self._h, *ptrs), "somier_load")
+
+    def load_ptrs(self, ptrs: Sequence[int]) -> None:
+        N.check(N.lib().somier_load(self._h, *[_dptr(p) for p in ptrs]), "somier_load")
+
+    # -- multi-process -------------------------------------------------------
+    def ipc_export(self) -> bytes:
+        n = ctypes.c_size_t()
+        N.check(N.lib().somier_ipc_export(self._h, None, 0, ctypes.byref(n)), "somier_ipc_export")
+        buf = ctypes.create_string_buffer(n.value)
+        N.check(N.lib().somier_ipc_export(self._h, buf, n.value, ctypes.byref(n)), "somier_ipc_export")
+        return buf.raw[: n.value]
+
+    def ipc_connect(self, blobs: Sequence[bytes]) -> None:
+        bufs = [ctypes.create_string_buffer(b, len(b)) for b in blobs]
+        ptrs = (ctypes.c_void_p * len(bufs))(*[ctypes.cast(b, ctypes.c_void_p) for b in bufs])
+        lens = (ctypes.c_size_t * len(bufs))(*[len(b) for b in blobs])
+        N.check(N.lib().somier_ipc_connect(self._h, ptrs, lens, len(bufs)), "somier_ipc_connect")
+
+    # -- streams / counters --------------------------------------------------
+    def set_stream(self, device_pos: int, stream_ptr: int) -> None:
+        N.check(N.lib().somier_set_stream(self._h, device_pos, ctypes.c_void_p(stream_ptr)), "somier_set_stream")
+
+    def get_stream(self, device_pos: int) -> int:
+        v = ctypes.c_void_p()
+        N.check(N.lib().somier_get_stream(self._h, device_pos, ctypes.byref(v)), "somier_get_stream")
+        return v.value or 0
+
+    def _i64(self, fn, name) -> int:
+        v = ctypes.c_int64()
+        N.check(fn(self._h, ctypes.byref(v)), name)
+        return v.value
+
+    @property
+    def step_count(self) -> int:
+        return self._i64(N.lib().somier_step_count, "somier_step_count")
+
+    @property
+    def local_chunks(self) -> int:
+        return self._i64(N.lib().somier_local_chunks, "somier_local_chunks")
+
+    @property
+    def launches(self) -> int:
+        return self._i64(N.lib().somier_launch_count, "somier_launch_count")
+
+    @property
+    def device_bytes(self) -> int:
+        return self._i64(N.lib().somier_device_bytes, "somier_device_bytes")

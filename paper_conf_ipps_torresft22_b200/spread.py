@@ -1,0 +1,93 @@
+"""The `target spread` descriptor (include/spread.h)."""
+from __future__ import annotations
+
+import ctypes
+from typing import List, NamedTuple, Sequence
+
+from . import _native as N
+
+
+class Chunk(NamedTuple):
+    index: int
+    device_pos: int   # list position: distribution order
+    device_id: int
+    start: int        # omp_spread_start
+    size: int         # omp_spread_size
+
+
+class Spread:
+    """devices(...) + range(start:len) + spread_schedule(static, chunk).
+
+    chunk == 0 means ceil(len / ndevices): one contiguous slab per device.
+    """
+
+    def __init__(self, devices: Sequence[int], range_start: int, range_len: int, chunk: int = 0, sched: int = 0):
+        L = N.lib()
+        arr = (ctypes.c_int * len(devices))(*devices)
+        h = ctypes.c_void_p()
+        N.check(L.spread_create(arr, len(devices), range_start, range_len, sched, chunk, ctypes.byref(h)),
+                "spread_create")
+        self._h = h
+        self.devices = list(devices)
+
+    @property
+    def handle(self) -> ctypes.c_void_p:
+        return self._h
+
+    def close(self) -> None:
+        if self._h:
+            N.lib().spread_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    @property
+    def num_chunks(self) -> int:
+        v = ctypes.c_int64()
+        N.check(N.lib().spread_num_chunks(self._h, ctypes.byref(v)), "spread_num_chunks")
+        return v.value
+
+    @property
+    def chunk_size(self) -> int:
+        v = ctypes.c_int64()
+        N.check(N.lib().spread_chunk_size(self._h, ctypes.byref(v)), "spread_chunk_size")
+        return v.value
+
+    @property
+    def range(self):
+        a, b = ctypes.c_int64(), ctypes.c_int64()
+        N.check(N.lib().spread_range(self._h, ctypes.byref(a), ctypes.byref(b)), "spread_range")
+        return a.value, b.value
+
+    def chunk(self, c: int) -> Chunk:
+        pos, dev = ctypes.c_int(), ctypes.c_int()
+        start, size = ctypes.c_int64(), ctypes.c_int64()
+        N.check(N.lib().spread_get_chunk(self._h, c, ctypes.byref(pos), ctypes.byref(dev), ctypes.byref(start),
+                                         ctypes.byref(size)), "spread_get_chunk")
+        return Chunk(c, pos.value, dev.value, start.value, size.value)
+
+    def chunks(self) -> List[Chunk]:
+        return [self.chunk(c) for c in range(self.num_chunks)]
+
+    def chunk_of(self, iteration: int) -> int:
+        v = ctypes.c_int64()
+        N.check(N.lib().spread_chunk_of(self._h, iteration, ctypes.byref(v)), "spread_chunk_of")
+        return v.value
+
+    def map_extent(self, c: int, array_len: int, lo_halo: int = 0, hi_halo: int = 0, map_type: int = N.MAP_TO):
+        """Section [first, first+len) of A[omp_spread_start-lo : omp_spread_size+lo+hi]."""
+        first, ln = ctypes.c_int64(), ctypes.c_int64()
+        m = N.spread_map(map_type, lo_halo, hi_halo)
+        N.check(N.lib().spread_map_extent(self._h, c, m, array_len, ctypes.byref(first), ctypes.byref(ln)),
+                "spread_map_extent")
+        return first.value, ln.value

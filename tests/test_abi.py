@@ -1,0 +1,80 @@
+"""The C-ABI boundary: libsomier.so loads and exports every symbol that
+include/*.h declares, with no torch types involved. No compute calls here."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_ipps_torresft22_b200 as P
+from paper_conf_ipps_torresft22_b200 import _native as N
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    names = []
+    for h in ("spread.h", "somier.h"):
+        text = open(os.path.join(ROOT, "include", h)).read()
+        text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+        names += re.findall(r"^\s*(?:const\s+)?[a-z_]+[\s\*]+((?:spread|somier)_[a-z0-9_]+)\s*\(", text, re.M)
+    return sorted(set(names))
+
+
+def test_every_declared_symbol_is_exported_and_bound():
+    L = N.lib()
+    declared = _declared()
+    assert len(declared) >= 25
+    for name in declared:
+        assert hasattr(L, name), name
+    bound = {s[0] for s in N.SIGNATURES}
+    assert set(declared) == bound
+
+
+def test_exports_match_nm():
+    out = subprocess.run(["nm", "-D", "--defined-only", N.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T ((?:spread|somier)_\w+)", out))
+    assert set(_declared()) <= exported
+
+
+def test_library_links_no_torch():
+    out = subprocess.run(["ldd", N.LIB_PATH], capture_output=True, text=True).stdout
+    assert "torch" not in out and "c10" not in out
+    out = subprocess.run(["cuobjdump", "--list-elf", N.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_status_strings_and_version():
+    assert N.status_string(0) == "SPREAD_OK"
+    assert N.status_string(-7) == "SPREAD_ESTATE"
+    assert "sm_100a" in P.version()
+
+
+def test_struct_layouts():
+    # include/somier.h: somier_params = 3*8 + 7*8 + 2*4 bytes; somier_stats_t = 16*8
+    assert ctypes.sizeof(N.somier_params) == 88
+    assert ctypes.sizeof(N.somier_stats_t) == 8 * (1 + 3 + 1 + 3 + 3 + 1 + 1)
+
+
+def test_stats_combine_is_exact_host_logic():
+    """somier_stats_combine is host arithmetic: int128 sums add exactly."""
+    sp = P.SomierParams(n=(4, 4, 4))
+    big = (1 << 100) + 12345
+    a = P.Stats(3, (0.0,) * 3, 0.0, (big, -big, 7), 0x3FF0000000000000, 32)
+    b = P.Stats(3, (0.0,) * 3, 0.0, (-(1 << 100), big, -7), 0x4000000000000000, 32)
+    c = P.combine_stats([a, b], sp)
+    assert c.sums == (12345, 0, 0)
+    assert c.vmax == 2.0 ** 0.5 and c.nodes == 64
+    assert c.centre[0] == (12345 * 2.0 ** -60) / 64
+    with pytest.raises(P.SpreadError):
+        P.combine_stats([a, P.Stats(4, (0.0,) * 3, 0.0, (0, 0, 0), 0, 0)], sp)
+
+
+def test_somier_init_without_gpu_fails_loudly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(P.SpreadError) as e:
+        P.Somier(P.Spread([0], 1, 8), P.SomierParams(n=(10, 10, 10)))
+    assert e.value.status == N.ENODEV

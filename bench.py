@@ -1,0 +1,355 @@
+#!/usr/bin/env python3
+"""bench.py -- Somier node-updates/s on 1..8 B200 (BASELINE.json metric).
+
+Workload (BASELINE.json configs[3]): Somier 512^3 grid, fp64, strong scaling
+over 1/2/4/8 GPUs; the spread is devices(0..N-1) over the i-loop [1, 511) with
+spread_schedule(static, ceil(510/N)) -- one slab per GPU. One bench "step" is
+one Somier time step: the fused K1 kernel per chunk (forces, accelerations,
+velocities, positions, centers, halo exchange). State = 12.9 GB >> 126 MB L2,
+so no L2 flush is needed between steps.
+
+  python bench.py [--gpus N --steps K --warmup W] [--n 512] [--impl ours|reference]
+
+N>1: launched by torch.distributed.run, one process per GPU (RANK/LOCAL_RANK/
+WORLD_SIZE); the halo exchange is fused into the kernel over CUDA IPC/NVLink.
+Rank 0 prints ONE JSON line. --impl reference times the CPU oracle (the
+"reference arm" of this tier) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Somier node-updates/sec at 1/2/4/8 B200; % of HBM peak; parallel efficiency"
+UNIT = "node-updates/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--n", type=int, nargs="+", default=[512])
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--kernel", choices=["auto", "direct", "march"], default="auto")
+    ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    a = ap.parse_args()
+    a.n = tuple(a.n * 3 if len(a.n) == 1 else a.n)
+    return a
+
+
+def workload_name(n):
+    return "Somier %dx%dx%d grid, fp64, strong scaling 1/2/4/8 B200 (BASELINE configs[3])" % n
+
+
+def interior(n):
+    return (n[0] - 2) * (n[1] - 2) * (n[2] - 2)
+
+
+def algorithmic_bytes(n, start, size):
+    """Per K1 launch over one chunk: read X_t on the owned planes + 2 halo planes
+    (24 B/node), read V, write V, write X_{t+1} on interior nodes (72 B/node)."""
+    return 24 * (size + 2) * n[1] * n[2] + 72 * size * (n[1] - 2) * (n[2] - 2)
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_traffic(n, kernel):
+    """DRAM bytes per K1 launch from the committed ncu --set full capture, if it
+    was taken on this workload (profiles/k1_traffic.json)."""
+    path = os.path.join(ROOT, "profiles", "k1_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        e = d.get("%dx%dx%d/%s" % (n[0], n[1], n[2], kernel))
+        return None if e is None else float(e["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        out, _ = self.proc.communicate(timeout=10)
+        sms, maxes, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sms.append(float(f[1]))
+                maxes.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sms:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        loaded = [s for s in sms if s > 0.5 * max(sms)] or sms
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": max(maxes), "reasons": sorted(reasons),
+                "samples": len(sms)}
+
+
+# --------------------------------------------------------------------------- oracle arm
+
+def oracle_sample(n, budget_s, max_steps=None, warmup=0):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload: a
+    (planes+2) x n1 x n2 slab -- `planes` interior planes of the full cross
+    section -- stepped repeatedly. Returns (node-updates/s, sample description, steps)."""
+    import oracle as O
+
+    planes = 8
+    p = O.Params(n=(planes + 2, n[1], n[2]), seed=42)
+    s = O.init(p)
+    per_step = planes * (n[1] - 2) * (n[2] - 2)
+    for _ in range(warmup):
+        s, _ = O.step(s)
+    t0 = time.perf_counter()
+    steps = 0
+    while True:
+        s, _ = O.step(s)
+        steps += 1
+        el = time.perf_counter() - t0
+        if max_steps is not None and steps >= max_steps:
+            break
+        if max_steps is None and el >= budget_s:
+            break
+    rate = per_step * steps / el
+    desc = ("CPU oracle (oracle/somier_oracle.c, sequential fp64, gcc -O2) on a %d-plane slab of the %dx%dx%d "
+            "cross-section (+2 halo planes), %d steps = %.3g node-updates in %.1f s"
+            % (planes, n[0], n[1], n[2], steps, per_step * steps, el))
+    return rate, desc, steps, el
+
+
+def run_reference(a):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    n = a.n
+    rate, desc, steps, el = oracle_sample(n, budget_s=None, max_steps=a.steps, warmup=a.warmup)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": a.gpus, "steps": a.steps,
+        "warmup": a.warmup, "ms_per_step": 1e3 * el / steps, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload_name(n), "n": list(n), "sample": "8-plane slab per step"},
+        "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
+        "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# --------------------------------------------------------------------------- our arm
+
+def run_ours(a):
+    import numpy as np
+    import torch
+
+    import paper_conf_ipps_torresft22_b200 as P
+    from paper_conf_ipps_torresft22_b200 import dist as PD
+
+    rank, world, local = PD.env_rank()
+    if world != a.gpus:
+        raise SystemExit("--gpus %d but WORLD_SIZE %d" % (a.gpus, world))
+    multi = world > 1
+    torch.cuda.set_device(local)
+    if multi:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n = a.n
+    kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH}[a.kernel]
+    params = P.SomierParams(n=n, seed=42, kernel=kernel)
+    if multi:
+        s = PD.open_local(params, chunk=a.chunk, cuda_device=local)
+    else:
+        s = P.Somier(P.Spread([local], 1, n[0] - 2, chunk=a.chunk), params)
+    spread = s.spread
+    my_chunks = [c for c in spread.chunks() if (not multi) or c.device_pos == rank]
+
+    stream = torch.cuda.Stream(device=local)
+    s.set_stream(rank if multi else 0, stream.cuda_stream)
+
+    def barrier():
+        torch.cuda.synchronize(local)
+        if multi:
+            torch.distributed.barrier()
+
+    # warm-up
+    with torch.cuda.stream(stream):
+        s.step(a.warmup)
+    s.sync()
+    barrier()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
+    l0 = s.launches
+    barrier()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for i in range(a.steps):
+        ev[i][0].record(stream)
+        s.step(1)
+        ev[i][1].record(stream)
+    t_end.record(stream)
+    s.sync()
+    barrier()
+    clk = clocks.stop()
+    launches = s.launches - l0
+    ms = t_start.elapsed_time(t_end)
+    per_step = [b.elapsed_time(e) for b, e in ev]
+    if multi:
+        t = torch.tensor([ms], device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+        lt = torch.tensor([launches], device="cuda", dtype=torch.int64)
+        torch.distributed.all_reduce(lt)
+        launches = int(lt.item())
+    value = interior(n) * a.steps / (ms * 1e-3)
+
+    # roofline of the dominant kernel (K1) on this rank's launches
+    k1_ms = statistics.mean(per_step) / max(1, len(my_chunks))
+    c0 = my_chunks[0]
+    alg = algorithmic_bytes(n, c0.start, c0.size)
+    peak, peak_src = load_peaks()
+    achieved = alg / (k1_ms * 1e-3) / 1e9
+    kname = "march" if kernel in (P.K1_AUTO, P.K1_MARCH) else "direct"
+    traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
+    st = PD.gather_stats(s) if multi else s.stats()
+
+    # end-to-end through the public API with pinned host buffers: per step,
+    # map(to) the whole state (X with halos, V), one step, read the centers
+    # result and map(from) the state -- the paper's One Buffer cycle, in core.
+    e2e = None
+    if not a.no_e2e:
+        shape = tuple(n)
+        host = [torch.empty(shape, dtype=torch.float64, pin_memory=True) for _ in range(6)]
+        ptrs = [h.data_ptr() for h in host]
+        s.read_ptrs(ptrs)
+        h2d = d2h = 0
+        for c in my_chunks:
+            plane = n[1] * n[2] * 8
+            h2d += 3 * (c.size + 2) * plane + 3 * c.size * plane
+            d2h += 3 * c.size * plane * 2 + (3 * plane if c.start == 1 else 0) + (3 * plane if c.start + c.size == n[0] - 1 else 0)
+        # warm-up cycle
+        s.load_ptrs(ptrs)
+        s.step(1)
+        s.stats()
+        s.read_ptrs(ptrs)
+        barrier()
+        k = max(1, a.e2e_steps)
+        t0 = time.perf_counter()
+        e_start = torch.cuda.Event(enable_timing=True)
+        e_end = torch.cuda.Event(enable_timing=True)
+        e_start.record(stream)
+        for _ in range(k):
+            s.load_ptrs(ptrs)
+            if multi:
+                s.sync()
+                torch.distributed.barrier()
+            s.step(1)
+            if multi:
+                PD.gather_stats(s)
+            else:
+                s.stats()
+            s.read_ptrs(ptrs)
+        e_end.record(stream)
+        s.sync()
+        barrier()
+        e_ms = e_start.elapsed_time(e_end)
+        wall = time.perf_counter() - t0
+        if multi:
+            t = torch.tensor([e_ms], device="cuda")
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            e_ms = float(t.item())
+        e2e = {"value": interior(n) * k / (e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": int(h2d * world),
+               "d2h_bytes_per_step": int(d2h * world) + 88 * world, "steps": k, "wall_s": wall,
+               "cycle": "somier_load (map to: X[start-1:size+2], V) -> somier_step(1) -> somier_stats -> "
+                        "somier_read (map from) per step, pinned host buffers"}
+        del host
+
+    cpu = None
+    if rank == 0 and not multi and not a.no_cpu_baseline:
+        rate, desc, steps, el = oracle_sample(n, budget_s=a.cpu_seconds)
+        cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+            "ms_per_step": ms / a.steps, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_name(n), "n": list(n), "parallelism": "spread%d" % world,
+                       "spread": "devices(%s) range(1:%d) spread_schedule(static,%d)"
+                                 % (",".join(str(d) for d in spread.devices), n[0] - 2, spread.chunk_size),
+                       "kernel": "K1_" + kname.upper(), "l2": "no flush: 12.9 GB state >> 126 MB L2",
+                       "seed": 42},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "kernel": "k1_%s_kernel" % kname, "algorithmic_bytes_per_launch": alg,
+                         "avg_launch_ms": k1_ms},
+            "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
+            "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},
+        }
+        print(json.dumps(line), flush=True)
+    s.close()
+    if multi:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def main():
+    a = parse()
+    if a.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if a.impl == "reference":
+        return run_reference(a)
+    return run_ours(a)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -5,7 +5,7 @@
 //   * a CTA owns a 32 (k) x 8 (j) column tile and MARCHES along i over a
 //     segment of planes; one warp per row, one lane per k;
 //   * TMA (cp.async.bulk.tensor, 4-D fp64 tensor maps) streams each plane's
-//     X tile with its 1-node halo ring (34 x 10 x 3 doubles) and the matching
+//     X tile with its halo ring (a 36 x 10 x 3 box) and the matching
 //     V tile into a kStages-deep shared-memory ring signalled by mbarriers;
 //   * each spring is evaluated ONCE (bit-exact antisymmetry):
 //     a node computes its +i, +j, +k springs; -i comes from the previous plane
@@ -35,12 +35,17 @@ namespace {
 constexpr int kTK = 32;                 // tile width along k (one warp)
 constexpr int kTJ = 8;                  // tile height along j (warps per CTA)
 constexpr int kThreads = kTK * kTJ;
-constexpr int kBK = kTK + 2;            // X box with halo: 34 x 10
-constexpr int kBJ = kTJ + 2;
-constexpr int kXBoxBytes = kBK * kBJ * 3 * 8;   // 8160
+// X box with its halo ring: columns k0-2 .. k0+33 (the TMA box must start on a
+// 16-byte boundary along the contiguous axis -- an odd fp64 start coordinate
+// faults, measured with tools/tma_probe -- so the left halo is 2 columns wide,
+// of which only k0-1 is used), rows j0-1 .. j0+8.
+constexpr int kBK = kTK + 4;            // 36
+constexpr int kBJ = kTJ + 2;            // 10
+constexpr int kCol0 = 2;                // box column of k0
+constexpr int kXBoxBytes = kBK * kBJ * 3 * 8;   // 8640
 constexpr int kVBoxBytes = kTK * kTJ * 3 * 8;   // 6144
-constexpr int kXSlot = 8192;                    // 128-byte aligned slots
-constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 14336
+constexpr int kXSlot = 8704;                    // 128-byte aligned slots
+constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 14848
 constexpr int kStages = 4;
 constexpr int kSegPlanes = 64;                  // planes per CTA march (segment)
 
@@ -115,6 +120,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int tile_j = blockIdx.x / mp.tiles_k;
     const int k0 = tile_k * kTK, j0 = tile_j * kTJ;
     const int k = k0 + lane, j = j0 + w;
+    const int ck = lane + kCol0, rj = w + 1;  // the node's column / row in the X box
     // output planes [pb, pe) in slab numbering (owned planes are 1..size)
     const int pb = 1 + blockIdx.y * mp.seg_planes;
     const int pe = min((int)g.size + 1, pb + mp.seg_planes);
@@ -129,7 +135,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         unsigned char* st = sm.stage[s];
         const bool with_v = q >= pb + 1;  // V of output plane q-1 rides with X(q)
         mbar_expect_tx(&sm.full[s], kXBoxBytes + (with_v ? kVBoxBytes : 0));
-        tma_load_4d(st, &tmap_x, k0 - 1, j0 - 1, 0, q, &sm.full[s]);
+        tma_load_4d(st, &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);  // OOB -> zeros
         if (with_v) tma_load_4d(st + kXSlot, &tmap_v, k0, j0, 0, q - 2, &sm.full[s]);
     };
     auto wait = [&](int q) {
@@ -157,8 +163,8 @@ __global__ void __launch_bounds__(kThreads, 2)
     // prologue: the -i spring of plane pb is the +i spring of plane pb-1 (negated)
     wait(q0);
     wait(pb);
-    Vec3 carry = spring_force(ldx(xbox(q0), w + 1, lane + 1), ldx(xbox(pb), w + 1, lane + 1), a.K, a.L);
-    Vec3 xc = ldx(xbox(pb), w + 1, lane + 1);
+    Vec3 carry = spring_force(ldx(xbox(q0), rj, ck), ldx(xbox(pb), rj, ck), a.K, a.L);
+    Vec3 xc = ldx(xbox(pb), rj, ck);
     __syncthreads();
     if (tid == 0 && q0 + kStages <= qlast) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -173,15 +179,15 @@ __global__ void __launch_bounds__(kThreads, 2)
         const double* Xc = xbox(p);
         const double* Xn = xbox(p + 1);
         // ---- phase 1: the three "+" springs of every node, plus tile borders
-        const Vec3 xni = ldx(Xn, w + 1, lane + 1);
+        const Vec3 xni = ldx(Xn, rj, ck);
         const Vec3 gpi = spring_force(xc, xni, a.K, a.L);
-        const Vec3 gpj = spring_force(xc, ldx(Xc, w + 2, lane + 1), a.K, a.L);
-        const Vec3 gpk = spring_force(xc, ldx(Xc, w + 1, lane + 2), a.K, a.L);
+        const Vec3 gpj = spring_force(xc, ldx(Xc, rj + 1, ck), a.K, a.L);
+        const Vec3 gpk = spring_force(xc, ldx(Xc, rj, ck + 1), a.K, a.L);
         sm.gj[par][w][lane] = gpj;
         if (w == 0) {
-            sm.gbj[par][lane] = spring_force(ldx(Xc, 0, lane + 1), ldx(Xc, 1, lane + 1), a.K, a.L);
+            sm.gbj[par][lane] = spring_force(ldx(Xc, 0, ck), ldx(Xc, 1, ck), a.K, a.L);
         } else if (w == 1 && lane < kTJ) {
-            sm.gbk[par][lane] = spring_force(ldx(Xc, lane + 1, 0), ldx(Xc, lane + 1, 1), a.K, a.L);
+            sm.gbk[par][lane] = spring_force(ldx(Xc, lane + 1, kCol0 - 1), ldx(Xc, lane + 1, kCol0), a.K, a.L);
         }
         const Vec3 up = shfl_up(gpk);
         __syncthreads();

@@ -247,7 +247,7 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     ia.seed = h->p.seed;
     CUDA_TRY(h, paper::launch_init(ia, s));
     for (int b = 0; b < 2; b++) {
-        spread_status st = encode_slab_map(h, &c.tmap_x[b], c.x(b), c.size + 2, 34, 10);
+        spread_status st = encode_slab_map(h, &c.tmap_x[b], c.x(b), c.size + 2, 36, 10);
         if (st != SPREAD_OK) return st;
     }
     spread_status st = encode_slab_map(h, &c.tmap_v, c.v(), c.size, 32, 8);

@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--copy-check", action="store_true",
+                    help="also time a sustained torch copy of the same byte volume (context for the roofline)")
     a = ap.parse_args()
     a.n = tuple(a.n * 3 if len(a.n) == 1 else a.n)
     return a
@@ -183,6 +185,30 @@ def run_reference(a):
 
 # --------------------------------------------------------------------------- our arm
 
+def sustained_copy(device, stream, gib=6, iters=30):
+    """Context only: a plain torch copy (read+write bytes) sustained back to back,
+    the way K1 runs inside the bench, to compare against the burst hbm_gbs."""
+    import torch
+
+    n = gib * (1 << 30) // 8
+    a = torch.empty(n, dtype=torch.float64, device=device)
+    b = torch.empty_like(a)
+    a.fill_(1.0)
+    with torch.cuda.stream(stream):
+        for _ in range(3):
+            b.copy_(a)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(iters):
+            b.copy_(a)
+        e1.record(stream)
+    e1.synchronize()
+    gbs = 2 * n * 8 * iters / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    del a, b
+    torch.cuda.empty_cache()
+    return gbs
+
+
 def run_ours(a):
     import numpy as np
     import torch
@@ -251,6 +277,8 @@ def run_ours(a):
         launches = int(lt.item())
     value = interior(n) * a.steps / (ms * 1e-3)
 
+    step_dist = {"min": min(per_step), "median": statistics.median(per_step), "max": max(per_step),
+                 "first5": statistics.mean(per_step[:5]), "last5": statistics.mean(per_step[-5:])}
     # roofline of the dominant kernel (K1) on this rank's launches
     k1_ms = statistics.mean(per_step) / max(1, len(my_chunks))
     c0 = my_chunks[0]
@@ -259,6 +287,7 @@ def run_ours(a):
     achieved = alg / (k1_ms * 1e-3) / 1e9
     kname = "march" if kernel in (P.K1_AUTO, P.K1_MARCH) else "direct"
     traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
+    copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()
 
     # end-to-end through the public API with pinned host buffers: per step,
@@ -330,7 +359,8 @@ def run_ours(a):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "k1_%s_kernel" % kname, "algorithmic_bytes_per_launch": alg,
-                         "avg_launch_ms": k1_ms},
+                         "avg_launch_ms": k1_ms, "launch_ms_distribution": step_dist,
+                         "sustained_copy_gbs": copy_gbs},
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
             "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},
         }

@@ -96,17 +96,13 @@ struct MarchParams {
     int seg_planes;
 };
 
-__device__ __forceinline__ Vec3 ldx(const double* box, int r, int col) {
-    return Vec3{box[(0 * kBJ + r) * kBK + col], box[(1 * kBJ + r) * kBK + col], box[(2 * kBJ + r) * kBK + col]};
-}
-
 __device__ __forceinline__ Vec3 shfl_up(const Vec3& v) {
     return Vec3{__shfl_up_sync(0xffffffffu, v.x, 1), __shfl_up_sync(0xffffffffu, v.y, 1),
                 __shfl_up_sync(0xffffffffu, v.z, 1)};
 }
 
 template <bool kUnitMass>
-__global__ void __launch_bounds__(kThreads, 2)
+__global__ void __launch_bounds__(kThreads, 3)
     k1_march_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                     const MarchParams mp) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -142,8 +138,6 @@ __global__ void __launch_bounds__(kThreads, 2)
         const int s = (q - q0) % kStages;
         mbar_wait(&sm.full[s], (unsigned)(((q - q0) / kStages) & 1));
     };
-    auto xbox = [&](int q) { return reinterpret_cast<const double*>(sm.stage[(q - q0) % kStages]); };
-    auto vbox = [&](int q) { return reinterpret_cast<const double*>(sm.stage[(q - q0) % kStages] + kXSlot); };
 
     if (tid == 0) {
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap_x)) : "memory");
@@ -159,35 +153,47 @@ __global__ void __launch_bounds__(kThreads, 2)
     const bool interior = j >= 1 && j < g.n1 - 1 && k >= 1 && k < g.n2 - 1;
     const int64_t cs = g.comp_stride(), ps = g.plane_stride();
     const int64_t off = (int64_t)j * g.ld + k;
+    // per-thread offsets (in doubles) inside a stage: own node of the X box, V box
+    constexpr int kXComp = kBJ * kBK, kVComp = kTJ * kTK;
+    const int xo_own = rj * kBK + ck;
+    const int vo_own = w * kTK + lane;
+    auto stage_x = [&](int s) { return reinterpret_cast<const double*>(smem_raw + s * kStageBytes); };
+    auto ld3 = [&](const double* p) { return Vec3{p[0], p[kXComp], p[2 * kXComp]}; };
 
     // prologue: the -i spring of plane pb is the +i spring of plane pb-1 (negated)
     wait(q0);
     wait(pb);
-    Vec3 carry = spring_force(ldx(xbox(q0), rj, ck), ldx(xbox(pb), rj, ck), a.K, a.L);
-    Vec3 xc = ldx(xbox(pb), rj, ck);
+    Vec3 carry = spring_force(ld3(stage_x(0) + xo_own), ld3(stage_x(1) + xo_own), a.K, a.L);
+    Vec3 xc = ld3(stage_x(1) + xo_own);
     __syncthreads();
     if (tid == 0 && q0 + kStages <= qlast) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         issue(q0 + kStages);
     }
 
+    double* xo = a.x_nxt + (int64_t)pb * ps + off;      // X_{t+1} of this node, plane pb
+    double* vo = a.v + (int64_t)(pb - 1) * ps + off;    // V of this node, plane pb
+    int s_cur = 1, s_nxt = 2 % kStages;                 // stages of planes p and p+1
+    unsigned ph_nxt = (2 / kStages) & 1;                // mbarrier parity of plane p+1
     NodeStats st;
     st.zero();
     for (int p = pb; p < pe; p++) {
         const int par = p & 1;
-        wait(p + 1);
-        const double* Xc = xbox(p);
-        const double* Xn = xbox(p + 1);
+        mbar_wait(&sm.full[s_nxt], ph_nxt);
+        const double* Xc = stage_x(s_cur);
+        const double* Xn = stage_x(s_nxt);
+        const double* me = Xc + xo_own;
         // ---- phase 1: the three "+" springs of every node, plus tile borders
-        const Vec3 xni = ldx(Xn, rj, ck);
+        const Vec3 gpk = spring_force(xc, ld3(me + 1), a.K, a.L);
+        const Vec3 xni = ld3(Xn + xo_own);
         const Vec3 gpi = spring_force(xc, xni, a.K, a.L);
-        const Vec3 gpj = spring_force(xc, ldx(Xc, rj + 1, ck), a.K, a.L);
-        const Vec3 gpk = spring_force(xc, ldx(Xc, rj, ck + 1), a.K, a.L);
+        const Vec3 gpj = spring_force(xc, ld3(me + kBK), a.K, a.L);
         sm.gj[par][w][lane] = gpj;
         if (w == 0) {
-            sm.gbj[par][lane] = spring_force(ldx(Xc, 0, ck), ldx(Xc, 1, ck), a.K, a.L);
+            sm.gbj[par][lane] = spring_force(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
         } else if (w == 1 && lane < kTJ) {
-            sm.gbk[par][lane] = spring_force(ldx(Xc, lane + 1, kCol0 - 1), ldx(Xc, lane + 1, kCol0), a.K, a.L);
+            const double* b = Xc + (lane + 1) * kBK + kCol0;
+            sm.gbk[par][lane] = spring_force(ld3(b - 1), ld3(b), a.K, a.L);
         }
         const Vec3 up = shfl_up(gpk);
         __syncthreads();
@@ -201,39 +207,39 @@ __global__ void __launch_bounds__(kThreads, 2)
         const Vec3 gmj = neg(w == 0 ? sm.gbj[par][lane] : sm.gj[par][w - 1][lane]);
         const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][w] : up);
         carry = gpi;
-        if (valid) {
-            if (interior) {
-                const Vec3 F = sum_forces(gmi, gpi, gmj, gpj, gmk, gpk);
-                const double* Vb = vbox(p + 1);
-                Vec3 v{Vb[(0 * kTJ + w) * kTK + lane], Vb[(1 * kTJ + w) * kTK + lane],
-                       Vb[(2 * kTJ + w) * kTK + lane]};
-                Vec3 xn;
-                kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
-                double* vo = a.v + (int64_t)(p - 1) * ps + off;
-                vo[0] = v.x;
-                vo[cs] = v.y;
-                vo[2 * cs] = v.z;
-                double* xo = a.x_nxt + (int64_t)p * ps + off;
-                xo[0] = xn.x;
-                xo[cs] = xn.y;
-                xo[2 * cs] = xn.z;
-                if (p == 1 && a.lo_dst) {
-                    a.lo_dst[off] = xn.x;
-                    a.lo_dst[off + cs] = xn.y;
-                    a.lo_dst[off + 2 * cs] = xn.z;
-                }
-                if (p == g.size && a.hi_dst) {
-                    a.hi_dst[off] = xn.x;
-                    a.hi_dst[off + cs] = xn.y;
-                    a.hi_dst[off + 2 * cs] = xn.z;
-                }
-                st.add_position(xn);
-                st.add_velocity(v);
-            } else {
-                st.add_position(xc);  // fixed face node
+        if (interior) {
+            const Vec3 F = sum_forces(gmi, gpi, gmj, gpj, gmk, gpk);
+            const double* Vb = reinterpret_cast<const double*>(smem_raw + s_nxt * kStageBytes + kXSlot) + vo_own;
+            Vec3 v{Vb[0], Vb[kVComp], Vb[2 * kVComp]};
+            Vec3 xn;
+            kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
+            vo[0] = v.x;
+            vo[cs] = v.y;
+            vo[2 * cs] = v.z;
+            xo[0] = xn.x;
+            xo[cs] = xn.y;
+            xo[2 * cs] = xn.z;
+            if (p == 1 && a.lo_dst) {
+                a.lo_dst[off] = xn.x;
+                a.lo_dst[off + cs] = xn.y;
+                a.lo_dst[off + 2 * cs] = xn.z;
             }
+            if (p == g.size && a.hi_dst) {
+                a.hi_dst[off] = xn.x;
+                a.hi_dst[off + cs] = xn.y;
+                a.hi_dst[off + 2 * cs] = xn.z;
+            }
+            st.add_position(xn);
+            st.add_velocity(v);
+        } else if (valid) {
+            st.add_position(xc);  // fixed face node: X_{t+1} == X_t, V == 0
         }
         xc = xni;
+        xo += ps;
+        vo += ps;
+        s_cur = s_nxt;
+        s_nxt = (s_nxt + 1 == kStages) ? 0 : s_nxt + 1;
+        ph_nxt ^= (s_nxt == 0) ? 1u : 0u;
     }
     block_accumulate(st, sm.scratch, a.acc);
     signal_neighbours(a);

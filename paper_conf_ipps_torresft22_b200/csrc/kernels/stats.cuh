@@ -1,7 +1,19 @@
 // stats.cuh -- the "centers" reduction fused into the step
-// kernels: exact int128 fixed-point sums of the positions (reading S15:
-// order-independent, so every launch configuration and every chunk partition
-// gives the same bits) and the max of v.v as an unsigned bit pattern.
+// kernels: the exact sum over nodes of q(x) = round_half_even(x * 2^60) for
+// each coordinate (reading S15: order-independent, so every launch
+// configuration and chunk partition gives the same bits) and the max of v.v.
+//
+// Per thread the exact sum is carried in fp64 registers without any integer
+// work (the integer-heavy int128 path made K1 issue-bound, profiles/r01_v1):
+//   y = x * 2^28                      exact (power-of-two scale)
+//   h = (y + C) - C,  C = 1.5 * 2^52  = round_half_even(y), an integer, |y| < 2^51
+//   r = y - h                         exact, |r| <= 1/2
+//   l = fma(r, 2^32, C) - C           = round_half_even(r * 2^32), an integer
+// Since h * 2^32 is an even integer, q(x) = h * 2^32 + l exactly. The sums of
+// h and of l stay exact in fp64 while they are below 2^53: |x| < 2^18 (checked
+// by somier_init) and at most kMaxNodesPerThread nodes per thread give
+// |sum h| < 2^46 * 128 and |sum l| < 2^31 * 128. The block reduction converts
+// to int128 once; the device accumulator adds int128 with 64-bit atomics.
 #pragma once
 #include <cstdint>
 
@@ -10,39 +22,47 @@
 
 namespace paper {
 
-// round_half_even(x * 2^60) as an exact int128. x*2^60 is exact (power-of-two
-// scale). Below 2^62 in magnitude __double2ll_rn rounds half to even; above it
-// the value is already an integer and is rebuilt from its significand.
-// Non-finite inputs contribute 0 (their v.v makes vmax non-finite instead).
-__device__ __forceinline__ __int128 quantise_2p60(double x) {
-    const double s = __dmul_rn(x, 0x1p60);
-    if (fabs(s) < 0x1p62) return (__int128)__double2ll_rn(s);
-    const unsigned long long bits = (unsigned long long)__double_as_longlong(s);
-    const int e = (int)((bits >> 52) & 0x7FF);
-    if (e == 0x7FF) return 0;
-    const unsigned long long m = (bits & ((1ull << 52) - 1)) | (1ull << 52);
-    const int shift = e - 1075;  // >= 10 here
-    const __int128 q = (shift < 74) ? ((__int128)m << shift) : (__int128)0;
-    return (bits >> 63) ? -q : q;
-}
+constexpr int kMaxNodesPerThread = 128;
+constexpr double kRoundC = 6755399441055744.0;  // 1.5 * 2^52
 
 struct NodeStats {
-    __int128 s[3];
-    unsigned long long vmax2;
+    double h[3], l[3];
+    double vmax2;  // NaN-sticky max of v.v
 
     __device__ __forceinline__ void zero() {
-        s[0] = s[1] = s[2] = 0;
-        vmax2 = 0ull;
+        h[0] = h[1] = h[2] = 0.0;
+        l[0] = l[1] = l[2] = 0.0;
+        vmax2 = 0.0;
+    }
+    __device__ __forceinline__ void add_coord(int c, double x) {
+        // fma with an exact power-of-two product == the unfused sequence above
+        const double hh = __dsub_rn(__fma_rn(x, 0x1p28, kRoundC), kRoundC);
+        const double r = __fma_rn(x, 0x1p28, -hh);
+        const double ll = __dsub_rn(__fma_rn(r, 0x1p32, kRoundC), kRoundC);
+        h[c] = __dadd_rn(h[c], hh);
+        l[c] = __dadd_rn(l[c], ll);
     }
     __device__ __forceinline__ void add_position(const Vec3& x) {
-        s[0] += quantise_2p60(x.x);
-        s[1] += quantise_2p60(x.y);
-        s[2] += quantise_2p60(x.z);
+        add_coord(0, x.x);
+        add_coord(1, x.y);
+        add_coord(2, x.z);
     }
     __device__ __forceinline__ void add_velocity(const Vec3& v) {
-        const unsigned long long b = (unsigned long long)__double_as_longlong(dot_self(v));
-        vmax2 = b > vmax2 ? b : vmax2;
+        const double v2 = dot_self(v);
+        vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
     }
+    // exact int128 value of sum q(x) for coordinate c
+    __device__ __forceinline__ __int128 sum(int c) const {
+        return (__int128)__double2ll_rn(h[c]) * ((__int128)1 << 32) + (__int128)__double2ll_rn(l[c]);
+    }
+    __device__ __forceinline__ unsigned long long vmax2_bits() const {
+        return (unsigned long long)__double_as_longlong(vmax2);
+    }
+};
+
+struct I128Stats {
+    __int128 s[3];
+    unsigned long long vmax2;
 };
 
 __device__ __forceinline__ __int128 shfl_xor_i128(__int128 v, int m) {
@@ -53,7 +73,7 @@ __device__ __forceinline__ __int128 shfl_xor_i128(__int128 v, int m) {
     return (__int128)(((unsigned __int128)hi << 64) | lo);
 }
 
-__device__ __forceinline__ void warp_reduce(NodeStats& st) {
+__device__ __forceinline__ void warp_reduce(I128Stats& st) {
 #pragma unroll
     for (int m = 16; m > 0; m >>= 1) {
 #pragma unroll
@@ -78,13 +98,16 @@ __device__ __forceinline__ void atomic_add_i128(unsigned long long* lo_word, uns
     }
 }
 
-// Block-wide reduction of per-thread NodeStats into the step's accumulator.
-// All threads of the block must call it. `scratch` holds >= nwarps entries.
 struct WarpStats {
     unsigned long long lo[3], hi[3], vmax2, pad;
 };
 
-__device__ __forceinline__ void block_accumulate(NodeStats st, WarpStats* scratch, StatsAccum* acc) {
+// Block-wide reduction of per-thread NodeStats into the step's accumulator.
+// All threads of the block must call it. `scratch` holds >= nwarps entries.
+__device__ __forceinline__ void block_accumulate(const NodeStats& ns, WarpStats* scratch, StatsAccum* acc) {
+    I128Stats st;
+    for (int c = 0; c < 3; c++) st.s[c] = ns.sum(c);
+    st.vmax2 = ns.vmax2_bits();
     warp_reduce(st);
     const int lane = threadIdx.x & 31;
     const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
@@ -99,8 +122,9 @@ __device__ __forceinline__ void block_accumulate(NodeStats st, WarpStats* scratc
     }
     __syncthreads();
     if (warp == 0) {
-        NodeStats t;
-        t.zero();
+        I128Stats t;
+        t.s[0] = t.s[1] = t.s[2] = 0;
+        t.vmax2 = 0ull;
         if (lane < nwarps) {
             for (int c = 0; c < 3; c++)
                 t.s[c] = (__int128)(((unsigned __int128)scratch[lane].hi[c] << 64) | scratch[lane].lo[c]);

@@ -146,7 +146,17 @@ spread_status check_params(const somier_params* p) {
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
     if (n1 > 65535LL * 8 || n0 > 65535 + 2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: grid too large for the launch geometry");
-    (void)n2;
+    // the branch-free sqrt / division of the spring law (kernels/node_math.cuh)
+    // are correctly rounded for |K|, |L| in [2^-100, 2^100] (or 0)
+    auto in_domain = [](double v) { return v == 0.0 || (std::fabs(v) >= 0x1p-100 && std::fabs(v) <= 0x1p100); };
+    if (!in_domain(p->k_spring) || !in_domain(p->rest_len))
+        PAPER_FAIL(SPREAD_EINVAL, "somier: k_spring and rest_len must be 0 or of magnitude in [2^-100, 2^100]");
+    // the fused exact centre sums (kernels/stats.cuh) need |x| < 2^18; keep a
+    // factor-2 margin over the initial extent of the lattice
+    const double extent = (double)(std::max(n0, std::max(n1, n2)) - 1) / 2.0 * std::fabs(p->spacing) +
+                          std::fabs(p->amplitude);
+    if (!(extent < 131072.0))
+        PAPER_FAIL(SPREAD_EINVAL, "somier: lattice extent %.3g too large for exact centre sums (< 2^17)", extent);
     return SPREAD_OK;
 }
 

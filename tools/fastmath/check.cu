@@ -1,0 +1,53 @@
+// Validates the branch-free correctly-rounded fp64 sqrt / div used by K1
+// (csrc/kernels/node_math.cuh: sqrt_rn_nb, div_rn_nb) against the CUDA
+// library __dsqrt_rn / __ddiv_rn over many random and adversarial inputs in
+// the operating range. Prints the mismatch counts (must be 0).
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "../../paper_conf_ipps_torresft22_b200/csrc/kernels/node_math.cuh"
+
+__device__ __forceinline__ uint64_t mix(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull; z = (z ^ (z >> 27)) * 0x94D049BB133111EBull; return z ^ (z >> 31);
+}
+__device__ __forceinline__ double u01(uint64_t r) { return (double)(r >> 11) * 0x1p-53; }
+
+__global__ void check(uint64_t seed, long long iters, unsigned long long* bad, unsigned long long* tot) {
+  unsigned long long b_s = 0, b_d = 0, n = 0;
+  uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  for (long long it = 0; it < iters; it++) {
+    uint64_t r1 = mix(seed + (t * 1000003ull + it) * 0x9E3779B97F4A7C15ull);
+    uint64_t r2 = mix(r1 ^ 0x1234567ull);
+    uint64_t r3 = mix(r2 + 77);
+    // sqrt argument: d2 around 1 with wide spread: 2^[-40, 40] log-uniform, plus near-1 uniform
+    double a;
+    int mode = (int)(r3 & 3);
+    if (mode == 0) a = exp2(-40.0 + 80.0 * u01(r1));
+    else if (mode == 1) a = 0.2 + 5.0 * u01(r1);
+    else if (mode == 2) a = 1.0 + (u01(r1) - 0.5) * 1e-6;
+    else a = __longlong_as_double((long long)(0x3FF0000000000000ull + (r1 & 0xFFFFFull)) ); // near 1, low bits
+    double s0 = __dsqrt_rn(a), s1 = paper::sqrt_rn_nb(a);
+    if (__double_as_longlong(s0) != __double_as_longlong(s1)) b_s++;
+    // division n / d: d in [2^-20, 2^20] and near 1; n signed, wide range and tiny, and 0
+    double d = (mode == 0) ? exp2(-20.0 + 40.0 * u01(r2)) : 0.3 + 3.0 * u01(r2);
+    double num;
+    int m2 = (int)((r3 >> 2) & 3);
+    if (m2 == 0) num = (u01(r3 >> 4 | r1) - 0.5) * 20.0;
+    else if (m2 == 1) num = (u01(r2 ^ r1) - 0.5) * exp2(-60.0 + 100.0 * u01(r3));
+    else if (m2 == 2) num = 10.0 * (__dsub_rn(d, 1.0));
+    else num = (r3 & 16) ? 0.0 : -0.0;
+    double q0 = __ddiv_rn(num, d), q1 = paper::div_rn_nb(num, d);
+    if (__double_as_longlong(q0) != __double_as_longlong(q1)) b_d++;
+    n++;
+  }
+  atomicAdd(&bad[0], b_s); atomicAdd(&bad[1], b_d); atomicAdd(tot, n);
+}
+
+int main(int argc, char** argv) {
+  long long iters = argc > 1 ? atoll(argv[1]) : 2000;
+  unsigned long long *bad, *tot; cudaMalloc(&bad, 16); cudaMalloc(&tot, 8); cudaMemset(bad, 0, 16); cudaMemset(tot, 0, 8);
+  check<<<148 * 8, 256>>>(12345, iters, bad, tot);
+  unsigned long long hb[2], ht; cudaMemcpy(hb, bad, 16, cudaMemcpyDeviceToHost); cudaMemcpy(&ht, tot, 8, cudaMemcpyDeviceToHost);
+  printf("samples %llu sqrt_mismatch %llu div_mismatch %llu (%s)\n", ht, hb[0], hb[1], cudaGetErrorString(cudaGetLastError()));
+  return (hb[0] || hb[1]) ? 1 : 0;
+}

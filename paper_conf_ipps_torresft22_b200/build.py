@@ -17,13 +17,15 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-BUILD = os.path.join(PKG, "_build")
-LIB = os.path.join(PKG, "libsomier.so")
+# SOMIER_BUILD_TAG / SOMIER_NVCC_DEFS: variant builds for experiments (tools/variants.sh)
+_TAG = os.environ.get("SOMIER_BUILD_TAG", "")
+BUILD = os.path.join(PKG, "_build" + (("_" + _TAG) if _TAG else ""))
+LIB = os.path.join(PKG, "libsomier%s.so" % (("_" + _TAG) if _TAG else ""))
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall,-Wno-unknown-pragmas",
           "-I" + INCLUDE, "-I" + CSRC]
-CU_FLAGS = ARCH + ["-Xptxas", "-v", "--expt-relaxed-constexpr"]
+CU_FLAGS = ARCH + ["-Xptxas", "-v", "--expt-relaxed-constexpr"] + os.environ.get("SOMIER_NVCC_DEFS", "").split()
 
 
 def sources():

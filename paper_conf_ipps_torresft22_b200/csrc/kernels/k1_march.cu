@@ -101,8 +101,20 @@ __device__ __forceinline__ Vec3 shfl_up(const Vec3& v) {
                 __shfl_up_sync(0xffffffffu, v.z, 1)};
 }
 
+// Occupancy / unroll knobs (tools/variants.sh). Measured on 512^3 (r01): 2 CTAs
+// per SM (<= 128 registers, no spills) with the plane loop unrolled by 2 beats
+// 3 CTAs per SM (80 registers, spills, index rematerialisation): under the
+// 1 kW power cap the kernel is energy-bound, so fewer issued instructions win.
+#ifndef K1_MIN_BLOCKS
+#define K1_MIN_BLOCKS 2
+#endif
+#ifndef K1_UNROLL
+#define K1_UNROLL 2
+#endif
+constexpr int kUnroll = K1_UNROLL;
+
 template <bool kUnitMass>
-__global__ void __launch_bounds__(kThreads, 3)
+__global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     k1_march_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                     const MarchParams mp) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -177,6 +189,7 @@ __global__ void __launch_bounds__(kThreads, 3)
     unsigned ph_nxt = (2 / kStages) & 1;                // mbarrier parity of plane p+1
     NodeStats st;
     st.zero();
+#pragma unroll(kUnroll)
     for (int p = pb; p < pe; p++) {
         const int par = p & 1;
         mbar_wait(&sm.full[s_nxt], ph_nxt);

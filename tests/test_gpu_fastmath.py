@@ -21,4 +21,4 @@ def test_fast_sqrt_div_bit_identical_to_library(tmp_path):
     r = subprocess.run([exe, "4000"], capture_output=True, text=True, timeout=300)
     print(r.stdout)
     assert r.returncode == 0, r.stdout + r.stderr
-    assert "sqrt_mismatch 0 div_mismatch 0" in r.stdout
+    assert "sqrt_mismatch 0 div_mismatch 0 fused_mismatch 0" in r.stdout

@@ -13,7 +13,7 @@ __device__ __forceinline__ uint64_t mix(uint64_t z) {
 __device__ __forceinline__ double u01(uint64_t r) { return (double)(r >> 11) * 0x1p-53; }
 
 __global__ void check(uint64_t seed, long long iters, unsigned long long* bad, unsigned long long* tot) {
-  unsigned long long b_s = 0, b_d = 0, n = 0;
+  unsigned long long b_s = 0, b_d = 0, b_f = 0, n = 0;
   uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
   for (long long it = 0; it < iters; it++) {
     uint64_t r1 = mix(seed + (t * 1000003ull + it) * 0x9E3779B97F4A7C15ull);
@@ -38,16 +38,30 @@ __global__ void check(uint64_t seed, long long iters, unsigned long long* bad, u
     else num = (r3 & 16) ? 0.0 : -0.0;
     double q0 = __ddiv_rn(num, d), q1 = paper::div_rn_nb(num, d);
     if (__double_as_longlong(q0) != __double_as_longlong(q1)) b_d++;
+    // the spring law's fused form: d = sqrt(a), f = n(d) / d with n = K (d - L)
+    {
+      double r, dd = paper::sqrt_recip_rn_nb(a, r);
+      double dl = __dsqrt_rn(a);
+      if (__double_as_longlong(dd) != __double_as_longlong(dl)) b_f++;
+      double K = (m2 == 3) ? 0.0 : 10.0 * (0.25 + u01(r3 ^ r2));
+      double Lr = (m2 == 2) ? dl : 1.0;   // d == L exactly: zero numerator
+      double n1 = __dmul_rn(K, __dsub_rn(dl, Lr));
+      double f0 = __ddiv_rn(n1, dl), f1 = paper::div_by(n1, dd, r);
+      if (__double_as_longlong(f0) != __double_as_longlong(f1)) b_f++;
+      double mynum = num;  // arbitrary numerator against the fused reciprocal too
+      double g0 = __ddiv_rn(mynum, dl), g1 = paper::div_by(mynum, dd, r);
+      if (__double_as_longlong(g0) != __double_as_longlong(g1)) b_f++;
+    }
     n++;
   }
-  atomicAdd(&bad[0], b_s); atomicAdd(&bad[1], b_d); atomicAdd(tot, n);
+  atomicAdd(&bad[0], b_s); atomicAdd(&bad[1], b_d); atomicAdd(&bad[2], b_f); atomicAdd(tot, n);
 }
 
 int main(int argc, char** argv) {
   long long iters = argc > 1 ? atoll(argv[1]) : 2000;
-  unsigned long long *bad, *tot; cudaMalloc(&bad, 16); cudaMalloc(&tot, 8); cudaMemset(bad, 0, 16); cudaMemset(tot, 0, 8);
+  unsigned long long *bad, *tot; cudaMalloc(&bad, 24); cudaMalloc(&tot, 8); cudaMemset(bad, 0, 24); cudaMemset(tot, 0, 8);
   check<<<148 * 8, 256>>>(12345, iters, bad, tot);
-  unsigned long long hb[2], ht; cudaMemcpy(hb, bad, 16, cudaMemcpyDeviceToHost); cudaMemcpy(&ht, tot, 8, cudaMemcpyDeviceToHost);
-  printf("samples %llu sqrt_mismatch %llu div_mismatch %llu (%s)\n", ht, hb[0], hb[1], cudaGetErrorString(cudaGetLastError()));
-  return (hb[0] || hb[1]) ? 1 : 0;
+  unsigned long long hb[3], ht; cudaMemcpy(hb, bad, 24, cudaMemcpyDeviceToHost); cudaMemcpy(&ht, tot, 8, cudaMemcpyDeviceToHost);
+  printf("samples %llu sqrt_mismatch %llu div_mismatch %llu fused_mismatch %llu (%s)\n", ht, hb[0], hb[1], hb[2], cudaGetErrorString(cudaGetLastError()));
+  return (hb[0] || hb[1] || hb[2]) ? 1 : 0;
 }

@@ -113,7 +113,7 @@ __device__ __forceinline__ Vec3 shfl_up(const Vec3& v) {
 #endif
 constexpr int kUnroll = K1_UNROLL;
 
-template <bool kUnitMass>
+template <bool kUnitMass, bool kPosK>
 __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     k1_march_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                     const MarchParams mp) {
@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     // prologue: the -i spring of plane pb is the +i spring of plane pb-1 (negated)
     wait(q0);
     wait(pb);
-    Vec3 carry = spring_force(ld3(stage_x(0) + xo_own), ld3(stage_x(1) + xo_own), a.K, a.L);
+    Vec3 carry = spring_force<kPosK>(ld3(stage_x(0) + xo_own), ld3(stage_x(1) + xo_own), a.K, a.L);
     Vec3 xc = ld3(stage_x(1) + xo_own);
     __syncthreads();
     if (tid == 0 && q0 + kStages <= qlast) {
@@ -197,16 +197,16 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
         const double* Xn = stage_x(s_nxt);
         const double* me = Xc + xo_own;
         // ---- phase 1: the three "+" springs of every node, plus tile borders
-        const Vec3 gpk = spring_force(xc, ld3(me + 1), a.K, a.L);
+        const Vec3 gpk = spring_force<kPosK>(xc, ld3(me + 1), a.K, a.L);
         const Vec3 xni = ld3(Xn + xo_own);
-        const Vec3 gpi = spring_force(xc, xni, a.K, a.L);
-        const Vec3 gpj = spring_force(xc, ld3(me + kBK), a.K, a.L);
+        const Vec3 gpi = spring_force<kPosK>(xc, xni, a.K, a.L);
+        const Vec3 gpj = spring_force<kPosK>(xc, ld3(me + kBK), a.K, a.L);
         sm.gj[par][w][lane] = gpj;
         if (w == 0) {
-            sm.gbj[par][lane] = spring_force(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
+            sm.gbj[par][lane] = spring_force<kPosK>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
         } else if (w == 1 && lane < kTJ) {
             const double* b = Xc + (lane + 1) * kBK + kCol0;
-            sm.gbk[par][lane] = spring_force(ld3(b - 1), ld3(b), a.K, a.L);
+            sm.gbk[par][lane] = spring_force<kPosK>(ld3(b - 1), ld3(b), a.K, a.L);
         }
         const Vec3 up = shfl_up(gpk);
         __syncthreads();
@@ -274,13 +274,15 @@ cudaError_t launch_k1_march(const StepArgs& a, bool unit_mass, cudaStream_t stre
     const size_t smem = sizeof(Smem);
     const CUtensorMap& mx = *static_cast<const CUtensorMap*>(a.tmap_x_cur);
     const CUtensorMap& mv = *static_cast<const CUtensorMap*>(a.tmap_v);
-    if (unit_mass) {
-        cudaFuncSetAttribute(k1_march_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        k1_march_kernel<true><<<grid, block, smem, stream>>>(mx, mv, mp);
-    } else {
-        cudaFuncSetAttribute(k1_march_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        k1_march_kernel<false><<<grid, block, smem, stream>>>(mx, mv, mp);
-    }
+    auto launch = [&](auto kernel) {
+        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        kernel<<<grid, block, smem, stream>>>(mx, mv, mp);
+    };
+    const bool pos_k = a.K > 0.0;
+    if (unit_mass)
+        pos_k ? launch(k1_march_kernel<true, true>) : launch(k1_march_kernel<true, false>);
+    else
+        pos_k ? launch(k1_march_kernel<false, true>) : launch(k1_march_kernel<false, false>);
     return cudaGetLastError();
 }
 

@@ -237,3 +237,15 @@ def test_launch_count_and_footprint():
         s.sync()
         assert s.launches == 12
         assert s.device_bytes >= (2 * 34 + 32) * 3 * 20 * 40 * 8
+
+
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH])
+@pytest.mark.parametrize("K", [0.0, -2.0])
+def test_zero_and_negative_stiffness_signed_zeros(K, kernel):
+    """K <= 0 makes K*(d-L) = -0 possible; -0/d must stay -0 (the K > 0 fast
+    path drops that select). Bitwise vs the oracle, signed zeros included."""
+    sp = _params((9, 10, 33), seed=6, kernel=kernel, k_spring=K)
+    X, V, st = _run_gpu(sp, 12)
+    ref, rst = O.run(O.init(_oracle_params(sp)), 12)
+    assert np.array_equal(X.view(np.uint64), ref.X.view(np.uint64))
+    assert np.array_equal(V.view(np.uint64), ref.V.view(np.uint64))

@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="testing only: all ranks on cuda:0 with gloo plumbing (exercises the N>1 path on 1 GPU)")
     ap.add_argument("--copy-check", action="store_true",
                     help="also time a sustained torch copy of the same byte volume (context for the roofline)")
     a = ap.parse_args()
@@ -239,10 +241,26 @@ def run_ours(a):
     if world != a.gpus:
         raise SystemExit("--gpus %d but WORLD_SIZE %d" % (a.gpus, world))
     multi = world > 1
+    if a.share_gpu:  # test mode: every rank on cuda:0 (IPC within one device), gloo plumbing
+        local = 0
     torch.cuda.set_device(local)
+    dev = "cpu" if a.share_gpu else "cuda"
     if multi:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if a.share_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    def all_max(x, dtype=torch.float64):
+        t = torch.tensor([x], device=dev, dtype=dtype)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        return t.item()
+
+    def all_sum(x):
+        t = torch.tensor([x], device=dev, dtype=torch.int64)
+        torch.distributed.all_reduce(t)
+        return int(t.item())
     n = a.n
     kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH}[a.kernel]
     params = P.SomierParams(n=n, seed=42, kernel=kernel)
@@ -290,12 +308,8 @@ def run_ours(a):
     ms = t_start.elapsed_time(t_end)
     per_step = [b.elapsed_time(e) for b, e in ev]
     if multi:
-        t = torch.tensor([ms], device="cuda")
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        ms = float(t.item())
-        lt = torch.tensor([launches], device="cuda", dtype=torch.int64)
-        torch.distributed.all_reduce(lt)
-        launches = int(lt.item())
+        ms = float(all_max(ms))
+        launches = all_sum(launches)
     value = interior(n) * a.steps / (ms * 1e-3)
 
     step_dist = {"min": min(per_step), "median": statistics.median(per_step), "max": max(per_step),
@@ -353,9 +367,7 @@ def run_ours(a):
         e_ms = e_start.elapsed_time(e_end)
         wall = time.perf_counter() - t0
         if multi:
-            t = torch.tensor([e_ms], device="cuda")
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            e_ms = float(t.item())
+            e_ms = float(all_max(e_ms))
         e2e = {"value": interior(n) * k / (e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": int(h2d * world),
                "d2h_bytes_per_step": int(d2h * world) + 88 * world, "steps": k, "wall_s": wall,
                "cycle": "somier_load (map to: X[start-1:size+2], V) -> somier_step(1) -> somier_stats -> "

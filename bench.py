@@ -8,7 +8,7 @@ one Somier time step: the fused K1 kernel per chunk (forces, accelerations,
 velocities, positions, centers, halo exchange). State = 12.9 GB >> 126 MB L2,
 so no L2 flush is needed between steps.
 
-  python bench.py [--gpus N --steps K --warmup W] [--n 512] [--impl ours|reference]
+  python bench.py [--gpus N --steps K --warmup W] [--grid 512] [--impl ours|reference]
 
 N>1: launched by torch.distributed.run, one process per GPU (RANK/LOCAL_RANK/
 WORLD_SIZE); the halo exchange is fused into the kernel over CUDA IPC/NVLink.
@@ -37,7 +37,8 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--n", type=int, nargs="+", default=[512])
+    ap.add_argument("--grid", type=int, nargs="+", default=[512],
+                    help="grid nodes (one value: cube); not --n, which torch.distributed.run would claim")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--kernel", choices=["auto", "direct", "march"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
@@ -50,7 +51,7 @@ def parse():
     ap.add_argument("--copy-check", action="store_true",
                     help="also time a sustained torch copy of the same byte volume (context for the roofline)")
     a = ap.parse_args()
-    a.n = tuple(a.n * 3 if len(a.n) == 1 else a.n)
+    a.n = tuple(a.grid * 3 if len(a.grid) == 1 else a.grid)
     return a
 
 

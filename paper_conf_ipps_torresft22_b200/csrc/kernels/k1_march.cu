@@ -23,6 +23,8 @@
 // planes from L2, not DRAM.
 #include <cuda.h>
 
+#include <algorithm>
+
 #include "../kernels.hpp"
 #include "node_math.cuh"
 #include "signal.cuh"
@@ -47,7 +49,8 @@ constexpr int kVBoxBytes = kTK * kTJ * 3 * 8;   // 6144
 constexpr int kXSlot = 8704;                    // 128-byte aligned slots
 constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 14848
 constexpr int kStages = 4;
-constexpr int kSegPlanes = 64;                  // planes per CTA march (segment)
+constexpr int kSegPlanes = 64;                  // max planes per CTA march (segment)
+constexpr int kMinSegPlanes = 4;                // min planes per segment (small grids)
 
 struct __align__(16) Smem {
     unsigned char stage[kStages][kStageBytes];
@@ -267,8 +270,16 @@ cudaError_t launch_k1_march(const StepArgs& a, bool unit_mass, cudaStream_t stre
     mp.a = a;
     mp.tiles_k = (int)((a.g.n2 + kTK - 1) / kTK);
     const int tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
-    mp.seg_planes = kSegPlanes;
-    const int nseg = (int)((a.g.size + kSegPlanes - 1) / kSegPlanes);
+    // Segments of <= kSegPlanes planes; on small grids shorter segments so that
+    // the grid still holds ~4 waves of CTAs (148 SMs x 2 CTAs): each segment
+    // costs one extra plane of X (L2) and one pipeline fill.
+    const int tiles = mp.tiles_k * tiles_j;
+    const int want_ctas = 4 * 148 * K1_MIN_BLOCKS;
+    int nseg = (int)((a.g.size + kSegPlanes - 1) / kSegPlanes);
+    nseg = std::max(nseg, std::min((int)a.g.size, (want_ctas + tiles - 1) / tiles));
+    mp.seg_planes = (int)((a.g.size + nseg - 1) / nseg);
+    if (mp.seg_planes < kMinSegPlanes) mp.seg_planes = (int)std::min<int64_t>(kMinSegPlanes, a.g.size);
+    nseg = (int)((a.g.size + mp.seg_planes - 1) / mp.seg_planes);
     dim3 grid((unsigned)(mp.tiles_k * tiles_j), (unsigned)nseg);
     dim3 block(kTK, kTJ);
     const size_t smem = sizeof(Smem);

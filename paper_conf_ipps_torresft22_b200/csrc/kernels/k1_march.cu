@@ -48,8 +48,14 @@ constexpr int kXBoxBytes = kBK * kBJ * 3 * 8;   // 8640
 constexpr int kVBoxBytes = kTK * kTJ * 3 * 8;   // 6144
 constexpr int kXSlot = 8704;                    // 128-byte aligned slots
 constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 14848
-constexpr int kStages = 4;
-constexpr int kSegPlanes = 64;                  // max planes per CTA march (segment)
+#ifndef K1_STAGES
+#define K1_STAGES 4
+#endif
+#ifndef K1_SEG
+#define K1_SEG 64
+#endif
+constexpr int kStages = K1_STAGES;              // TMA ring depth (planes)
+constexpr int kSegPlanes = K1_SEG;              // max planes per CTA march (segment)
 constexpr int kMinSegPlanes = 4;                // min planes per segment (small grids)
 
 struct __align__(16) Smem {

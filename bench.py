@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--kernel", choices=["auto", "direct", "march"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--stream-chunk", type=int, default=32, help="planes per chunk in the host-streamed e2e")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -207,6 +208,82 @@ def run_reference(a):
 
 # --------------------------------------------------------------------------- our arm
 
+def pcie_rates(local, nbytes=1 << 30):
+    """Pinned host<->device copy rates (GB/s), one direction at a time and both
+    directions concurrently -- the roofline of the host-streamed mode."""
+    import torch
+
+    h1 = torch.empty(nbytes // 8, dtype=torch.float64, pin_memory=True)
+    h2 = torch.empty_like(h1, pin_memory=True)
+    d1 = torch.empty(nbytes // 8, dtype=torch.float64, device="cuda")
+    d2 = torch.empty_like(d1)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    res = {}
+    for name, fn in (("h2d", lambda: d1.copy_(h1, non_blocking=True)),
+                     ("d2h", lambda: h1.copy_(d1, non_blocking=True))):
+        fn()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        res[name] = 3 * nbytes / (time.perf_counter() - t0) / 1e9
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(3):
+        with torch.cuda.stream(s1):
+            d1.copy_(h1, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+    torch.cuda.synchronize()
+    res["bidir_total"] = 6 * nbytes / (time.perf_counter() - t0) / 1e9
+    del h1, h2, d1, d2
+    torch.cuda.empty_cache()
+    return res
+
+
+def e2e_stream(n, params, local, a):
+    """End to end through the public C ABI with HOST buffers: somier_stream_step
+    maps every chunk to the GPU (X with halo planes, V), runs the fused step and
+    maps X_{t+1}, V back, each step -- the paper's One Buffer `target spread`
+    cycle with double buffering (3 device slots, 3 streams). Wall-clock timed:
+    every host<->device copy is inside the timed region."""
+    import numpy as np
+    import torch
+
+    import paper_conf_ipps_torresft22_b200 as P
+
+    chunk = a.stream_chunk
+    st = P.SomierStream(P.Spread([local], 1, n[0] - 2, chunk=chunk), params, buffers=3)
+    grids = [torch.empty(tuple(n), dtype=torch.float64, pin_memory=True) for _ in range(9)]
+    X, V, XN = [g.data_ptr() for g in grids[0:3]], [g.data_ptr() for g in grids[3:6]], \
+        [g.data_ptr() for g in grids[6:9]]
+    st.generate_ptrs(X + V)
+    st.step_ptrs(X, V, XN)  # warm-up step
+    X, XN = XN, X
+    k = max(1, a.e2e_steps)
+    t0 = time.perf_counter()
+    for _ in range(k):
+        stats = st.step_ptrs(X, V, XN)
+        X, XN = XN, X
+    wall = time.perf_counter() - t0
+    tr = st.traffic()
+    st.close()
+    del grids
+    rates = pcie_rates(local)
+    bytes_step = tr["h2d_bytes"] + tr["d2h_bytes"]
+    return {"value": interior(n) * k / wall, "unit": UNIT, "h2d_bytes_per_step": tr["h2d_bytes"],
+            "d2h_bytes_per_step": tr["d2h_bytes"] + 88, "steps": k, "wall_s": wall,
+            "cycle": "somier_stream_step on pinned host grids: per chunk of %d planes map(to: X[start-1:size+2], "
+                     "V[start:size]) -> fused K1 -> map(from: X[start:size], V[start:size]); 3 device slots, "
+                     "H2D/K1/D2H overlapped; stats read back each step" % chunk,
+            "roofline": {"bound": "pcie", "achieved_gbs": bytes_step / (wall / k) / 1e9,
+                         "peak_gbs_bidir_measured": rates["bidir_total"], "h2d_gbs": rates["h2d"],
+                         "d2h_gbs": rates["d2h"],
+                         "frac": bytes_step / (wall / k) / 1e9 / rates["bidir_total"]},
+            "last_step_vmax": stats.vmax}
+
+
 def sustained_copy(device, stream, gib=6, iters=30):
     """Context only: a plain torch copy (read+write bytes) sustained back to back,
     the way K1 runs inside the bench, to compare against the burst hbm_gbs."""
@@ -330,7 +407,11 @@ def run_ours(a):
     # map(to) the whole state (X with halos, V), one step, read the centers
     # result and map(from) the state -- the paper's One Buffer cycle, in core.
     e2e = None
-    if not a.no_e2e:
+    if not a.no_e2e and not multi:
+        s.close()  # free the resident grid: the streamed mode needs only a few chunk buffers
+        torch.cuda.empty_cache()
+        e2e = e2e_stream(n, params, local, a)
+    elif not a.no_e2e:
         shape = tuple(n)
         host = [torch.empty(shape, dtype=torch.float64, pin_memory=True) for _ in range(6)]
         ptrs = [h.data_ptr() for h in host]

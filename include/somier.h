@@ -181,6 +181,56 @@ spread_status somier_destroy(somier_t h);
 /* Library version string. */
 const char* somier_version(void);
 
+/* ------------------------------------------------------------------------
+ * Host-streamed ("out-of-core") mode -- the paper's own experiment (PAPER.md
+ * §V-A/B/C, 336-659): the state lives in HOST memory and
+ * every time step streams it through the devices chunk by chunk:
+ *   target enter data spread map(to: X[start-1:size+2], V[start:size])   (H2D)
+ *   target spread ... forces/accelerations/velocities/positions/centers   (K1)
+ *   target exit data spread map(from: X[start:size], V[start:size])      (D2H)
+ * `buffers` device buffers per GPU: 1 = the paper's One Buffer (transfers and
+ * kernels serialised per chunk); >= 2 = double buffering:
+ * the H2D of the next chunk, the kernel of this one and the D2H of the
+ * previous one run concurrently on three streams. Halos come from the host
+ * copy of X_t (overlapping array sections), so no device-to-device
+ * exchange exists in this mode.
+ * ------------------------------------------------------------------------ */
+typedef struct somier_stream_s* somier_stream_t;
+
+/*
+ * somier_stream_create -- s: spread over range(1 : n0-2); each chunk is the
+ * slice one device processes at a time (Listing 10: chunk = buffer / ndevices).
+ * buffers >= 1 device slots per list device. Device memory = buffers x
+ * (3 slabs of chunk+2 planes), independent of n0: the grid may exceed HBM.
+ * Errors: EINVAL, ENODEV, ENOMEM, ECUDA.
+ */
+spread_status somier_stream_create(spread_t s, const somier_params* p, int buffers, somier_stream_t* out);
+
+/*
+ * somier_stream_generate -- write the initial state (reading S7, bit-identical
+ * to somier_init's) into caller-owned host grids (layout as in somier_read),
+ * generated on the devices chunk by chunk. Blocking.
+ */
+spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                     double* vz);
+
+/*
+ * somier_stream_step -- one time step on host-resident state: reads X_t from
+ * (x, y, z), writes X_{t+1} to (xn, yn, zn) -- every node, fixed faces
+ * included -- and updates V = (vx, vy, vz) in place. X_t and X_{t+1} must not
+ * overlap (Jacobi). `stats` (may be NULL) receives the centres / vmax of
+ * X_{t+1}, V_{t+1}. Blocking. Host grids should be page-locked for the copies
+ * to overlap with the kernels.
+ */
+spread_status somier_stream_step(somier_stream_t h, const double* x, const double* y, const double* z, double* vx,
+                                 double* vy, double* vz, double* xn, double* yn, double* zn, somier_stats_t* stats);
+
+/* Bytes moved host->device and device->host by one somier_stream_step, and
+ * K1 launches so far. */
+spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches);
+
+spread_status somier_stream_destroy(somier_stream_t h);
+
 #ifdef __cplusplus
 }
 #endif

@@ -8,10 +8,10 @@ This package is the Python binding (argument marshalling only).
 """
 from . import _native
 from ._native import K1_AUTO, K1_DIRECT, K1_MARCH, SpreadError
-from .somier import Somier, SomierParams, Stats, combine_stats
+from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
 from .spread import Chunk, Spread
 
-__all__ = ["Spread", "Chunk", "Somier", "SomierParams", "Stats", "combine_stats", "SpreadError",
+__all__ = ["Spread", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats", "combine_stats", "SpreadError",
            "K1_AUTO", "K1_DIRECT", "K1_MARCH", "version"]
 
 

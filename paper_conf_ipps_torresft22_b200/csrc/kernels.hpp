@@ -46,6 +46,9 @@ struct StepArgs {
     // kernel by value as __grid_constant__ parameters).
     const void* tmap_x_cur;
     const void* tmap_v;
+    // Host-streamed mode: x_nxt is a fresh buffer, so fixed face nodes of the
+    // owned planes are copied into it too (resident mode leaves them in place).
+    int write_fixed;
 };
 
 struct InitArgs {

@@ -67,6 +67,12 @@ __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
             st.add_velocity(v);
         } else {
             st.add_position(xp);  // fixed node: X_{t+1} == X_t, V == 0
+            if (a.write_fixed) {
+                double* xo = a.x_nxt + (p + 1) * g.plane_stride() + off;
+                xo[0] = xp.x;
+                xo[g.comp_stride()] = xp.y;
+                xo[2 * g.comp_stride()] = xp.z;
+            }
         }
     }
     block_accumulate(st, scratch, a.acc);

@@ -255,6 +255,11 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
             st.add_velocity(v);
         } else if (valid) {
             st.add_position(xc);  // fixed face node: X_{t+1} == X_t, V == 0
+            if (a.write_fixed) {
+                xo[0] = xc.x;
+                xo[cs] = xc.y;
+                xo[2 * cs] = xc.z;
+            }
         }
         xc = xni;
         xo += ps;

@@ -15,6 +15,7 @@
 #include <string>
 #include <vector>
 
+#include "driver_util.hpp"
 #include "kernels.hpp"
 #include "somier.h"
 #include "spread_impl.hpp"
@@ -409,10 +410,50 @@ void finish_stats(const somier_params* p, __int128 sums[3], unsigned long long v
 // a host grid of one component (n0 x n1 x n2, dense).
 cudaError_t copy_planes(somier_t h, double* slab, int comp, int64_t slab_plane, double* host, int64_t host_plane,
                         int64_t nplanes, cudaMemcpyKind kind, cudaStream_t s) {
-    const int64_t n1 = h->p.n[1], n2 = h->p.n[2];
+    return paper::copy_slab_planes(h->geom, slab, comp, slab_plane, host, host_plane, nplanes, kind, s);
+}
+
+}  // namespace
+
+namespace paper {
+
+spread_status check_somier_params(const somier_params* p) { return check_params(p); }
+
+void finish_somier_stats(const somier_params* p, const __int128 sums[3], unsigned long long vmax2, int64_t nodes,
+                         int64_t step, somier_stats_t* out) {
+    __int128 s[3] = {sums[0], sums[1], sums[2]};
+    finish_stats(p, s, vmax2, nodes, step, out);
+}
+
+spread_status encode_slab_tmap(CUtensorMap* map, const SlabGeom& g, double* base, int64_t planes, uint32_t box_k,
+                               uint32_t box_j) {
+    static PFN_encodeTiled encode = nullptr;
+    if (!encode) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+        if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+            PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled unavailable (%s)", cudaGetErrorString(e));
+        encode = (PFN_encodeTiled)fn;
+    }
+    const cuuint64_t dims[4] = {(cuuint64_t)g.n2, (cuuint64_t)g.n1, 3, (cuuint64_t)planes};
+    const cuuint64_t strides[3] = {(cuuint64_t)g.ld * 8, (cuuint64_t)(g.n1 * g.ld) * 8,
+                                   (cuuint64_t)(3 * g.n1 * g.ld) * 8};
+    const cuuint32_t box[4] = {box_k, box_j, 3, 1};
+    const cuuint32_t estr[4] = {1, 1, 1, 1};
+    CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, base, dims, strides, box, estr,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled failed (%d)", (int)r);
+    return SPREAD_OK;
+}
+
+cudaError_t copy_slab_planes(const SlabGeom& g, double* slab, int comp, int64_t slab_plane, double* host,
+                             int64_t host_plane, int64_t nplanes, cudaMemcpyKind kind, cudaStream_t s) {
+    const int64_t n1 = g.n1, n2 = g.n2;
     cudaMemcpy3DParms m;
     std::memset(&m, 0, sizeof m);
-    cudaPitchedPtr sp = make_cudaPitchedPtr(slab + comp * n1 * h->ld, (size_t)h->ld * sizeof(double), (size_t)n2,
+    cudaPitchedPtr sp = make_cudaPitchedPtr(slab + comp * n1 * g.ld, (size_t)g.ld * sizeof(double), (size_t)n2,
                                             (size_t)(3 * n1));
     cudaPitchedPtr hp = make_cudaPitchedPtr(host, (size_t)n2 * sizeof(double), (size_t)n2, (size_t)n1);
     if (kind == cudaMemcpyDeviceToHost) {
@@ -431,7 +472,7 @@ cudaError_t copy_planes(somier_t h, double* slab, int comp, int64_t slab_plane, 
     return cudaMemcpy3DAsync(&m, s);
 }
 
-}  // namespace
+}  // namespace paper
 
 extern "C" {
 

@@ -1,0 +1,350 @@
+// somier_stream.cpp -- host-streamed ("out-of-core") Somier: the paper's own
+// experiment (§V-A..C, 336-659) on B200. The state stays in host
+// memory; each time step maps every chunk of the spread to its device
+// (X[start-1 : size+2] and V[start : size]), runs the
+// fused K1 on it, and maps X[start : size], V[start : size] back
+// (PAPER.md:218-219). With `buffers` >= 2 device slots the H2D of chunk m+1,
+// K1 of chunk m and the D2H of chunk m-1 overlap on three streams -- the
+// paper's double buffering expressed with CUDA streams and
+// events instead of OpenMP tasks and `depend`.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "driver_util.hpp"
+#include "kernels.hpp"
+#include "somier.h"
+#include "spread_impl.hpp"
+#include "status.hpp"
+
+using paper::set_last_error;
+
+namespace {
+
+struct Slot {
+    void* base = nullptr;
+    double* x_in = nullptr;   // X_t of the chunk, size+2 planes (halo planes included)
+    double* x_out = nullptr;  // X_{t+1}, planes 1..size written by K1
+    double* v = nullptr;      // V of the chunk, size planes
+    alignas(64) CUtensorMap tmap_x;
+    alignas(64) CUtensorMap tmap_v;
+    cudaEvent_t h2d_done = nullptr, comp_done = nullptr, d2h_done = nullptr;
+    bool used = false;
+};
+
+struct Dev {
+    int pos = 0, device = 0;
+    cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
+    std::vector<Slot> slots;
+    void* acc_base = nullptr;  // StatsAccum[2]: chunk sums, fixed end planes
+    std::vector<int64_t> chunks;
+    paper::StatsAccum* acc() const { return (paper::StatsAccum*)acc_base; }
+};
+
+}  // namespace
+
+struct somier_stream_s {
+    somier_params p{};
+    spread_s spread;
+    paper::SlabGeom geom{};
+    int buffers = 1;
+    int64_t max_chunk = 0;
+    int64_t step = 0;
+    int64_t launches = 0;
+    std::vector<Dev> devs;
+    std::string sticky;
+};
+
+namespace {
+
+spread_status sfail(somier_stream_t h, cudaError_t e, const char* what) {
+    std::string msg = std::string(what) + ": " + cudaGetErrorString(e);
+    if (h && h->sticky.empty()) h->sticky = msg;
+    set_last_error("%s", msg.c_str());
+    return e == cudaErrorMemoryAllocation ? SPREAD_ENOMEM : SPREAD_ECUDA;
+}
+
+#define S_TRY(h, call)                                        \
+    do {                                                      \
+        cudaError_t e_ = (call);                              \
+        if (e_ != cudaSuccess) return sfail((h), e_, #call);  \
+    } while (0)
+
+size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+void destroy_all(somier_stream_t h) {
+    for (auto& d : h->devs) {
+        cudaSetDevice(d.device);
+        for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
+            if (s) cudaStreamSynchronize(s);
+        for (auto& sl : d.slots) {
+            for (cudaEvent_t e : {sl.h2d_done, sl.comp_done, sl.d2h_done})
+                if (e) cudaEventDestroy(e);
+            if (sl.base) cudaFree(sl.base);
+        }
+        if (d.acc_base) cudaFree(d.acc_base);
+        for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
+            if (s) cudaStreamDestroy(s);
+    }
+    h->devs.clear();
+}
+
+paper::SlabGeom geom_of(const somier_stream_s* h, const paper::ChunkInfo& c) {
+    paper::SlabGeom g = h->geom;
+    g.start = c.start;
+    g.size = c.size;
+    return g;
+}
+
+spread_status sync_devs(somier_stream_t h) {
+    for (auto& d : h->devs) {
+        cudaError_t e = cudaSetDevice(d.device);
+        for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
+            if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) return sfail(h, e, "somier_stream: synchronize");
+    }
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    return SPREAD_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+spread_status somier_stream_create(spread_t s, const somier_params* p, int buffers, somier_stream_t* out) {
+    if (!out) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: out is NULL");
+    *out = nullptr;
+    if (!s) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: spread is NULL");
+    spread_status st = paper::check_somier_params(p);
+    if (st != SPREAD_OK) return st;
+    if (buffers < 1 || buffers > 16) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: buffers %d outside [1, 16]", buffers);
+    if (s->range_start != 1 || s->range_len != p->n[0] - 2)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: spread range must be range(1:%lld)", (long long)(p->n[0] - 2));
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) PAPER_FAIL(SPREAD_ENODEV, "somier_stream_create: no CUDA device (%s)", cudaGetErrorString(e));
+    for (int id : s->devices)
+        if (id >= ndev) PAPER_FAIL(SPREAD_ENODEV, "somier_stream_create: device %d not present (%d visible)", id, ndev);
+
+    somier_stream_s* h = new (std::nothrow) somier_stream_s;
+    if (!h) PAPER_FAIL(SPREAD_ENOMEM, "somier_stream_create: out of host memory");
+    h->p = *p;
+    h->spread = *s;
+    h->buffers = buffers;
+    h->geom = paper::SlabGeom{p->n[0], p->n[1], p->n[2], paper::slab_ld(p->n[2]), 0, 0};
+    h->max_chunk = std::min<int64_t>(s->chunk, s->range_len);
+    h->devs.resize(s->devices.size());
+    for (size_t q = 0; q < s->devices.size(); q++) {
+        h->devs[q].pos = (int)q;
+        h->devs[q].device = s->devices[q];
+    }
+    for (int64_t c = 0; c < s->nchunks; c++) h->devs[s->chunk_info(c).pos].chunks.push_back(c);
+
+    auto fail = [&](spread_status code) {
+        std::string msg = paper::last_error();
+        destroy_all(h);
+        delete h;
+        set_last_error("%s", msg.c_str());
+        return code;
+    };
+    const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
+    const size_t xb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
+    const size_t vb = round_up(plane * (size_t)h->max_chunk, 4096);
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        if ((e = cudaSetDevice(d.device)) != cudaSuccess) return fail(sfail(h, e, "cudaSetDevice"));
+        for (cudaStream_t* ps : {&d.s_h2d, &d.s_comp, &d.s_d2h})
+            if ((e = cudaStreamCreateWithFlags(ps, cudaStreamNonBlocking)) != cudaSuccess)
+                return fail(sfail(h, e, "cudaStreamCreate"));
+        if ((e = cudaMalloc(&d.acc_base, 2 * sizeof(paper::StatsAccum))) != cudaSuccess)
+            return fail(sfail(h, e, "cudaMalloc(stats)"));
+        d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
+        for (auto& sl : d.slots) {
+            if ((e = cudaMalloc(&sl.base, 2 * xb + vb)) != cudaSuccess) return fail(sfail(h, e, "cudaMalloc(slot)"));
+            sl.x_in = (double*)sl.base;
+            sl.x_out = (double*)((char*)sl.base + xb);
+            sl.v = (double*)((char*)sl.base + 2 * xb);
+            for (cudaEvent_t* pe : {&sl.h2d_done, &sl.comp_done, &sl.d2h_done})
+                if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
+                    return fail(sfail(h, e, "cudaEventCreate"));
+            paper::SlabGeom g = h->geom;
+            st = paper::encode_slab_tmap(&sl.tmap_x, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK, paper::kXBoxJ);
+            if (st != SPREAD_OK) return fail(st);
+            st = paper::encode_slab_tmap(&sl.tmap_v, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kVBoxJ);
+            if (st != SPREAD_OK) return fail(st);
+        }
+    }
+    *out = h;
+    return SPREAD_OK;
+}
+
+spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                     double* vz) {
+    if (!h || !x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_generate: NULL argument");
+    double* X[3] = {x, y, z};
+    const int64_t n0 = h->p.n[0];
+    const size_t grid = (size_t)(h->p.n[0] * h->p.n[1] * h->p.n[2]);
+    std::memset(vx, 0, grid * sizeof(double));
+    std::memset(vy, 0, grid * sizeof(double));
+    std::memset(vz, 0, grid * sizeof(double));
+    size_t maxm = 0;
+    for (auto& d : h->devs) maxm = std::max(maxm, d.chunks.size());
+    for (size_t m = 0; m < maxm; m++) {
+        for (auto& d : h->devs) {
+            if (m >= d.chunks.size()) continue;
+            Slot& sl = d.slots[m % d.slots.size()];
+            const paper::ChunkInfo c = h->spread.chunk_info(d.chunks[m]);
+            const paper::SlabGeom g = geom_of(h, c);
+            S_TRY(h, cudaSetDevice(d.device));
+            if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_comp, sl.d2h_done, 0));
+            paper::InitArgs ia;
+            ia.x0 = sl.x_in;
+            ia.x1 = sl.x_out;  // scratch second buffer
+            ia.g = g;
+            ia.spacing = h->p.spacing;
+            ia.amplitude = h->p.amplitude;
+            ia.seed = h->p.seed;
+            S_TRY(h, paper::launch_init(ia, d.s_comp));
+            S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
+            S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
+            for (int q = 0; q < 3; q++) {
+                S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 1, X[q], c.start, c.size, cudaMemcpyDeviceToHost,
+                                                 d.s_d2h));
+                if (c.start == 1)
+                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, X[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
+                if (c.start + c.size == n0 - 1)
+                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, c.size + 1, X[q], n0 - 1, 1,
+                                                     cudaMemcpyDeviceToHost, d.s_d2h));
+            }
+            S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
+            sl.used = true;
+        }
+    }
+    return sync_devs(h);
+}
+
+spread_status somier_stream_step(somier_stream_t h, const double* x, const double* y, const double* z, double* vx,
+                                 double* vy, double* vz, double* xn, double* yn, double* zn, somier_stats_t* stats) {
+    if (!h || !x || !y || !z || !vx || !vy || !vz || !xn || !yn || !zn)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_step: NULL argument");
+    if (x == xn || y == yn || z == zn) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_step: X_t and X_{t+1} alias (Jacobi)");
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    double* X[3] = {const_cast<double*>(x), const_cast<double*>(y), const_cast<double*>(z)};
+    double* XN[3] = {xn, yn, zn};
+    double* V[3] = {vx, vy, vz};
+    const int64_t n0 = h->p.n[0];
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * sizeof(paper::StatsAccum), d.s_comp));
+    }
+    size_t maxm = 0;
+    for (auto& d : h->devs) maxm = std::max(maxm, d.chunks.size());
+    for (size_t m = 0; m < maxm; m++) {
+        for (auto& d : h->devs) {
+            if (m >= d.chunks.size()) continue;
+            Slot& sl = d.slots[m % d.slots.size()];
+            const paper::ChunkInfo c = h->spread.chunk_info(d.chunks[m]);
+            const paper::SlabGeom g = geom_of(h, c);
+            const bool first = c.start == 1, last = c.start + c.size == n0 - 1;
+            S_TRY(h, cudaSetDevice(d.device));
+            // map(to: X[start-1 : size+2], V[start : size])
+            if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
+            for (int q = 0; q < 3; q++) {
+                S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, X[q], c.start - 1, c.size + 2,
+                                                 cudaMemcpyHostToDevice, d.s_h2d));
+                S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], c.start, c.size, cudaMemcpyHostToDevice,
+                                                 d.s_h2d));
+            }
+            S_TRY(h, cudaEventRecord(sl.h2d_done, d.s_h2d));
+            // the fused step (forces, accelerations, velocities, positions, centers)
+            S_TRY(h, cudaStreamWaitEvent(d.s_comp, sl.h2d_done, 0));
+            if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, d.acc() + 1, d.s_comp));
+            if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, c.size + 1, 1, d.acc() + 1, d.s_comp));
+            paper::StepArgs a;
+            std::memset(&a, 0, sizeof a);
+            a.x_cur = sl.x_in;
+            a.x_nxt = sl.x_out;
+            a.v = sl.v;
+            a.g = g;
+            a.K = h->p.k_spring;
+            a.L = h->p.rest_len;
+            a.M = h->p.mass;
+            a.dt = h->p.dt;
+            a.acc = d.acc();
+            a.tmap_x_cur = &sl.tmap_x;
+            a.tmap_v = &sl.tmap_v;
+            a.write_fixed = 1;
+            const paper::K1Variant var =
+                h->p.kernel == SOMIER_K1_DIRECT ? paper::K1Variant::Direct : paper::K1Variant::March;
+            S_TRY(h, paper::launch_k1(var, a, h->p.mass == 1.0, d.s_comp));
+            h->launches++;
+            S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
+            // map(from: X[start : size], V[start : size]) (+ the fixed end planes)
+            S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
+            for (int q = 0; q < 3; q++) {
+                S_TRY(h, paper::copy_slab_planes(g, sl.x_out, q, 1, XN[q], c.start, c.size, cudaMemcpyDeviceToHost,
+                                                 d.s_d2h));
+                S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], c.start, c.size, cudaMemcpyDeviceToHost,
+                                                 d.s_d2h));
+                if (first)
+                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, XN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
+                if (last)
+                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, c.size + 1, XN[q], n0 - 1, 1,
+                                                     cudaMemcpyDeviceToHost, d.s_d2h));
+            }
+            S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
+            sl.used = true;
+        }
+    }
+    spread_status st = sync_devs(h);
+    if (st != SPREAD_OK) return st;
+    h->step++;
+    if (stats) {
+        __int128 sums[3] = {0, 0, 0};
+        unsigned long long vmax2 = 0;
+        for (auto& d : h->devs) {
+            if (d.chunks.empty()) continue;
+            paper::StatsAccum acc[2];
+            S_TRY(h, cudaSetDevice(d.device));
+            S_TRY(h, cudaMemcpy(acc, d.acc_base, sizeof acc, cudaMemcpyDeviceToHost));
+            for (int q = 0; q < 2; q++) {
+                for (int k = 0; k < 3; k++)
+                    sums[k] += (__int128)(((unsigned __int128)acc[q].hi[k] << 64) | acc[q].lo[k]);
+                vmax2 = std::max(vmax2, (unsigned long long)acc[q].vmax2);
+            }
+        }
+        paper::finish_somier_stats(&h->p, sums, vmax2, h->p.n[0] * h->p.n[1] * h->p.n[2], h->step, stats);
+    }
+    return SPREAD_OK;
+}
+
+spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_traffic: NULL handle");
+    const int64_t plane = 3 * h->p.n[1] * h->p.n[2] * (int64_t)sizeof(double);
+    int64_t in = 0, outb = 0;
+    for (int64_t c = 0; c < h->spread.nchunks; c++) {
+        const paper::ChunkInfo ci = h->spread.chunk_info(c);
+        in += plane * (ci.size + 2) + plane * ci.size;
+        outb += 2 * plane * ci.size;
+    }
+    outb += 2 * plane;  // fixed end planes
+    if (h2d_bytes) *h2d_bytes = in;
+    if (d2h_bytes) *d2h_bytes = outb;
+    if (launches) *launches = h->launches;
+    return SPREAD_OK;
+}
+
+spread_status somier_stream_destroy(somier_stream_t h) {
+    if (!h) return SPREAD_OK;
+    destroy_all(h);
+    delete h;
+    return SPREAD_OK;
+}
+
+}  // extern "C"

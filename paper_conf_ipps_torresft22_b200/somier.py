@@ -212,3 +212,63 @@ class Somier:
     @property
     def device_bytes(self) -> int:
         return self._i64(N.lib().somier_device_bytes, "somier_device_bytes")
+
+
+class SomierStream:
+    """Host-streamed Somier (include/somier.h, somier_stream_*): the state lives
+    in host memory and each step maps every chunk of `spread` to its device,
+    runs the fused step and maps the result back -- the paper's experiment
+    (§V-A..C). buffers=1: One Buffer; >= 2: double buffering."""
+
+    def __init__(self, spread: Spread, params: SomierParams, buffers: int = 2):
+        self.params = params
+        self.spread = spread
+        self._pc = params.c()
+        h = ctypes.c_void_p()
+        N.check(N.lib().somier_stream_create(spread.handle, ctypes.byref(self._pc), int(buffers), ctypes.byref(h)),
+                "somier_stream_create")
+        self._h = h
+
+    def close(self) -> None:
+        if getattr(self, "_h", None):
+            N.lib().somier_stream_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def generate(self, X=None, V=None):
+        """Initial state (bit-identical to Somier's) into host grids; returns (X, V)."""
+        shape = (3,) + tuple(int(v) for v in self.params.n)
+        X = np.zeros(shape, np.float64) if X is None else X
+        V = np.zeros(shape, np.float64) if V is None else V
+        self.generate_ptrs([X[0], X[1], X[2], V[0], V[1], V[2]])
+        return X, V
+
+    def generate_ptrs(self, grids) -> None:
+        N.check(N.lib().somier_stream_generate(self._h, *[_dptr(g) for g in grids]), "somier_stream_generate")
+
+    def step(self, X, V, XN) -> Stats:
+        """One step: X (3 grids, read), V (3 grids, updated in place), XN (3 grids, written)."""
+        return self.step_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]])
+
+    def step_ptrs(self, X, V, XN) -> Stats:
+        out = N.somier_stats_t()
+        N.check(N.lib().somier_stream_step(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
+                                           *[_dptr(g) for g in XN], ctypes.byref(out)), "somier_stream_step")
+        return Stats.from_c(out)
+
+    def traffic(self):
+        a, b, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        N.check(N.lib().somier_stream_traffic(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)),
+                "somier_stream_traffic")
+        return {"h2d_bytes": a.value, "d2h_bytes": b.value, "launches": c.value}

@@ -1,0 +1,79 @@
+"""Host-streamed mode (somier_stream_*): the paper's
+out-of-core cycle -- per step, per chunk: map to (X with halo, V), fused step,
+map from -- bit-identical to the CPU oracle for One Buffer (1 slot) and
+double buffering (2-3 slots), any chunking."""
+import numpy as np
+import pytest
+
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+P = pytest.importorskip("paper_conf_ipps_torresft22_b200")
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def _op(sp):
+    return O.Params(n=sp.n, spacing=sp.spacing, rest_len=sp.rest_len, k_spring=sp.k_spring, mass=sp.mass,
+                    dt=sp.dt, amplitude=sp.amplitude, seed=sp.seed)
+
+
+def _stream_run(sp, steps, chunk, buffers):
+    with P.SomierStream(P.Spread([0], 1, sp.n[0] - 2, chunk=chunk), sp, buffers=buffers) as s:
+        X, V = s.generate()
+        XN = np.zeros_like(X)
+        st = None
+        for _ in range(steps):
+            st = s.step(X, V, XN)
+            X, XN = XN, X
+        tr = s.traffic()
+    return X, V, st, tr
+
+
+def test_generate_bitwise_equals_oracle_and_resident():
+    sp = P.SomierParams(n=(11, 13, 37), seed=8)
+    with P.SomierStream(P.Spread([0], 1, 9, chunk=4), sp, buffers=2) as s:
+        X, V = s.generate()
+    ref = O.init(_op(sp))
+    assert np.array_equal(X, ref.X) and not V.any()
+    with P.Somier(P.Spread([0], 1, 9), sp) as r:
+        Xr, Vr = r.read()
+    assert np.array_equal(X, Xr)
+
+
+@pytest.mark.parametrize("buffers", [1, 2, 3])
+@pytest.mark.parametrize("chunk", [3, 5, 100])
+def test_stream_steps_bitwise_equal_oracle(buffers, chunk):
+    sp = P.SomierParams(n=(14, 17, 40), seed=2)
+    X, V, st, tr = _stream_run(sp, 8, chunk, buffers)
+    ref, rst = O.run(O.init(_op(sp)), 8)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+    assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits and st.centre == rst.centre
+    nch = -(-12 // min(chunk, 12))
+    assert tr["launches"] == 8 * nch
+
+
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH])
+def test_stream_matches_resident_and_nonunit_mass(kernel):
+    sp = P.SomierParams(n=(20, 9, 33), seed=4, mass=1.7, k_spring=6.0, kernel=kernel)
+    X, V, st, _ = _stream_run(sp, 12, 6, 2)
+    with P.Somier(P.Spread([0], 1, 18, chunk=7), sp) as r:
+        r.step(12)
+        Xr, Vr = r.read()
+        sr = r.stats()
+    assert np.array_equal(X, Xr) and np.array_equal(V, Vr) and st.sums == sr.sums
+
+
+def test_stream_rejects_aliasing_and_bad_buffers():
+    sp = P.SomierParams(n=(8, 8, 8))
+    with pytest.raises(P.SpreadError):
+        P.SomierStream(P.Spread([0], 1, 6), sp, buffers=0)
+    with P.SomierStream(P.Spread([0], 1, 6), sp) as s:
+        X, V = s.generate()
+        with pytest.raises(P.SpreadError):
+            s.step(X, V, X)

@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <new>
@@ -97,6 +98,10 @@ struct somier_s {
     PFN_waitValue64 wait_value64 = nullptr;
     PFN_encodeTiled encode_tiled = nullptr;
     bool connected = true;
+    // CUDA graph of an (even, odd) step pair, when every chunk is on one stream
+    bool graph_ok = false;
+    int graph_pos = -1;
+    cudaGraphExec_t graph_exec = nullptr;
 
     bool unit_mass() const { return p.mass == 1.0; }
     paper::K1Variant variant() const {
@@ -381,6 +386,22 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         if ((c > 0 && !h->chunks[c - 1].local) || (c + 1 < h->chunks.size() && !h->chunks[c + 1].local))
             h->connected = false;
     }
+    // graph replay needs a single stream and no flag protocol (SOMIER_NO_GRAPH=1 disables it)
+    {
+        int pos = -1;
+        bool one = true;
+        for (auto& c : h->chunks) {
+            if (!c.local) {
+                one = false;
+                break;
+            }
+            if (pos < 0) pos = c.pos;
+            if (c.pos != pos) one = false;
+        }
+        const char* ng = std::getenv("SOMIER_NO_GRAPH");
+        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1');
+        h->graph_pos = pos;
+    }
     *out = h;
     return SPREAD_OK;
 }
@@ -473,6 +494,14 @@ cudaError_t copy_slab_planes(const SlabGeom& g, double* slab, int comp, int64_t 
 }
 
 }  // namespace paper
+
+extern "C" {
+
+}  // extern "C"
+
+namespace {
+spread_status enqueue_steps(somier_t h, int64_t nsteps);
+}
 
 extern "C" {
 
@@ -582,6 +611,50 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_step: nsteps < 0");
     if (!h->connected) PAPER_FAIL(SPREAD_ESTATE, "somier_step: remote neighbour chunks not connected (somier_ipc_connect)");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    // All chunks on one stream (no cross-stream flags): the launches of two
+    // consecutive steps depend only on the buffer parity, so a CUDA graph of an
+    // (even, odd) step pair is captured once and replayed.
+    if (h->graph_ok && nsteps >= 2) {
+        if (h->step & 1) {
+            spread_status st = enqueue_steps(h, 1);
+            if (st != SPREAD_OK) return st;
+            nsteps--;
+        }
+        DevCtx& d = h->devs[h->graph_pos];
+        if (!h->graph_exec && nsteps >= 2) {
+            CUDA_TRY(h, cudaSetDevice(d.device));
+            CUDA_TRY(h, cudaStreamBeginCapture(d.stream, cudaStreamCaptureModeThreadLocal));
+            const int64_t s0 = h->step, l0 = h->launches;
+            spread_status st = enqueue_steps(h, 2);
+            h->step = s0;
+            h->launches = l0;
+            cudaGraph_t g = nullptr;
+            cudaError_t e = cudaStreamEndCapture(d.stream, &g);
+            if (st != SPREAD_OK) return st;
+            if (e != cudaSuccess) return cuda_fail(h, e, "somier_step: graph capture");
+            e = cudaGraphInstantiate(&h->graph_exec, g, 0);
+            cudaGraphDestroy(g);
+            if (e != cudaSuccess) return cuda_fail(h, e, "somier_step: graph instantiate");
+        }
+        if (h->graph_exec) {
+            CUDA_TRY(h, cudaSetDevice(d.device));
+            int64_t nloc = 0;
+            for (auto& c : h->chunks) nloc += c.local ? 1 : 0;
+            for (; nsteps >= 2; nsteps -= 2) {
+                CUDA_TRY(h, cudaGraphLaunch(h->graph_exec, d.stream));
+                h->step += 2;
+                h->launches += 2 * nloc;
+            }
+        }
+    }
+    return enqueue_steps(h, nsteps);
+}
+
+}  // extern "C"
+
+namespace {
+
+spread_status enqueue_steps(somier_t h, int64_t nsteps) {
     const int64_t nch = (int64_t)h->chunks.size();
     int cur_dev = -1;
     for (int64_t s = 0; s < nsteps; s++) {
@@ -639,6 +712,10 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     }
     return SPREAD_OK;
 }
+
+}  // namespace
+
+extern "C" {
 
 spread_status somier_sync(somier_t h) {
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_sync: NULL handle");
@@ -806,6 +883,7 @@ spread_status somier_destroy(somier_t h) {
             cudaSetDevice(d.device);
             cudaStreamSynchronize(d.stream);
         }
+    if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
     free_all(h);
     delete h;
     return SPREAD_OK;

@@ -1,0 +1,45 @@
+"""CUDA-graph replay of (even, odd) step pairs: any split of
+the step count, starting on either parity, gives the oracle's bits; launch
+counting stays exact; SOMIER_NO_GRAPH=1 (eager launches) gives the same bits."""
+import os
+
+import numpy as np
+import pytest
+
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+P = pytest.importorskip("paper_conf_ipps_torresft22_b200")
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+@pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7)])
+@pytest.mark.parametrize("chunk", [0, 4])
+def test_graph_splits_bitwise(splits, chunk):
+    sp = P.SomierParams(n=(12, 10, 36), seed=3)
+    with P.Somier(P.Spread([0], 1, 10, chunk=chunk), sp) as s:
+        for k in splits:
+            s.step(k)
+        X, V = s.read()
+        st = s.stats()
+        nloc = s.local_chunks
+        assert s.launches == 13 * nloc
+    ref, rst = O.run(O.init(O.Params(n=sp.n, seed=3)), 13)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V) and st.sums == rst.sums
+
+
+def test_eager_and_graph_identical(monkeypatch):
+    sp = P.SomierParams(n=(16, 16, 40), seed=9)
+    outs = []
+    for env in ("0", "1"):
+        monkeypatch.setenv("SOMIER_NO_GRAPH", env)
+        with P.Somier(P.Spread([0], 1, 14, chunk=5), sp) as s:
+            s.step(20)
+            outs.append(s.read())
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])

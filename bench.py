@@ -40,7 +40,7 @@ def parse():
     ap.add_argument("--grid", type=int, nargs="+", default=[512],
                     help="grid nodes (one value: cube); not --n, which torch.distributed.run would claim")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--kernel", choices=["auto", "direct", "march"], default="auto")
+    ap.add_argument("--kernel", choices=["auto", "direct", "march", "march2"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--stream-chunk", type=int, default=32, help="planes per chunk in the host-streamed e2e")
@@ -340,7 +340,7 @@ def run_ours(a):
         torch.distributed.all_reduce(t)
         return int(t.item())
     n = a.n
-    kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH}[a.kernel]
+    kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH, "march2": P.K1_MARCH2}[a.kernel]
     params = P.SomierParams(n=n, seed=42, kernel=kernel)
     if multi:
         s = PD.open_local(params, chunk=a.chunk, cuda_device=local)
@@ -398,7 +398,7 @@ def run_ours(a):
     alg = algorithmic_bytes(n, c0.start, c0.size)
     peak, peak_src = load_peaks()
     achieved = alg / (k1_ms * 1e-3) / 1e9
-    kname = "march" if kernel in (P.K1_AUTO, P.K1_MARCH) else "direct"
+    kname = {P.K1_AUTO: "march2", P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct"}[kernel]
     traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()

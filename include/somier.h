@@ -49,9 +49,10 @@ extern "C" {
 
 /* K1 implementations (all compute bit-identical results). */
 typedef enum {
-    SOMIER_K1_AUTO = 0,      /* the fastest available (currently SOMIER_K1_MARCH)     */
+    SOMIER_K1_AUTO = 0,      /* the fastest available (currently SOMIER_K1_MARCH2)    */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
-    SOMIER_K1_MARCH = 2      /* plane-marching, smem-staged, 3 springs/node with reuse */
+    SOMIER_K1_MARCH = 2,     /* plane-marching, smem-staged, 3 springs/node with reuse */
+    SOMIER_K1_MARCH2 = 3     /* as MARCH with two rows per warp (32 x 16 tiles)        */
 } somier_kernel;
 
 typedef struct {

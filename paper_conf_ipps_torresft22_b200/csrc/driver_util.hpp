@@ -30,6 +30,18 @@ spread_status encode_slab_tmap(CUtensorMap* map, const SlabGeom& g, double* base
 
 // Box shapes K1_MARCH expects for the X and V maps.
 constexpr uint32_t kXBoxK = 36, kXBoxJ = 10, kVBoxK = 32, kVBoxJ = 8;
+// ... and K1_MARCH2 (two rows per warp, 32 x 16 tiles)
+constexpr uint32_t kX2BoxJ = 18, kV2BoxJ = 16;
+
+// somier_params.kernel -> K1 implementation (AUTO = the fastest measured)
+inline K1Variant k1_variant(int32_t kernel) {
+    switch (kernel) {
+        case SOMIER_K1_DIRECT: return K1Variant::Direct;
+        case SOMIER_K1_MARCH: return K1Variant::March;
+        case SOMIER_K1_MARCH2: return K1Variant::March2;
+        default: return K1Variant::March2;  // measured fastest at 512^3
+    }
+}
 
 // Row pitch (doubles) of a slab for rows of n2 nodes: 256-byte aligned rows.
 inline int64_t slab_ld(int64_t n2) { return (n2 + 31) / 32 * 32; }

@@ -46,6 +46,9 @@ struct StepArgs {
     // kernel by value as __grid_constant__ parameters).
     const void* tmap_x_cur;
     const void* tmap_v;
+    // K1_MARCH2 (32 x 16 tiles): the same slabs with its box shapes
+    const void* tmap_x2_cur;
+    const void* tmap_v2;
     // Host-streamed mode: x_nxt is a fresh buffer, so fixed face nodes of the
     // owned planes are copied into it too (resident mode leaves them in place).
     int write_fixed;
@@ -59,7 +62,7 @@ struct InitArgs {
     uint64_t seed;
 };
 
-enum class K1Variant { Direct = 1, March = 2 };
+enum class K1Variant { Direct = 1, March = 2, March2 = 3 };
 
 cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);

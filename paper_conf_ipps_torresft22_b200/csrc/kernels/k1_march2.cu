@@ -1,0 +1,268 @@
+// k1_march2.cu -- SOMIER_K1_MARCH2: K1_MARCH with two rows per warp.
+//
+// Same arithmetic (node_math.cuh; bit-identical) and the same TMA ring, but a
+// CTA owns a 32 (k) x 16 (j) tile and warp w handles the ADJACENT rows 2w and
+// 2w+1. The -j spring of row 2w+1 is then the +j spring of row 2w, already in
+// the thread's registers; only row 2w's -j crosses warps (shared memory). Per
+// plane, the fixed costs -- mbarrier wait, CTA barrier, stage rotation, the
+// tile-border springs, pointer updates -- are paid once per 64 node-updates
+// per warp instead of 32, and the two rows' springs give each thread twice the
+// independent fp64 work to hide latency with. K1 is energy-bound under the
+// 1 kW cap, so fewer issued instructions per node is the lever.
+#include <cuda.h>
+
+#include <algorithm>
+
+#include "../kernels.hpp"
+#include "node_math.cuh"
+#include "signal.cuh"
+#include "stats.cuh"
+#include "tma.cuh"
+
+namespace paper {
+
+namespace {
+
+constexpr int kTK = 32;                 // tile width along k (one warp)
+constexpr int kW = 8;                   // warps per CTA
+constexpr int kTJ = 2 * kW;             // tile height along j: two rows per warp
+constexpr int kThreads = kTK * kW;
+constexpr int kBK = kTK + 4;            // X box columns k0-2 .. k0+33
+constexpr int kBJ = kTJ + 2;            // X box rows j0-1 .. j0+16
+constexpr int kCol0 = 2;
+constexpr int kXBoxBytes = kBK * kBJ * 3 * 8;     // 15552
+constexpr int kVBoxBytes = kTK * kTJ * 3 * 8;     // 12288
+constexpr int kXSlot = 15616;                     // 128-byte aligned
+constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 27904
+#ifndef K1M2_STAGES
+#define K1M2_STAGES 3
+#endif
+constexpr int kStages = K1M2_STAGES;
+constexpr int kSegPlanes = 64;
+constexpr int kMinSegPlanes = 4;
+constexpr int kXComp = kBJ * kBK, kVComp = kTJ * kTK;
+
+struct __align__(16) Smem {
+    unsigned char stage[kStages][kStageBytes];
+    Vec3 gj[2][kW][kTK];   // +j springs of each warp's second row, by plane parity
+    Vec3 gbj[2][kTK];      // tile-border springs (j0-1 -> j0)
+    Vec3 gbk[2][kTJ];      // tile-border springs (k0-1 -> k0), per row
+    unsigned long long full[kStages];
+    WarpStats scratch[kThreads / 32];
+};
+
+struct March2Params {
+    StepArgs a;
+    int tiles_k;
+    int seg_planes;
+};
+
+__device__ __forceinline__ Vec3 shfl_up1(const Vec3& v) {
+    return Vec3{__shfl_up_sync(0xffffffffu, v.x, 1), __shfl_up_sync(0xffffffffu, v.y, 1),
+                __shfl_up_sync(0xffffffffu, v.z, 1)};
+}
+
+__device__ __forceinline__ Vec3 ld3(const double* p) { return Vec3{p[0], p[kXComp], p[2 * kXComp]}; }
+
+template <bool kUnitMass, bool kPosK>
+__device__ __forceinline__ void update_node(bool interior, bool valid, bool write_fixed, const Vec3& F, const double* vb,
+                                            const Vec3& xc, double* vo, double* xo, int64_t cs, double* lo_dst,
+                                            double* hi_dst, int64_t off, const StepArgs& a, NodeStats& st) {
+    if (interior) {
+        Vec3 v{vb[0], vb[kVComp], vb[2 * kVComp]};
+        Vec3 xn;
+        kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
+        vo[0] = v.x;
+        vo[cs] = v.y;
+        vo[2 * cs] = v.z;
+        xo[0] = xn.x;
+        xo[cs] = xn.y;
+        xo[2 * cs] = xn.z;
+        if (lo_dst) {
+            lo_dst[off] = xn.x;
+            lo_dst[off + cs] = xn.y;
+            lo_dst[off + 2 * cs] = xn.z;
+        }
+        if (hi_dst) {
+            hi_dst[off] = xn.x;
+            hi_dst[off + cs] = xn.y;
+            hi_dst[off + 2 * cs] = xn.z;
+        }
+        st.add_position(xn);
+        st.add_velocity(v);
+    } else if (valid) {
+        st.add_position(xc);
+        if (write_fixed) {
+            xo[0] = xc.x;
+            xo[cs] = xc.y;
+            xo[2 * cs] = xc.z;
+        }
+    }
+}
+
+template <bool kUnitMass, bool kPosK>
+__global__ void __launch_bounds__(kThreads, 2)
+    k1_march2_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
+                     const March2Params mp) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Smem& sm = *reinterpret_cast<Smem*>(smem_raw);
+    const StepArgs& a = mp.a;
+    const SlabGeom& g = a.g;
+    const int lane = threadIdx.x;
+    const int w = threadIdx.y;
+    const int tid = w * kTK + lane;
+    const int tile_k = blockIdx.x % mp.tiles_k;
+    const int tile_j = blockIdx.x / mp.tiles_k;
+    const int k0 = tile_k * kTK, j0 = tile_j * kTJ;
+    const int k = k0 + lane;
+    const int jA = j0 + 2 * w, jB = jA + 1;
+    const int ck = lane + kCol0;
+    const int rA = 2 * w + 1, rB = rA + 1;  // box rows
+    const int pb = 1 + blockIdx.y * mp.seg_planes;
+    const int pe = min((int)g.size + 1, pb + mp.seg_planes);
+    const int q0 = pb - 1;
+    const int qlast = pe;
+
+    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
+        reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
+
+    auto issue = [&](int q) {
+        const int s = (q - q0) % kStages;
+        unsigned char* stg = sm.stage[s];
+        const bool with_v = q >= pb + 1;
+        mbar_expect_tx(&sm.full[s], kXBoxBytes + (with_v ? kVBoxBytes : 0));
+        tma_load_4d(stg, &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);
+        if (with_v) tma_load_4d(stg + kXSlot, &tmap_v, k0, j0, 0, q - 2, &sm.full[s]);
+    };
+    if (tid == 0) {
+        prefetch_tmap(&tmap_x);
+        prefetch_tmap(&tmap_v);
+        for (int s = 0; s < kStages; s++) mbar_init(&sm.full[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        fence_proxy_async();
+        for (int q = q0; q < q0 + kStages && q <= qlast; q++) issue(q);
+    }
+    __syncthreads();
+
+    const bool kin = k >= 1 && k < g.n2 - 1, kval = k < g.n2;
+    const bool validA = kval && jA < g.n1, validB = kval && jB < g.n1;
+    const bool intA = kin && jA >= 1 && jA < g.n1 - 1, intB = kin && jB >= 1 && jB < g.n1 - 1;
+    const int64_t cs = g.comp_stride(), ps = g.plane_stride();
+    const int64_t offA = (int64_t)jA * g.ld + k, offB = offA + g.ld;
+    const int xA = rA * kBK + ck, xB = xA + kBK;
+    const int vA = (2 * w) * kTK + lane, vB = vA + kTK;
+    auto stage_x = [&](int s) { return reinterpret_cast<const double*>(smem_raw + s * kStageBytes); };
+
+    // prologue: +i springs of plane pb-1 (the -i springs of plane pb)
+    {
+        const int s0 = 0, s1 = 1;
+        mbar_wait(&sm.full[s0], 0);
+        mbar_wait(&sm.full[s1], 0);
+    }
+    Vec3 carryA = spring_force<kPosK>(ld3(stage_x(0) + xA), ld3(stage_x(1) + xA), a.K, a.L);
+    Vec3 carryB = spring_force<kPosK>(ld3(stage_x(0) + xB), ld3(stage_x(1) + xB), a.K, a.L);
+    Vec3 xcA = ld3(stage_x(1) + xA), xcB = ld3(stage_x(1) + xB);
+    __syncthreads();
+    if (tid == 0 && q0 + kStages <= qlast) {
+        fence_proxy_async();
+        issue(q0 + kStages);
+    }
+
+    double* xo = a.x_nxt + (int64_t)pb * ps + offA;
+    double* vo = a.v + (int64_t)(pb - 1) * ps + offA;
+    int s_cur = 1, s_nxt = 2 % kStages;
+    unsigned ph_nxt = (2 / kStages) & 1;
+    NodeStats st;
+    st.zero();
+#pragma unroll 1
+    for (int p = pb; p < pe; p++) {
+        const int par = p & 1;
+        mbar_wait(&sm.full[s_nxt], ph_nxt);
+        const double* Xc = stage_x(s_cur);
+        const double* Xn = stage_x(s_nxt);
+        // ---- phase 1: "+" springs of both rows (+j of row A uses row B's position)
+        const Vec3 gpkA = spring_force<kPosK>(xcA, ld3(Xc + xA + 1), a.K, a.L);
+        const Vec3 gpkB = spring_force<kPosK>(xcB, ld3(Xc + xB + 1), a.K, a.L);
+        const Vec3 gpjA = spring_force<kPosK>(xcA, xcB, a.K, a.L);
+        const Vec3 gpjB = spring_force<kPosK>(xcB, ld3(Xc + xB + kBK), a.K, a.L);
+        sm.gj[par][w][lane] = gpjB;
+        const Vec3 niA = ld3(Xn + xA), niB = ld3(Xn + xB);
+        const Vec3 gpiA = spring_force<kPosK>(xcA, niA, a.K, a.L);
+        const Vec3 gpiB = spring_force<kPosK>(xcB, niB, a.K, a.L);
+        if (w == 0) {
+            sm.gbj[par][lane] = spring_force<kPosK>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
+        } else if (w == 1 && lane < kTJ) {
+            const double* b = Xc + (lane + 1) * kBK + kCol0;
+            sm.gbk[par][lane] = spring_force<kPosK>(ld3(b - 1), ld3(b), a.K, a.L);
+        }
+        const Vec3 upA = shfl_up1(gpkA), upB = shfl_up1(gpkB);
+        __syncthreads();
+        if (tid == 0 && p + kStages <= qlast) {
+            fence_proxy_async();
+            issue(p + kStages);
+        }
+        // ---- phase 2
+        const double* Vb = reinterpret_cast<const double*>(smem_raw + s_nxt * kStageBytes + kXSlot);
+        {
+            const Vec3 gmj = neg(w == 0 ? sm.gbj[par][lane] : sm.gj[par][w - 1][lane]);
+            const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w] : upA);
+            const Vec3 F = sum_forces(neg(carryA), gpiA, gmj, gpjA, gmk, gpkA);
+            update_node<kUnitMass, kPosK>(intA, validA, a.write_fixed, F, Vb + vA, xcA, vo, xo, cs,
+                                          (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offA,
+                                          a, st);
+        }
+        {
+            const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w + 1] : upB);
+            const Vec3 F = sum_forces(neg(carryB), gpiB, neg(gpjA), gpjB, gmk, gpkB);
+            update_node<kUnitMass, kPosK>(intB, validB, a.write_fixed, F, Vb + vB, xcB, vo + g.ld, xo + g.ld, cs,
+                                          (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offB,
+                                          a, st);
+        }
+        carryA = gpiA;
+        carryB = gpiB;
+        xcA = niA;
+        xcB = niB;
+        xo += ps;
+        vo += ps;
+        s_cur = s_nxt;
+        s_nxt = (s_nxt + 1 == kStages) ? 0 : s_nxt + 1;
+        ph_nxt ^= (s_nxt == 0) ? 1u : 0u;
+    }
+    block_accumulate(st, sm.scratch, a.acc);
+    signal_neighbours(a);
+}
+
+}  // namespace
+
+cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t stream) {
+    if (a.g.size <= 0) return cudaSuccess;
+    if (!a.tmap_x_cur || !a.tmap_v2) return cudaErrorInvalidValue;
+    March2Params mp;
+    mp.a = a;
+    mp.tiles_k = (int)((a.g.n2 + kTK - 1) / kTK);
+    const int tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
+    const int tiles = mp.tiles_k * tiles_j;
+    const int want_ctas = 4 * 148 * 2;
+    int nseg = (int)((a.g.size + kSegPlanes - 1) / kSegPlanes);
+    nseg = std::max(nseg, std::min((int)a.g.size, (want_ctas + tiles - 1) / tiles));
+    mp.seg_planes = (int)((a.g.size + nseg - 1) / nseg);
+    if (mp.seg_planes < kMinSegPlanes) mp.seg_planes = (int)std::min<int64_t>(kMinSegPlanes, a.g.size);
+    nseg = (int)((a.g.size + mp.seg_planes - 1) / mp.seg_planes);
+    dim3 grid((unsigned)tiles, (unsigned)nseg);
+    dim3 block(kTK, kW);
+    const size_t smem = sizeof(Smem);
+    const CUtensorMap& mx = *static_cast<const CUtensorMap*>(a.tmap_x2_cur);
+    const CUtensorMap& mv = *static_cast<const CUtensorMap*>(a.tmap_v2);
+    auto launch = [&](auto kernel) {
+        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        kernel<<<grid, block, smem, stream>>>(mx, mv, mp);
+    };
+    const bool pos_k = a.K > 0.0;
+    if (unit_mass)
+        pos_k ? launch(k1_march2_kernel<true, true>) : launch(k1_march2_kernel<true, false>);
+    else
+        pos_k ? launch(k1_march2_kernel<false, true>) : launch(k1_march2_kernel<false, false>);
+    return cudaGetLastError();
+}
+
+}  // namespace paper

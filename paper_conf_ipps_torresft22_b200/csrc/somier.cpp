@@ -54,6 +54,8 @@ struct Chunk {
     // TMA descriptors of the local slabs (K1_MARCH): X buffers 0/1 and V
     alignas(64) CUtensorMap tmap_x[2];
     alignas(64) CUtensorMap tmap_v;
+    alignas(64) CUtensorMap tmap_x2[2];  // K1_MARCH2 box shapes
+    alignas(64) CUtensorMap tmap_v2;
 
     void* mem() const { return local ? base : remote_base; }
     double* x(int parity) const { return (double*)((char*)mem() + off_x[parity]); }
@@ -105,7 +107,7 @@ struct somier_s {
 
     bool unit_mass() const { return p.mass == 1.0; }
     paper::K1Variant variant() const {
-        return p.kernel == SOMIER_K1_DIRECT ? paper::K1Variant::Direct : paper::K1Variant::March;
+        return paper::k1_variant(p.kernel);
     }
     paper::SlabGeom geom_of(const Chunk& c) const {
         paper::SlabGeom g = geom;
@@ -146,7 +148,7 @@ spread_status check_params(const somier_params* p) {
         if (!std::isfinite(v)) PAPER_FAIL(SPREAD_EINVAL, "somier: non-finite parameter");
     if (!(p->mass > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: mass must be > 0");
     if (!(p->dt > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: dt must be > 0");
-    if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_MARCH)
+    if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_MARCH2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown kernel %d", p->kernel);
     if (p->reserved != 0) PAPER_FAIL(SPREAD_EINVAL, "somier: reserved field must be 0");
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
@@ -267,6 +269,12 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
         if (st != SPREAD_OK) return st;
     }
     spread_status st = encode_slab_map(h, &c.tmap_v, c.v(), c.size, 32, 8);
+    if (st != SPREAD_OK) return st;
+    for (int b = 0; b < 2; b++) {
+        st = paper::encode_slab_tmap(&c.tmap_x2[b], g, c.x(b), c.size + 2, paper::kXBoxK, paper::kX2BoxJ);
+        if (st != SPREAD_OK) return st;
+    }
+    st = paper::encode_slab_tmap(&c.tmap_v2, g, c.v(), c.size, paper::kVBoxK, paper::kV2BoxJ);
     if (st != SPREAD_OK) return st;
     return reset_stats(h, c);
 }
@@ -705,6 +713,8 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.done_counter = me.counter();
             a.tmap_x_cur = &me.tmap_x[cur];
             a.tmap_v = &me.tmap_v;
+            a.tmap_x2_cur = &me.tmap_x2[cur];
+            a.tmap_v2 = &me.tmap_v2;
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
             h->launches++;
         }

@@ -33,6 +33,8 @@ struct Slot {
     double* v = nullptr;      // V of the chunk, size planes
     alignas(64) CUtensorMap tmap_x;
     alignas(64) CUtensorMap tmap_v;
+    alignas(64) CUtensorMap tmap_x2;
+    alignas(64) CUtensorMap tmap_v2;
     cudaEvent_t h2d_done = nullptr, comp_done = nullptr, d2h_done = nullptr;
     bool used = false;
 };
@@ -177,6 +179,10 @@ spread_status somier_stream_create(spread_t s, const somier_params* p, int buffe
             if (st != SPREAD_OK) return fail(st);
             st = paper::encode_slab_tmap(&sl.tmap_v, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kVBoxJ);
             if (st != SPREAD_OK) return fail(st);
+            st = paper::encode_slab_tmap(&sl.tmap_x2, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK, paper::kX2BoxJ);
+            if (st != SPREAD_OK) return fail(st);
+            st = paper::encode_slab_tmap(&sl.tmap_v2, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kV2BoxJ);
+            if (st != SPREAD_OK) return fail(st);
         }
     }
     *out = h;
@@ -279,9 +285,10 @@ spread_status somier_stream_step(somier_stream_t h, const double* x, const doubl
             a.acc = d.acc();
             a.tmap_x_cur = &sl.tmap_x;
             a.tmap_v = &sl.tmap_v;
+            a.tmap_x2_cur = &sl.tmap_x2;
+            a.tmap_v2 = &sl.tmap_v2;
             a.write_fixed = 1;
-            const paper::K1Variant var =
-                h->p.kernel == SOMIER_K1_DIRECT ? paper::K1Variant::Direct : paper::K1Variant::March;
+            const paper::K1Variant var = paper::k1_variant(h->p.kernel);
             S_TRY(h, paper::launch_k1(var, a, h->p.mass == 1.0, d.s_comp));
             h->launches++;
             S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));

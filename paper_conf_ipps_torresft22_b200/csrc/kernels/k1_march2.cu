@@ -33,21 +33,30 @@ constexpr int kCol0 = 2;
 constexpr int kXBoxBytes = kBK * kBJ * 3 * 8;     // 15552
 constexpr int kVBoxBytes = kTK * kTJ * 3 * 8;     // 12288
 constexpr int kXSlot = 15616;                     // 128-byte aligned
-constexpr int kStageBytes = kXSlot + kVBoxBytes;  // 27904
+// Two TMA rings: X (needed one plane ahead, by phase 1) and V (needed by
+// phase 2 only). Measured at 512^3 (tools/variants.sh): X3+V3 5.95e10,
+// X4+V2 5.82e10 (faster in burst, slower once the power cap engages), X5+V1
+// 4.72e10 (V latency exposed). Two CTAs per SM must fit in 228 KB.
 #ifndef K1M2_STAGES
 #define K1M2_STAGES 3
 #endif
+#ifndef K1M2_VSTAGES
+#define K1M2_VSTAGES 3
+#endif
 constexpr int kStages = K1M2_STAGES;
+constexpr int kVStages = K1M2_VSTAGES;
 constexpr int kSegPlanes = 64;
 constexpr int kMinSegPlanes = 4;
 constexpr int kXComp = kBJ * kBK, kVComp = kTJ * kTK;
 
 struct __align__(16) Smem {
-    unsigned char stage[kStages][kStageBytes];
+    unsigned char xst[kStages][kXSlot];
+    unsigned char vst[kVStages][kVBoxBytes];
     Vec3 gj[2][kW][kTK];   // +j springs of each warp's second row, by plane parity
     Vec3 gbj[2][kTK];      // tile-border springs (j0-1 -> j0)
     Vec3 gbk[2][kTJ];      // tile-border springs (k0-1 -> k0), per row
     unsigned long long full[kStages];
+    unsigned long long vfull[kVStages];
     WarpStats scratch[kThreads / 32];
 };
 
@@ -126,21 +135,25 @@ __global__ void __launch_bounds__(kThreads, 2)
     if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
         reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
 
-    auto issue = [&](int q) {
+    auto issue = [&](int q) {  // X of plane q
         const int s = (q - q0) % kStages;
-        unsigned char* stg = sm.stage[s];
-        const bool with_v = q >= pb + 1;
-        mbar_expect_tx(&sm.full[s], kXBoxBytes + (with_v ? kVBoxBytes : 0));
-        tma_load_4d(stg, &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);
-        if (with_v) tma_load_4d(stg + kXSlot, &tmap_v, k0, j0, 0, q - 2, &sm.full[s]);
+        mbar_expect_tx(&sm.full[s], kXBoxBytes);
+        tma_load_4d(sm.xst[s], &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);
+    };
+    auto issue_v = [&](int p) {  // V of output plane p (V slab plane p-1)
+        const int s = (p - pb) % kVStages;
+        mbar_expect_tx(&sm.vfull[s], kVBoxBytes);
+        tma_load_4d(sm.vst[s], &tmap_v, k0, j0, 0, p - 1, &sm.vfull[s]);
     };
     if (tid == 0) {
         prefetch_tmap(&tmap_x);
         prefetch_tmap(&tmap_v);
         for (int s = 0; s < kStages; s++) mbar_init(&sm.full[s], 1);
+        for (int s = 0; s < kVStages; s++) mbar_init(&sm.vfull[s], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         fence_proxy_async();
         for (int q = q0; q < q0 + kStages && q <= qlast; q++) issue(q);
+        for (int p = pb; p < pb + kVStages && p < pe; p++) issue_v(p);
     }
     __syncthreads();
 
@@ -151,7 +164,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int64_t offA = (int64_t)jA * g.ld + k, offB = offA + g.ld;
     const int xA = rA * kBK + ck, xB = xA + kBK;
     const int vA = (2 * w) * kTK + lane, vB = vA + kTK;
-    auto stage_x = [&](int s) { return reinterpret_cast<const double*>(smem_raw + s * kStageBytes); };
+    auto stage_x = [&](int s) { return reinterpret_cast<const double*>(sm.xst[s]); };
 
     // prologue: +i springs of plane pb-1 (the -i springs of plane pb)
     {
@@ -197,12 +210,16 @@ __global__ void __launch_bounds__(kThreads, 2)
         }
         const Vec3 upA = shfl_up1(gpkA), upB = shfl_up1(gpkB);
         __syncthreads();
-        if (tid == 0 && p + kStages <= qlast) {
+        // X stage of plane p and V slot of plane p-1 are free now
+        if (tid == 0) {
             fence_proxy_async();
-            issue(p + kStages);
+            if (p + kStages <= qlast) issue(p + kStages);
+            if (p > pb && p - 1 + kVStages < pe) issue_v(p - 1 + kVStages);
         }
         // ---- phase 2
-        const double* Vb = reinterpret_cast<const double*>(smem_raw + s_nxt * kStageBytes + kXSlot);
+        const int vs = (p - pb) % kVStages;
+        mbar_wait(&sm.vfull[vs], (unsigned)(((p - pb) / kVStages) & 1));
+        const double* Vb = reinterpret_cast<const double*>(sm.vst[vs]);
         {
             const Vec3 gmj = neg(w == 0 ? sm.gbj[par][lane] : sm.gj[par][w - 1][lane]);
             const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w] : upA);

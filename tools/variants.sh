@@ -11,7 +11,7 @@ if [ "$MODE" = build ]; then
 else
   mkdir -p gpurun_out/variants
   for tag in "$@"; do
-    SOMIER_LIB=$PWD/paper_conf_ipps_torresft22_b200/libsomier_$tag.so timeout 300 python bench.py --steps 100 --warmup 5 --no-e2e --no-cpu-baseline > gpurun_out/variants/$tag.json 2>gpurun_out/variants/$tag.err
+    SOMIER_LIB=$PWD/paper_conf_ipps_torresft22_b200/libsomier_$tag.so timeout 300 python bench.py --steps 100 --warmup 5 --no-e2e --no-cpu-baseline ${VBENCH} > gpurun_out/variants/$tag.json 2>gpurun_out/variants/$tag.err
     python -c "import json;d=json.load(open('gpurun_out/variants/$tag.json'));r=d['roofline'];print('$tag', '%.4g'%d['value'], 'ms %.4f'%d['ms_per_step'], 'first5 %.4f last5 %.4f'%(r['launch_ms_distribution']['first5'], r['launch_ms_distribution']['last5']))" 2>&1 | tail -1
   done
 fi

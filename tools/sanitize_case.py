@@ -1,0 +1,27 @@
+#!/usr/bin/env python3
+"""Small runs of every kernel path for compute-sanitizer (tests/test_gpu_sanitizer.py):
+K1 direct / march / march2 over a multi-chunk spread (fused halo stores), the
+host-streamed mode, K2 and K3."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+import paper_conf_ipps_torresft22_b200 as P  # noqa: E402
+
+n = (10, 19, 37)
+for kern in (P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2):
+    sp = P.SomierParams(n=n, seed=3, kernel=kern)
+    with P.Somier(P.Spread([0], 1, n[0] - 2, chunk=3), sp) as s:
+        s.step(3)
+        s.stats()
+        X, V = s.read()
+        s.load(X, V)
+        s.step(1)
+        s.sync()
+    with P.SomierStream(P.Spread([0], 1, n[0] - 2, chunk=4), sp, buffers=2) as st:
+        X, V = st.generate()
+        XN = np.zeros_like(X)
+        st.step(X, V, XN)
+print("sanitize case ok")

@@ -78,6 +78,7 @@ SIGNATURES = [
     ("spread_get_chunk", ctypes.c_int, [_VP, ctypes.c_int64, _IP, _IP, _I64P, _I64P]),
     ("spread_chunk_of", ctypes.c_int, [_VP, ctypes.c_int64, _I64P]),
     ("spread_map_extent", ctypes.c_int, [_VP, ctypes.c_int64, spread_map, ctypes.c_int64, _I64P, _I64P]),
+    ("spread_stencil3", ctypes.c_int, [_VP, _DP, _DP, ctypes.c_int64]),
     ("spread_last_error", ctypes.c_char_p, []),
     ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),

@@ -84,6 +84,18 @@ class Spread:
         N.check(N.lib().spread_chunk_of(self._h, iteration, ctypes.byref(v)), "spread_chunk_of")
         return v.value
 
+    def stencil3(self, A, B=None):
+        """Listing 3: B[i] = A[i-1] + A[i] + A[i+1] over the spread's range, each
+        chunk computed on its device (spread_stencil3). Returns B."""
+        import numpy as np
+
+        A = np.ascontiguousarray(A, dtype=np.float64)
+        B = np.zeros_like(A) if B is None else B
+        dp = ctypes.POINTER(ctypes.c_double)
+        N.check(N.lib().spread_stencil3(self._h, A.ctypes.data_as(dp), B.ctypes.data_as(dp), A.size),
+                "spread_stencil3")
+        return B
+
     def map_extent(self, c: int, array_len: int, lo_halo: int = 0, hi_halo: int = 0, map_type: int = N.MAP_TO):
         """Section [first, first+len) of A[omp_spread_start-lo : omp_spread_size+lo+hi]."""
         first, ln = ctypes.c_int64(), ctypes.c_int64()

@@ -38,6 +38,10 @@ struct DevCtx {
     int device = -1;
     cudaStream_t own = nullptr;   // created by the library
     cudaStream_t stream = nullptr;  // in use (own or user-provided)
+    // CU_STREAM_WAIT_VALUE_FLUSH when the device supports it: remote (peer)
+    // halo stores that reached the device before the flag are made visible to
+    // the kernels after the wait
+    unsigned int wait_flush = 0;
 };
 
 // One chunk = one `target spread` iteration block (omp_spread_start/size).
@@ -357,6 +361,10 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
             return fail(SPREAD_ECUDA);
         }
         d.stream = d.own;
+        int can_flush = 0;
+        if (cudaDeviceGetAttribute(&can_flush, cudaDevAttrCanFlushRemoteWrites, d.device) == cudaSuccess && can_flush)
+            d.wait_flush = CU_STREAM_WAIT_VALUE_FLUSH;
+        cudaGetLastError();
     }
     // peer access between devices holding neighbouring local chunks
     for (size_t c = 0; c + 1 < h->chunks.size(); c++) {
@@ -685,12 +693,12 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             // about to write): flags[0] = from_left, flags[1] = from_right.
             if (t > 0 && fl) {
                 CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[0], (cuuint64_t)t,
-                                             CU_STREAM_WAIT_VALUE_GEQ);
+                                             CU_STREAM_WAIT_VALUE_GEQ | h->devs[me.pos].wait_flush);
                 if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
             }
             if (t > 0 && fr) {
                 CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[1], (cuuint64_t)t,
-                                             CU_STREAM_WAIT_VALUE_GEQ);
+                                             CU_STREAM_WAIT_VALUE_GEQ | h->devs[me.pos].wait_flush);
                 if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
             }
             paper::StepArgs a;

@@ -153,6 +153,16 @@ spread_status somier_stats_combine(const somier_stats_t* parts, int n, const som
 spread_status somier_read(somier_t h, double* x, double* y, double* z, double* vx, double* vy, double* vz);
 
 /*
+ * somier_read_planes -- `target update spread from(X[i0:count], V[i0:count])`
+ * (PAPER.md:222-243): like somier_read restricted to global planes
+ * [i0, i0+count); the six host grids hold count*n1*n2 doubles each (host plane
+ * = global plane - i0). Planes this handle does not own are left untouched.
+ * Errors: EINVAL if the range leaves [0, n0).
+ */
+spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* x, double* y, double* z, double* vx,
+                                 double* vy, double* vz);
+
+/*
  * somier_load -- update-to semantics: every owned chunk copies X[start-1 : size+2]
  * (with halos) and V[start : size] from caller-owned host grids (layout as in
  * somier_read) into device memory, and the step counter continues. Enqueued on

@@ -87,6 +87,8 @@ def lib():
         L.oracle_splitmix64_at.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
         L.oracle_rest_position.argtypes = [P, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, dp]
         L.oracle_init.argtypes = [P] + [dp] * 6
+        i64a = ctypes.POINTER(ctypes.c_int64)
+        L.oracle_init_window.argtypes = [P, i64a, i64a] + [dp] * 6
         L.oracle_spring.argtypes = [dp, dp, ctypes.c_double, ctypes.c_double, dp]
         for name in ("oracle_acceleration_1", "oracle_velocity_1", "oracle_position_1"):
             fn = getattr(L, name)
@@ -157,6 +159,21 @@ def init(p: Params) -> State:
     rc = lib().oracle_init(ctypes.byref(p.c()), *(_ptr(a) for a in (s.x, s.y, s.z, s.vx, s.vy, s.vz)))
     if rc != 0:
         raise ValueError("oracle_init rejected parameters %r" % (p,))
+    return s
+
+
+def init_window(p: Params, lo, w) -> State:
+    """Initial state of the global grid p.n restricted to [lo, lo+w); the returned
+    State is a standalone grid of shape w (its Params carry n = w)."""
+    sub = Params(n=tuple(int(v) for v in w), spacing=p.spacing, rest_len=p.rest_len, k_spring=p.k_spring,
+                 mass=p.mass, dt=p.dt, amplitude=p.amplitude, seed=p.seed)
+    s = empty(sub)
+    lo_a = (ctypes.c_int64 * 3)(*[int(v) for v in lo])
+    w_a = (ctypes.c_int64 * 3)(*[int(v) for v in w])
+    rc = lib().oracle_init_window(ctypes.byref(p.c()), lo_a, w_a,
+                                  *(_ptr(a) for a in (s.x, s.y, s.z, s.vx, s.vy, s.vz)))
+    if rc != 0:
+        raise ValueError("oracle_init_window rejected the window")
     return s
 
 

@@ -78,6 +78,37 @@ int oracle_init(const oracle_params* p, double* x, double* y, double* z,
     return 0;
 }
 
+int oracle_init_window(const oracle_params* p, const int64_t lo[3], const int64_t w[3], double* x, double* y,
+                       double* z, double* vx, double* vy, double* vz) {
+    if (!valid(p)) return -1;
+    for (int d = 0; d < 3; d++)
+        if (lo[d] < 0 || w[d] < 0 || lo[d] + w[d] > p->n[d]) return -1;
+    double* X[3] = {x, y, z};
+    for (int64_t a = 0; a < w[0]; a++)
+        for (int64_t b = 0; b < w[1]; b++)
+            for (int64_t e = 0; e < w[2]; e++) {
+                const int64_t i = lo[0] + a, j = lo[1] + b, k = lo[2] + e;
+                const int64_t g = IDX(p, i, j, k);
+                const int64_t l = (a * w[1] + b) * w[2] + e;
+                double x0[3];
+                oracle_rest_position(p, i, j, k, x0);
+                for (int c = 0; c < 3; c++) {
+                    double v = x0[c];
+                    if (is_interior(p, i, j, k)) {
+                        uint64_t r = oracle_splitmix64_at(p->seed, 3u * (uint64_t)g + (uint64_t)c);
+                        double u = (double)(r >> 11) * 0x1.0p-53;
+                        double s = 2.0 * u - 1.0;
+                        v = x0[c] + p->amplitude * s;
+                    }
+                    X[c][l] = v;
+                }
+                vx[l] = 0.0;
+                vy[l] = 0.0;
+                vz[l] = 0.0;
+            }
+    return 0;
+}
+
 void oracle_spring(const double xp[3], const double xq[3], double K, double L, double g[3]) {
     double dx = xq[0] - xp[0];
     double dy = xq[1] - xp[1];

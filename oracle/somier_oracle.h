@@ -63,6 +63,13 @@ void oracle_rest_position(const oracle_params* p, int64_t i, int64_t j, int64_t 
 int oracle_init(const oracle_params* p, double* x, double* y, double* z,
                 double* vx, double* vy, double* vz);
 
+/* The same initial state restricted to the window [lo[d], lo[d]+w[d]) of the
+ * global grid p->n (global indices, so the values equal the corresponding
+ * entries of oracle_init); arrays hold w0*w1*w2 doubles. Used to check single
+ * nodes of full-size GPU runs through their light cone. Returns 0 or -1. */
+int oracle_init_window(const oracle_params* p, const int64_t lo[3], const int64_t w[3], double* x, double* y,
+                       double* z, double* vx, double* vy, double* vz);
+
 /* One central Hooke spring (reading S1): force on node p from the spring to q.
  * d = xq - xp; |d| = sqrt((dx*dx+dy*dy)+dz*dz); f = (K*(|d|-L))/|d|; g = f*d. */
 void oracle_spring(const double xp[3], const double xq[3], double K, double L, double g[3]);

@@ -92,6 +92,7 @@ SIGNATURES = [
     ("somier_stats_combine", ctypes.c_int, [ctypes.POINTER(somier_stats_t), ctypes.c_int,
                                             ctypes.POINTER(somier_params), ctypes.POINTER(somier_stats_t)]),
     ("somier_read", ctypes.c_int, [_VP] + [_DP] * 6),
+    ("somier_read_planes", ctypes.c_int, [_VP, ctypes.c_int64, ctypes.c_int64] + [_DP] * 6),
     ("somier_load", ctypes.c_int, [_VP] + [_DP] * 6),
     ("somier_set_stream", ctypes.c_int, [_VP, ctypes.c_int, _VP]),
     ("somier_get_stream", ctypes.c_int, [_VP, ctypes.c_int, ctypes.POINTER(_VP)]),

@@ -781,35 +781,55 @@ spread_status somier_stats_combine(const somier_stats_t* parts, int n, const som
     return SPREAD_OK;
 }
 
-spread_status somier_read(somier_t h, double* x, double* y, double* z, double* vx, double* vy, double* vz) {
-    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_read: NULL handle");
+spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* x, double* y, double* z, double* vx,
+                                 double* vy, double* vz) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_read_planes: NULL handle");
+    const int64_t n0 = h->p.n[0];
+    if (i0 < 0 || count < 0 || i0 + count > n0)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_read_planes: planes [%lld, %lld) outside [0, %lld)", (long long)i0,
+                   (long long)(i0 + count), (long long)n0);
     spread_status st = sync_all(h);
     if (st != SPREAD_OK) return st;
     double* X[3] = {x, y, z};
     double* V[3] = {vx, vy, vz};
     const int cur = (int)(h->step & 1);
-    const int64_t n0 = h->p.n[0];
+    const size_t plane = (size_t)(h->p.n[1] * h->p.n[2]);
+    const int64_t i1 = i0 + count;
+    // host grids hold planes [i0, i1): global plane i -> host plane i - i0
     for (auto& c : h->chunks) {
         if (!c.local) continue;
         CUDA_TRY(h, cudaSetDevice(c.device));
         cudaStream_t s = h->stream_of(c);
-        for (int d = 0; d < 3; d++) {
-            if (X[d]) {
-                CUDA_TRY(h, copy_planes(h, c.x(cur), d, 1, X[d], c.start, c.size, cudaMemcpyDeviceToHost, s));
-                if (c.start == 1) CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, X[d], 0, 1, cudaMemcpyDeviceToHost, s));
-                if (c.start + c.size == n0 - 1)
-                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, c.size + 1, X[d], n0 - 1, 1, cudaMemcpyDeviceToHost, s));
-            }
-            if (V[d]) {
-                CUDA_TRY(h, copy_planes(h, c.v(), d, 0, V[d], c.start, c.size, cudaMemcpyDeviceToHost, s));
-                // fixed end planes have zero velocity
-                const size_t plane = (size_t)(h->p.n[1] * h->p.n[2]);
-                if (c.start == 1) std::memset(V[d], 0, plane * sizeof(double));
-                if (c.start + c.size == n0 - 1) std::memset(V[d] + (size_t)(n0 - 1) * plane, 0, plane * sizeof(double));
+        // owned planes [start, start+size) plus the fixed end planes held as halos
+        struct Span {
+            int64_t lo, hi, slab0;  // global planes [lo, hi) <- X slab plane slab0 + (i - lo)
+            bool fixed;
+        } spans[3] = {{c.start, c.start + c.size, 1, false},
+                      {0, c.start == 1 ? 1 : 0, 0, true},
+                      {n0 - 1, (c.start + c.size == n0 - 1) ? n0 : n0 - 1, c.size + 1, true}};
+        for (const Span& sp : spans) {
+            const int64_t lo = std::max(sp.lo, i0), hi = std::min(sp.hi, i1);
+            if (lo >= hi) continue;
+            for (int d = 0; d < 3; d++) {
+                if (X[d])
+                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, sp.slab0 + (lo - sp.lo), X[d], lo - i0, hi - lo,
+                                            cudaMemcpyDeviceToHost, s));
+                if (V[d]) {
+                    if (sp.fixed)  // fixed end planes have zero velocity
+                        std::memset(V[d] + (size_t)(lo - i0) * plane, 0, (size_t)(hi - lo) * plane * sizeof(double));
+                    else
+                        CUDA_TRY(h, copy_planes(h, c.v(), d, lo - c.start, V[d], lo - i0, hi - lo,
+                                                cudaMemcpyDeviceToHost, s));
+                }
             }
         }
     }
     return sync_all(h);
+}
+
+spread_status somier_read(somier_t h, double* x, double* y, double* z, double* vx, double* vy, double* vz) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_read: NULL handle");
+    return somier_read_planes(h, 0, h->p.n[0], x, y, z, vx, vy, vz);
 }
 
 spread_status somier_load(somier_t h, const double* x, const double* y, const double* z, const double* vx,

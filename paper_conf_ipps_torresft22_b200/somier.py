@@ -157,6 +157,15 @@ class Somier:
         N.check(N.lib().somier_read(self._h, *ptrs), "somier_read")
         return X, V
 
+    def read_planes(self, i0: int, count: int, X=None, V=None):
+        """target update spread from(X[i0:count], V[i0:count]): returns (X, V), each (3, count, n1, n2)."""
+        shape = (3, int(count), int(self.params.n[1]), int(self.params.n[2]))
+        X = np.zeros(shape, np.float64) if X is None else X
+        V = np.zeros(shape, np.float64) if V is None else V
+        ptrs = [_dptr(X[c]) for c in range(3)] + [_dptr(V[c]) for c in range(3)]
+        N.check(N.lib().somier_read_planes(self._h, int(i0), int(count), *ptrs), "somier_read_planes")
+        return X, V
+
     def read_ptrs(self, ptrs: Sequence[int]) -> None:
         N.check(N.lib().somier_read(self._h, *[_dptr(p) for p in ptrs]), "somier_read")
 

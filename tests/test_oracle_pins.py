@@ -82,6 +82,34 @@ def test_init_displacement_uniform_moments():
     assert abs(np.corrcoef(dd[0], dd[1])[0, 1]) < 5 / math.sqrt(dd.shape[1])
 
 
+def test_init_window_is_a_slice_of_the_full_init():
+    p = O.Params(n=(9, 11, 13), seed=5)
+    full = O.init(p)
+    for lo, w in [((0, 0, 0), (9, 11, 13)), ((2, 3, 4), (5, 6, 7)), ((8, 10, 12), (1, 1, 1))]:
+        s = O.init_window(p, lo, w)
+        sl = tuple(slice(a, a + b) for a, b in zip(lo, w))
+        assert np.array_equal(s.X, full.X[(slice(None),) + sl]) and not s.V.any()
+    with pytest.raises(ValueError):
+        O.init_window(p, (5, 0, 0), (5, 1, 1))
+
+
+def test_light_cone_window_reproduces_a_full_run_node():
+    """A node after S steps depends only on the initial state within distance S:
+    running the oracle on a window reaching S+1 beyond it reproduces the full
+    run there, bit for bit (the basis of the full-size GPU spot checks)."""
+    p = O.Params(n=(20, 21, 22), seed=6)
+    S = 4
+    full, _ = O.run(O.init(p), S)
+    for c in [(10, 10, 10), (1, 1, 1), (18, 5, 20), (6, 19, 2)]:
+        lo = [max(0, c[d] - S - 1) for d in range(3)]
+        hi = [min(p.n[d], c[d] + S + 2) for d in range(3)]
+        win = O.init_window(p, lo, [hi[d] - lo[d] for d in range(3)])
+        win, _ = O.run(win, S)
+        rel = tuple(c[d] - lo[d] for d in range(3))
+        assert np.array_equal(win.X[(slice(None),) + rel], full.X[(slice(None),) + tuple(c)])
+        assert np.array_equal(win.V[(slice(None),) + rel], full.V[(slice(None),) + tuple(c)])
+
+
 def test_init_rejects_invalid():
     for bad in [O.Params(n=(2, 5, 5)), O.Params(mass=0.0), O.Params(dt=-1.0), O.Params(k_spring=float("nan"))]:
         with pytest.raises(ValueError):

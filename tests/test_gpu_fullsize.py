@@ -1,0 +1,75 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times (single chunk, K1 AUTO): single nodes checked bit for bit through their
+light cone (a node after S steps depends only on initial values within
+distance S, so the oracle on a window reaching S+1 beyond it reproduces it
+exactly -- pinned in tests/test_oracle_pins.py), plus size-independent
+properties (rest lattice fixed point, centre exactly 0)."""
+import numpy as np
+import pytest
+
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+P = pytest.importorskip("paper_conf_ipps_torresft22_b200")
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def _samples(n, rng, count):
+    out = [(1, 1, 1), (n[0] - 2, n[1] - 2, n[2] - 2), (n[0] // 2, 1, n[2] - 2), (1, n[1] // 2, n[2] // 2),
+           (n[0] // 2, n[1] // 2, 31), (n[0] // 2, 15, 32), (65, 16, 33), (64, 17, 96)]
+    while len(out) < count:
+        out.append(tuple(int(rng.integers(1, n[d] - 1)) for d in range(3)))
+    return out
+
+
+def _check_nodes(n, steps, count, seed=42, kernel=P.K1_AUTO):
+    sp = P.SomierParams(n=n, seed=seed, kernel=kernel)
+    op = O.Params(n=n, seed=seed)
+    rng = np.random.default_rng(7)
+    nodes = _samples(n, rng, count)
+    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
+        s.step(steps)
+        got = {}
+        for c in nodes:
+            X, V = s.read_planes(c[0], 1)
+            got[c] = (X[:, 0, c[1], c[2]].copy(), V[:, 0, c[1], c[2]].copy())
+    for c in nodes:
+        lo = [max(0, c[d] - steps - 1) for d in range(3)]
+        hi = [min(n[d], c[d] + steps + 2) for d in range(3)]
+        win, _ = O.run(O.init_window(op, lo, [hi[d] - lo[d] for d in range(3)]), steps)
+        r = tuple(c[d] - lo[d] for d in range(3))
+        want_x = win.X[(slice(None),) + r]
+        want_v = win.V[(slice(None),) + r]
+        assert np.array_equal(got[c][0], want_x), (c, got[c][0], want_x)
+        assert np.array_equal(got[c][1], want_v), (c, got[c][1], want_v)
+
+
+def test_512cube_bench_config_sampled_nodes_bitwise():
+    """configs[3] (the bench workload): 512^3, 24 steps, 16 nodes."""
+    _check_nodes((512, 512, 512), 24, 16)
+
+
+def test_512cube_march_kernel_sampled_nodes_bitwise():
+    _check_nodes((512, 512, 512), 12, 6, kernel=P.K1_MARCH)
+
+
+def test_1024cube_sampled_nodes_bitwise():
+    """configs[4] grid (77 GB on one GPU): 1024^3, 10 steps, 8 nodes."""
+    _check_nodes((1024, 1024, 1024), 10, 8)
+
+
+def test_512cube_rest_lattice_fixed_point_and_zero_centre():
+    sp = P.SomierParams(n=(512, 512, 512), amplitude=0.0)
+    with P.Somier(P.Spread([0], 1, 510), sp) as s:
+        X0, _ = s.read_planes(200, 3)
+        s.step(6)
+        st = s.stats()
+        X1, V1 = s.read_planes(200, 3)
+    assert np.array_equal(X0, X1) and not V1.any()
+    assert st.centre == (0.0, 0.0, 0.0) and st.vmax == 0.0 and st.nodes == 512 ** 3

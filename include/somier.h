@@ -97,6 +97,16 @@ typedef struct somier_s* somier_t;
 spread_status somier_init(spread_t s, const somier_params* p, somier_t* out);
 
 /*
+ * somier_init_on -- somier_init with the list's device ids read as LOGICAL
+ * devices: list position q runs on CUDA device cuda_devices[q] (NULL = the
+ * ids themselves). Several positions may share one GPU; each position keeps
+ * its own stream and the cross-position protocol (in-kernel halo stores +
+ * completion flags + stream waits) runs exactly as between GPUs -- how the
+ * multi-device path is exercised on a one-GPU machine.
+ */
+spread_status somier_init_on(spread_t s, const somier_params* p, const int* cuda_devices, somier_t* out);
+
+/*
  * somier_init_local -- multi-process mode (one process per GPU): this handle owns
  * only the chunks at list position `device_pos` of `s`, on CUDA device
  * `cuda_device` of this process (-1: the id the list gives for that position;

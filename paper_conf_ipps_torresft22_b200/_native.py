@@ -82,6 +82,7 @@ SIGNATURES = [
     ("spread_last_error", ctypes.c_char_p, []),
     ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),
+    ("somier_init_on", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), _IP, ctypes.POINTER(_VP)]),
     ("somier_init_local", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.c_int, ctypes.c_int,
                                          ctypes.POINTER(_VP)]),
     ("somier_ipc_export", ctypes.c_int, [_VP, _VP, ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]),

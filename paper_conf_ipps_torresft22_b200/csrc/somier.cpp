@@ -294,7 +294,8 @@ spread_status sync_all(somier_t h) {
     return SPREAD_OK;
 }
 
-spread_status init_common(spread_t s, const somier_params* p, int local_pos, int cuda_device, somier_t* out) {
+spread_status init_common(spread_t s, const somier_params* p, int local_pos, int cuda_device, somier_t* out,
+                          const int* cuda_devices = nullptr) {
     if (!out) PAPER_FAIL(SPREAD_EINVAL, "somier_init: out is NULL");
     *out = nullptr;
     if (!s) PAPER_FAIL(SPREAD_EINVAL, "somier_init: spread is NULL");
@@ -312,8 +313,10 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
     if (local_pos >= npos) PAPER_FAIL(SPREAD_EINVAL, "somier_init_local: position %d outside the list", local_pos);
     for (int q = 0; q < npos; q++) {
         if (local_pos >= 0 && q != local_pos) continue;
-        const int dev = (q == local_pos && cuda_device >= 0) ? cuda_device : s->devices[q];
-        if (dev >= ndev) PAPER_FAIL(SPREAD_ENODEV, "somier_init: device %d not present (%d visible)", dev, ndev);
+        const int dev = cuda_devices ? cuda_devices[q]
+                                     : (q == local_pos && cuda_device >= 0) ? cuda_device : s->devices[q];
+        if (dev < 0 || dev >= ndev)
+            PAPER_FAIL(SPREAD_ENODEV, "somier_init: device %d not present (%d visible)", dev, ndev);
     }
 
     somier_s* h = new (std::nothrow) somier_s;
@@ -325,7 +328,7 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
     h->ld = (int64_t)round_up((size_t)p->n[2], 32);
     h->geom = paper::SlabGeom{p->n[0], p->n[1], p->n[2], h->ld, 0, 0};
     h->devs.resize(npos);
-    for (int q = 0; q < npos; q++) h->devs[q].device = s->devices[q];
+    for (int q = 0; q < npos; q++) h->devs[q].device = cuda_devices ? cuda_devices[q] : s->devices[q];
     if (local_pos >= 0 && cuda_device >= 0) h->devs[local_pos].device = cuda_device;
     h->chunks.resize(s->nchunks);
     for (int64_t c = 0; c < s->nchunks; c++) {
@@ -523,6 +526,11 @@ extern "C" {
 
 spread_status somier_init(spread_t s, const somier_params* p, somier_t* out) {
     return init_common(s, p, -1, -1, out);
+}
+
+spread_status somier_init_on(spread_t s, const somier_params* p, const int* cuda_devices, somier_t* out) {
+    if (!cuda_devices) return init_common(s, p, -1, -1, out);
+    return init_common(s, p, -1, -1, out, cuda_devices);
 }
 
 spread_status somier_init_local(spread_t s, const somier_params* p, int device_pos, int cuda_device,

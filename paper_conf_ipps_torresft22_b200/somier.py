@@ -101,13 +101,16 @@ class Somier:
     """
 
     def __init__(self, spread: Spread, params: SomierParams, device_pos: Optional[int] = None,
-                 cuda_device: int = -1):
+                 cuda_device: int = -1, cuda_devices: Optional[Sequence[int]] = None):
         L = N.lib()
         self.params = params
         self.spread = spread
         self._pc = params.c()
         h = ctypes.c_void_p()
-        if device_pos is None:
+        if cuda_devices is not None:
+            arr = (ctypes.c_int * len(cuda_devices))(*cuda_devices)
+            N.check(L.somier_init_on(spread.handle, ctypes.byref(self._pc), arr, ctypes.byref(h)), "somier_init_on")
+        elif device_pos is None:
             N.check(L.somier_init(spread.handle, ctypes.byref(self._pc), ctypes.byref(h)), "somier_init")
         else:
             N.check(L.somier_init_local(spread.handle, ctypes.byref(self._pc), int(device_pos), int(cuda_device),

@@ -227,6 +227,11 @@ typedef struct somier_stream_s* somier_stream_t;
  */
 spread_status somier_stream_create(spread_t s, const somier_params* p, int buffers, somier_stream_t* out);
 
+/* As somier_stream_create with list position q on CUDA device cuda_devices[q]
+ * (logical device ids, see somier_init_on); NULL = the spread's ids. */
+spread_status somier_stream_create_on(spread_t s, const somier_params* p, int buffers, const int* cuda_devices,
+                                      somier_stream_t* out);
+
 /*
  * somier_stream_generate -- write the initial state (reading S7, bit-identical
  * to somier_init's) into caller-owned host grids (layout as in somier_read),

@@ -104,6 +104,8 @@ SIGNATURES = [
     ("somier_destroy", ctypes.c_int, [_VP]),
     ("somier_version", ctypes.c_char_p, []),
     ("somier_stream_create", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.c_int, ctypes.POINTER(_VP)]),
+    ("somier_stream_create_on", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.c_int, _IP,
+                                               ctypes.POINTER(_VP)]),
     ("somier_stream_generate", ctypes.c_int, [_VP] + [_DP] * 6),
     ("somier_stream_step", ctypes.c_int, [_VP] + [_DP] * 9 + [ctypes.POINTER(somier_stats_t)]),
     ("somier_stream_traffic", ctypes.c_int, [_VP, _I64P, _I64P, _I64P]),

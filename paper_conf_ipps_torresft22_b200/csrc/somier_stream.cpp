@@ -119,6 +119,11 @@ spread_status sync_devs(somier_stream_t h) {
 extern "C" {
 
 spread_status somier_stream_create(spread_t s, const somier_params* p, int buffers, somier_stream_t* out) {
+    return somier_stream_create_on(s, p, buffers, nullptr, out);
+}
+
+spread_status somier_stream_create_on(spread_t s, const somier_params* p, int buffers, const int* cuda_devices,
+                                      somier_stream_t* out) {
     if (!out) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: out is NULL");
     *out = nullptr;
     if (!s) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_create: spread is NULL");
@@ -130,8 +135,11 @@ spread_status somier_stream_create(spread_t s, const somier_params* p, int buffe
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess) PAPER_FAIL(SPREAD_ENODEV, "somier_stream_create: no CUDA device (%s)", cudaGetErrorString(e));
-    for (int id : s->devices)
-        if (id >= ndev) PAPER_FAIL(SPREAD_ENODEV, "somier_stream_create: device %d not present (%d visible)", id, ndev);
+    for (size_t q = 0; q < s->devices.size(); q++) {
+        const int id = cuda_devices ? cuda_devices[q] : s->devices[q];
+        if (id < 0 || id >= ndev)
+            PAPER_FAIL(SPREAD_ENODEV, "somier_stream_create: device %d not present (%d visible)", id, ndev);
+    }
 
     somier_stream_s* h = new (std::nothrow) somier_stream_s;
     if (!h) PAPER_FAIL(SPREAD_ENOMEM, "somier_stream_create: out of host memory");
@@ -143,7 +151,7 @@ spread_status somier_stream_create(spread_t s, const somier_params* p, int buffe
     h->devs.resize(s->devices.size());
     for (size_t q = 0; q < s->devices.size(); q++) {
         h->devs[q].pos = (int)q;
-        h->devs[q].device = s->devices[q];
+        h->devs[q].device = cuda_devices ? cuda_devices[q] : s->devices[q];
     }
     for (int64_t c = 0; c < s->nchunks; c++) h->devs[s->chunk_info(c).pos].chunks.push_back(c);
 

@@ -232,13 +232,15 @@ class SomierStream:
     runs the fused step and maps the result back -- the paper's experiment
     (§V-A..C). buffers=1: One Buffer; >= 2: double buffering."""
 
-    def __init__(self, spread: Spread, params: SomierParams, buffers: int = 2):
+    def __init__(self, spread: Spread, params: SomierParams, buffers: int = 2,
+                 cuda_devices: Optional[Sequence[int]] = None):
         self.params = params
         self.spread = spread
         self._pc = params.c()
         h = ctypes.c_void_p()
-        N.check(N.lib().somier_stream_create(spread.handle, ctypes.byref(self._pc), int(buffers), ctypes.byref(h)),
-                "somier_stream_create")
+        arr = None if cuda_devices is None else (ctypes.c_int * len(cuda_devices))(*cuda_devices)
+        N.check(N.lib().somier_stream_create_on(spread.handle, ctypes.byref(self._pc), int(buffers), arr,
+                                                ctypes.byref(h)), "somier_stream_create")
         self._h = h
 
     def close(self) -> None:

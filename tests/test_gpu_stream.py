@@ -69,6 +69,22 @@ def test_stream_matches_resident_and_nonunit_mass(kernel):
     assert np.array_equal(X, Xr) and np.array_equal(V, Vr) and st.sums == sr.sums
 
 
+@pytest.mark.parametrize("devices,chunk,buffers", [([0, 1], 3, 2), ([2, 0, 1], 2, 1), ([0, 1, 2, 3], 5, 3)])
+def test_stream_multi_device_logical(devices, chunk, buffers):
+    """Listing 10's multi-device round robin (chunk = buffer / ndevices) with
+    every list position on its own streams (mapped onto the one GPU)."""
+    sp = P.SomierParams(n=(16, 12, 34), seed=5)
+    with P.SomierStream(P.Spread(devices, 1, 14, chunk=chunk), sp, buffers=buffers,
+                        cuda_devices=[0] * len(devices)) as s:
+        X, V = s.generate()
+        XN = np.zeros_like(X)
+        for _ in range(6):
+            st = s.step(X, V, XN)
+            X, XN = XN, X
+    ref, rst = O.run(O.init(_op(sp)), 6)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V) and st.sums == rst.sums
+
+
 def test_stream_rejects_aliasing_and_bad_buffers():
     sp = P.SomierParams(n=(8, 8, 8))
     with pytest.raises(P.SpreadError):

@@ -63,6 +63,7 @@ struct __align__(16) Smem {
 struct March2Params {
     StepArgs a;
     int tiles_k;
+    int tiles_j;
     int seg_planes;
 };
 
@@ -73,20 +74,32 @@ __device__ __forceinline__ Vec3 shfl_up1(const Vec3& v) {
 
 __device__ __forceinline__ Vec3 ld3(const double* p) { return Vec3{p[0], p[kXComp], p[2 * kXComp]}; }
 
+#ifndef K1M2_HINTS
+#define K1M2_HINTS 0  // bit 0: V loads evict-first, bit 1: output stores evict-first, bit 2: X loads evict-last
+#endif
+
+__device__ __forceinline__ void st_out(double* p, double v, uint64_t pol) {
+    if (K1M2_HINTS & 2)
+        st_hint(p, v, pol);
+    else
+        *p = v;
+}
+
 template <bool kUnitMass, bool kPosK>
 __device__ __forceinline__ void update_node(bool interior, bool valid, bool write_fixed, const Vec3& F, const double* vb,
                                             const Vec3& xc, double* vo, double* xo, int64_t cs, double* lo_dst,
-                                            double* hi_dst, int64_t off, const StepArgs& a, NodeStats& st) {
+                                            double* hi_dst, int64_t off, const StepArgs& a, NodeStats& st,
+                                            uint64_t pol) {
     if (interior) {
         Vec3 v{vb[0], vb[kVComp], vb[2 * kVComp]};
         Vec3 xn;
         kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
-        vo[0] = v.x;
-        vo[cs] = v.y;
-        vo[2 * cs] = v.z;
-        xo[0] = xn.x;
-        xo[cs] = xn.y;
-        xo[2 * cs] = xn.z;
+        st_out(vo, v.x, pol);
+        st_out(vo + cs, v.y, pol);
+        st_out(vo + 2 * cs, v.z, pol);
+        st_out(xo, xn.x, pol);
+        st_out(xo + cs, xn.y, pol);
+        st_out(xo + 2 * cs, xn.z, pol);
         if (lo_dst) {
             lo_dst[off] = xn.x;
             lo_dst[off + cs] = xn.y;
@@ -120,8 +133,27 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int lane = threadIdx.x;
     const int w = threadIdx.y;
     const int tid = w * kTK + lane;
-    const int tile_k = blockIdx.x % mp.tiles_k;
-    const int tile_j = blockIdx.x / mp.tiles_k;
+#ifndef K1M2_RASTER
+#define K1M2_RASTER 0
+#endif
+    // CTA -> tile order (L2 reuse of the halo rows / columns between tiles that
+    // run at the same time): 0 = k fastest, 1 = j fastest, G > 1 = bands of G
+    // k-tiles walked down j
+    int tile_k, tile_j;
+    if (K1M2_RASTER == 0) {
+        tile_k = blockIdx.x % mp.tiles_k;
+        tile_j = blockIdx.x / mp.tiles_k;
+    } else if (K1M2_RASTER == 1) {
+        tile_j = blockIdx.x % mp.tiles_j;
+        tile_k = blockIdx.x / mp.tiles_j;
+    } else {
+        const int G = K1M2_RASTER;
+        const int band = blockIdx.x / (G * mp.tiles_j);
+        const int gw = min(G, mp.tiles_k - band * G);
+        const int r = blockIdx.x - band * G * mp.tiles_j;
+        tile_k = band * G + r % gw;
+        tile_j = r / gw;
+    }
     const int k0 = tile_k * kTK, j0 = tile_j * kTJ;
     const int k = k0 + lane;
     const int jA = j0 + 2 * w, jB = jA + 1;
@@ -138,12 +170,18 @@ __global__ void __launch_bounds__(kThreads, 2)
     auto issue = [&](int q) {  // X of plane q
         const int s = (q - q0) % kStages;
         mbar_expect_tx(&sm.full[s], kXBoxBytes);
-        tma_load_4d(sm.xst[s], &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);
+        if (K1M2_HINTS & 4)
+            tma_load_4d_hint(sm.xst[s], &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s], policy_evict_last());
+        else
+            tma_load_4d(sm.xst[s], &tmap_x, k0 - kCol0, j0 - 1, 0, q, &sm.full[s]);
     };
     auto issue_v = [&](int p) {  // V of output plane p (V slab plane p-1)
         const int s = (p - pb) % kVStages;
         mbar_expect_tx(&sm.vfull[s], kVBoxBytes);
-        tma_load_4d(sm.vst[s], &tmap_v, k0, j0, 0, p - 1, &sm.vfull[s]);
+        if (K1M2_HINTS & 1)
+            tma_load_4d_hint(sm.vst[s], &tmap_v, k0, j0, 0, p - 1, &sm.vfull[s], policy_evict_first());
+        else
+            tma_load_4d(sm.vst[s], &tmap_v, k0, j0, 0, p - 1, &sm.vfull[s]);
     };
     if (tid == 0) {
         prefetch_tmap(&tmap_x);
@@ -185,6 +223,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     double* vo = a.v + (int64_t)(pb - 1) * ps + offA;
     int s_cur = 1, s_nxt = 2 % kStages;
     unsigned ph_nxt = (2 / kStages) & 1;
+    const uint64_t pol_st = (K1M2_HINTS & 2) ? policy_evict_first() : 0;
     NodeStats st;
     st.zero();
 #pragma unroll 1
@@ -226,14 +265,14 @@ __global__ void __launch_bounds__(kThreads, 2)
             const Vec3 F = sum_forces(neg(carryA), gpiA, gmj, gpjA, gmk, gpkA);
             update_node<kUnitMass, kPosK>(intA, validA, a.write_fixed, F, Vb + vA, xcA, vo, xo, cs,
                                           (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offA,
-                                          a, st);
+                                          a, st, pol_st);
         }
         {
             const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w + 1] : upB);
             const Vec3 F = sum_forces(neg(carryB), gpiB, neg(gpjA), gpjB, gmk, gpkB);
             update_node<kUnitMass, kPosK>(intB, validB, a.write_fixed, F, Vb + vB, xcB, vo + g.ld, xo + g.ld, cs,
                                           (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offB,
-                                          a, st);
+                                          a, st, pol_st);
         }
         carryA = gpiA;
         carryB = gpiB;
@@ -257,6 +296,7 @@ cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t str
     March2Params mp;
     mp.a = a;
     mp.tiles_k = (int)((a.g.n2 + kTK - 1) / kTK);
+    mp.tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
     const int tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
     const int tiles = mp.tiles_k * tiles_j;
     const int want_ctas = 4 * 148 * 2;

@@ -481,8 +481,16 @@ spread_status encode_slab_tmap(CUtensorMap* map, const SlabGeom& g, double* base
                                    (cuuint64_t)(3 * g.n1 * g.ld) * 8};
     const cuuint32_t box[4] = {box_k, box_j, 3, 1};
     const cuuint32_t estr[4] = {1, 1, 1, 1};
+    // L2 promotion: 256 B by default; SOMIER_TMA_PROMO=0/64/128/256 for experiments
+    CUtensorMapL2promotion promo = CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    if (const char* e = std::getenv("SOMIER_TMA_PROMO")) {
+        const int v = std::atoi(e);
+        promo = v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+                       : v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                                 : v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
+    }
     CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, base, dims, strides, box, estr,
-                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, promo,
                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled failed (%d)", (int)r);
     return SPREAD_OK;

@@ -208,6 +208,21 @@ def run_reference(a):
 
 # --------------------------------------------------------------------------- our arm
 
+def halo_info(n, chunks, world):
+    """Halo traffic of the fused exchange: each chunk boundary between list
+    positions moves one X plane (24 B per node of the n1 x n2 cross-section)
+    each way per step, stored by K1 straight into the neighbour's halo slot
+    (NVLink P2P / IPC). Reported against the measured 770 GB/s peer rate
+    (B200_PROFILING.md); the stores overlap the step, so this is a bound on
+    the exchange's cost, not a separate phase."""
+    plane = 24 * n[1] * n[2]
+    cross = sum(1 for a, b in zip(chunks, chunks[1:]) if a.device_pos != b.device_pos)
+    total = 2 * cross * plane
+    per_rank = total / max(1, world)
+    return {"bytes_per_step_total": total, "bytes_per_step_per_rank": per_rank,
+            "est_us_at_770_gbs": per_rank / 770e9 * 1e6, "mechanism": "in-kernel peer stores + completion flag"}
+
+
 def pcie_rates(local, nbytes=1 << 30):
     """Pinned host<->device copy rates (GB/s), one direction at a time and both
     directions concurrently -- the roofline of the host-streamed mode."""
@@ -477,6 +492,7 @@ def run_ours(a):
                          "avg_launch_ms": k1_ms, "launch_ms_distribution": step_dist,
                          "sustained_copy_gbs": copy_gbs},
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
+            "halo": halo_info(n, spread.chunks(), world),
             "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},
         }
         print(json.dumps(line), flush=True)

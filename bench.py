@@ -40,7 +40,7 @@ def parse():
     ap.add_argument("--grid", type=int, nargs="+", default=[512],
                     help="grid nodes (one value: cube); not --n, which torch.distributed.run would claim")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--kernel", choices=["auto", "direct", "march", "march2"], default="auto")
+    ap.add_argument("--kernel", choices=["auto", "direct", "march", "march2", "tb2"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--stream-chunk", type=int, default=32, help="planes per chunk in the host-streamed e2e")
@@ -355,7 +355,8 @@ def run_ours(a):
         torch.distributed.all_reduce(t)
         return int(t.item())
     n = a.n
-    kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH, "march2": P.K1_MARCH2}[a.kernel]
+    kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH, "march2": P.K1_MARCH2,
+              "tb2": P.K1_TB2}[a.kernel]
     params = P.SomierParams(n=n, seed=42, kernel=kernel)
     if multi:
         s = PD.open_local(params, chunk=a.chunk, cuda_device=local)
@@ -381,6 +382,10 @@ def run_ours(a):
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.5)
+    # K1_TB2 advances two steps per launch: time launches of 2 steps (K even)
+    per_call = 2 if (kernel == P.K1_TB2 and not multi and a.chunk == 0) else 1
+    if a.steps % per_call:
+        raise SystemExit("--kernel tb2 needs an even --steps")
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(a.steps)]
     l0 = s.launches
     barrier()
@@ -388,9 +393,9 @@ def run_ours(a):
     t_end = torch.cuda.Event(enable_timing=True)
     clocks.mark_start()
     t_start.record(stream)
-    for i in range(a.steps):
+    for i in range(0, a.steps, per_call):
         ev[i][0].record(stream)
-        s.step(1)
+        s.step(per_call)
         ev[i][1].record(stream)
     t_end.record(stream)
     s.sync()
@@ -399,7 +404,7 @@ def run_ours(a):
     clk = clocks.stop()
     launches = s.launches - l0
     ms = t_start.elapsed_time(t_end)
-    per_step = [b.elapsed_time(e) for b, e in ev]
+    per_step = [ev[i][0].elapsed_time(ev[i][1]) for i in range(0, a.steps, per_call)]  # per launch
     if multi:
         ms = float(all_max(ms))
         launches = all_sum(launches)
@@ -413,7 +418,8 @@ def run_ours(a):
     alg = algorithmic_bytes(n, c0.start, c0.size)
     peak, peak_src = load_peaks()
     achieved = alg / (k1_ms * 1e-3) / 1e9
-    kname = {P.K1_AUTO: "march2", P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct"}[kernel]
+    kname = {P.K1_AUTO: "march2", P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct",
+             P.K1_TB2: "tb2"}[kernel]
     traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()

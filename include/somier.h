@@ -52,7 +52,10 @@ typedef enum {
     SOMIER_K1_AUTO = 0,      /* the fastest available (currently SOMIER_K1_MARCH2)    */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
     SOMIER_K1_MARCH = 2,     /* plane-marching, smem-staged, 3 springs/node with reuse */
-    SOMIER_K1_MARCH2 = 3     /* as MARCH with two rows per warp (32 x 16 tiles)        */
+    SOMIER_K1_MARCH2 = 3,    /* as MARCH with two rows per warp (32 x 16 tiles)        */
+    SOMIER_K1_TB2 = 4        /* two time steps per pass over HBM (temporal blocking);
+                                only for a handle with a single local chunk (one slab,
+                                no halo exchange), else as MARCH2; V double-buffered  */
 } somier_kernel;
 
 typedef struct {

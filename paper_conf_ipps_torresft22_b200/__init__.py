@@ -7,7 +7,7 @@ include/somier.h, implemented by libsomier.so (hand-written sm_100a kernels).
 This package is the Python binding (argument marshalling only).
 """
 from . import _native
-from ._native import K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, SpreadError
+from ._native import K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2, SpreadError
 from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
 from .spread import Chunk, Spread
 

@@ -19,7 +19,7 @@ OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -
 # spread_map_type
 MAP_ALLOC, MAP_TO, MAP_FROM, MAP_TOFROM = 0, 1, 2, 3
 # somier_kernel
-K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2 = 0, 1, 2, 3
+K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2 = 0, 1, 2, 3, 4
 
 
 class SpreadError(RuntimeError):

@@ -65,6 +65,10 @@ struct InitArgs {
 enum class K1Variant { Direct = 1, March = 2, March2 = 3 };
 
 cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cudaStream_t stream);
+// K1_TB2: two steps in one launch (a.x_cur / a.v / tmaps with the TB2 box
+// shapes -> x_out / v_out; stats of the first step into acc1, second into a.acc)
+cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, StatsAccum* acc1, bool unit_mass,
+                          cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
 // Stats of planes [p0, p0+np) of an X slab (plane index inside the slab) and,
 // if v != null, of V planes [p0-1, ...) (V has no halo planes).

@@ -49,21 +49,25 @@ struct Chunk {
     int64_t index = 0, start = 0, size = 0;
     int pos = 0, device = 0;
     bool local = false;
-    // local allocation: [x0 | x1 | v | acc[3] | flags[2] | counter]
+    // local allocation: [x0 | x1 | v0 | (v1, K1_TB2 only) | acc[4] | flags[2] | counter]
+    // acc: [0], [1] stats of the last steps by step parity, [2] the fixed end
+    // planes, [3] scratch (K1_TB2's first step)
     void* base = nullptr;
     size_t bytes = 0;
-    size_t off_x[2] = {0, 0}, off_v = 0, off_acc = 0, off_flags = 0, off_counter = 0;
+    size_t off_x[2] = {0, 0}, off_v = 0, off_v1 = 0, off_acc = 0, off_flags = 0, off_counter = 0;
     // remote view (IPC-opened), for non-local neighbours
     void* remote_base = nullptr;
-    // TMA descriptors of the local slabs (K1_MARCH): X buffers 0/1 and V
+    // TMA descriptors of the local slabs, by X / V buffer: K1_MARCH, K1_MARCH2, K1_TB2 box shapes
     alignas(64) CUtensorMap tmap_x[2];
-    alignas(64) CUtensorMap tmap_v;
-    alignas(64) CUtensorMap tmap_x2[2];  // K1_MARCH2 box shapes
-    alignas(64) CUtensorMap tmap_v2;
+    alignas(64) CUtensorMap tmap_v[2];
+    alignas(64) CUtensorMap tmap_x2[2];
+    alignas(64) CUtensorMap tmap_v2[2];
+    alignas(64) CUtensorMap tmap_xt[2];
+    alignas(64) CUtensorMap tmap_vt[2];
 
     void* mem() const { return local ? base : remote_base; }
     double* x(int parity) const { return (double*)((char*)mem() + off_x[parity]); }
-    double* v() const { return (double*)((char*)mem() + off_v); }
+    double* v(int b = 0) const { return (double*)((char*)mem() + (b ? off_v1 : off_v)); }
     paper::StatsAccum* acc() const { return (paper::StatsAccum*)((char*)mem() + off_acc); }
     unsigned long long* flags() const { return (unsigned long long*)((char*)mem() + off_flags); }
     unsigned int* counter() const { return (unsigned int*)((char*)mem() + off_counter); }
@@ -96,6 +100,9 @@ struct somier_s {
     int64_t ld = 0;
     int64_t step = 0;
     int64_t launches = 0;
+    int xbuf = 0;      // X buffer holding X_t (flips once per launch)
+    int vbuf = 0;      // V buffer holding V_t (flips once per K1_TB2 launch; 1-step kernels update in place)
+    bool tb2 = false;  // K1_TB2 mode (single local chunk)
     bool multi_process = false;
     int local_pos = -1;
     std::vector<Chunk> chunks;
@@ -152,7 +159,7 @@ spread_status check_params(const somier_params* p) {
         if (!std::isfinite(v)) PAPER_FAIL(SPREAD_EINVAL, "somier: non-finite parameter");
     if (!(p->mass > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: mass must be > 0");
     if (!(p->dt > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: dt must be > 0");
-    if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_MARCH2)
+    if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_TB2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown kernel %d", p->kernel);
     if (p->reserved != 0) PAPER_FAIL(SPREAD_EINVAL, "somier: reserved field must be 0");
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
@@ -234,10 +241,10 @@ void free_all(somier_t h) {
 spread_status reset_stats(somier_t h, Chunk& c) {
     cudaStream_t s = h->stream_of(c);
     paper::SlabGeom g = h->geom_of(c);
-    CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 3 * sizeof(paper::StatsAccum), s));
-    const int cur = (int)(h->step & 1);
+    CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 4 * sizeof(paper::StatsAccum), s));
+    const int cur = h->xbuf;
     paper::StatsAccum* last = c.acc() + ((h->step - 1) & 1);
-    CUDA_TRY(h, paper::launch_stats(c.x(cur), c.v(), g, 1, c.size, last, s));
+    CUDA_TRY(h, paper::launch_stats(c.x(cur), c.v(h->vbuf), g, 1, c.size, last, s));
     if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, 0, 1, c.acc() + 2, s));
     if (c.start + c.size == h->p.n[0] - 1)
         CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
@@ -252,8 +259,9 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     c.off_x[0] = 0;
     c.off_x[1] = xb;
     c.off_v = 2 * xb;
-    c.off_acc = c.off_v + vb;
-    c.off_flags = c.off_acc + 3 * sizeof(paper::StatsAccum);
+    c.off_v1 = h->tb2 ? c.off_v + vb : c.off_v;
+    c.off_acc = c.off_v + (h->tb2 ? 2 : 1) * vb;
+    c.off_flags = c.off_acc + 4 * sizeof(paper::StatsAccum);
     c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);
     c.bytes = round_up(c.off_counter + 64, 4096);
     CUDA_TRY(h, cudaSetDevice(c.device));
@@ -269,17 +277,22 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     ia.seed = h->p.seed;
     CUDA_TRY(h, paper::launch_init(ia, s));
     for (int b = 0; b < 2; b++) {
-        spread_status st = encode_slab_map(h, &c.tmap_x[b], c.x(b), c.size + 2, 36, 10);
-        if (st != SPREAD_OK) return st;
+        const struct {
+            CUtensorMap* map;
+            double* base;
+            int64_t planes;
+            uint32_t bk, bj;
+        } maps[6] = {{&c.tmap_x[b], c.x(b), c.size + 2, paper::kXBoxK, paper::kXBoxJ},
+                     {&c.tmap_v[b], c.v(b), c.size, paper::kVBoxK, paper::kVBoxJ},
+                     {&c.tmap_x2[b], c.x(b), c.size + 2, paper::kXBoxK, paper::kX2BoxJ},
+                     {&c.tmap_v2[b], c.v(b), c.size, paper::kVBoxK, paper::kV2BoxJ},
+                     {&c.tmap_xt[b], c.x(b), c.size + 2, paper::kTB2XBoxK, paper::kTB2XBoxJ},
+                     {&c.tmap_vt[b], c.v(b), c.size, paper::kTB2VBoxK, paper::kTB2VBoxJ}};
+        for (const auto& m : maps) {
+            spread_status st = paper::encode_slab_tmap(m.map, g, m.base, m.planes, m.bk, m.bj);
+            if (st != SPREAD_OK) return st;
+        }
     }
-    spread_status st = encode_slab_map(h, &c.tmap_v, c.v(), c.size, 32, 8);
-    if (st != SPREAD_OK) return st;
-    for (int b = 0; b < 2; b++) {
-        st = paper::encode_slab_tmap(&c.tmap_x2[b], g, c.x(b), c.size + 2, paper::kXBoxK, paper::kX2BoxJ);
-        if (st != SPREAD_OK) return st;
-    }
-    st = paper::encode_slab_tmap(&c.tmap_v2, g, c.v(), c.size, paper::kVBoxK, paper::kV2BoxJ);
-    if (st != SPREAD_OK) return st;
     return reset_stats(h, c);
 }
 
@@ -341,6 +354,8 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         ch.device = h->devs[ci.pos].device;
         ch.local = (local_pos < 0) || (ci.pos == local_pos);
     }
+    // K1_TB2 (two steps per launch) needs one local chunk without neighbours
+    h->tb2 = p->kernel == SOMIER_K1_TB2 && local_pos < 0 && s->nchunks == 1;
     st = load_driver_entry(h);
     if (st != SPREAD_OK) {
         delete h;
@@ -418,7 +433,7 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
             if (c.pos != pos) one = false;
         }
         const char* ng = std::getenv("SOMIER_NO_GRAPH");
-        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1');
+        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1') && !h->tb2;
         h->graph_pos = pos;
     }
     *out = h;
@@ -528,6 +543,7 @@ extern "C" {
 
 namespace {
 spread_status enqueue_steps(somier_t h, int64_t nsteps);
+spread_status enqueue_tb2(somier_t h);
 }
 
 extern "C" {
@@ -643,6 +659,20 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_step: nsteps < 0");
     if (!h->connected) PAPER_FAIL(SPREAD_ESTATE, "somier_step: remote neighbour chunks not connected (somier_ipc_connect)");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    if (h->tb2) {
+        // K1_TB2: pairs of steps from an even step count; a leftover single step
+        // (or an odd start) runs the one-step K1
+        if ((h->step & 1) && nsteps > 0) {
+            spread_status st = enqueue_steps(h, 1);
+            if (st != SPREAD_OK) return st;
+            nsteps--;
+        }
+        for (; nsteps >= 2; nsteps -= 2) {
+            spread_status st = enqueue_tb2(h);
+            if (st != SPREAD_OK) return st;
+        }
+        return enqueue_steps(h, nsteps);
+    }
     // All chunks on one stream (no cross-stream flags): the launches of two
     // consecutive steps depend only on the buffer parity, so a CUDA graph of an
     // (even, odd) step pair is captured once and replayed.
@@ -691,7 +721,8 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
     int cur_dev = -1;
     for (int64_t s = 0; s < nsteps; s++) {
         const int64_t t = h->step;
-        const int cur = (int)(t & 1), nxt = cur ^ 1;
+        const int cur = h->xbuf, nxt = cur ^ 1;       // X buffers
+        const int slot = (int)(t & 1), vb = h->vbuf;  // stats slot of step t; V buffer
         for (int64_t c = 0; c < nch; c++) {
             Chunk& me = h->chunks[c];
             if (!me.local) continue;
@@ -721,7 +752,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             std::memset(&a, 0, sizeof a);
             a.x_cur = me.x(cur);
             a.x_nxt = me.x(nxt);
-            a.v = me.v();
+            a.v = me.v(vb);
             a.lo_dst = left ? left->x(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
             a.hi_dst = right ? right->x(nxt) : nullptr;
             a.g = h->geom_of(me);
@@ -729,21 +760,55 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.L = h->p.rest_len;
             a.M = h->p.mass;
             a.dt = h->p.dt;
-            a.acc = me.acc() + cur;
-            a.acc_clear = me.acc() + nxt;
+            a.acc = me.acc() + slot;
+            a.acc_clear = me.acc() + (slot ^ 1);
             a.signal_lo = fl ? &left->flags()[1] : nullptr;
             a.signal_hi = fr ? &right->flags()[0] : nullptr;
             a.signal_value = (unsigned long long)(t + 1);
             a.done_counter = me.counter();
             a.tmap_x_cur = &me.tmap_x[cur];
-            a.tmap_v = &me.tmap_v;
+            a.tmap_v = &me.tmap_v[vb];
             a.tmap_x2_cur = &me.tmap_x2[cur];
-            a.tmap_v2 = &me.tmap_v2;
+            a.tmap_v2 = &me.tmap_v2[vb];
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
             h->launches++;
         }
         h->step++;
+        h->xbuf ^= 1;
     }
+    return SPREAD_OK;
+}
+
+// K1_TB2: steps t, t+1 (t even) in one launch of the single local chunk.
+// Stats of step t go to the scratch slot 3, of step t+1 to slot 1 (the slot
+// somier_stats reads after t+2 steps); slot 0 stays zero for step t+2.
+spread_status enqueue_tb2(somier_t h) {
+    Chunk* me = nullptr;
+    for (auto& c : h->chunks)
+        if (c.local) me = &c;
+    if (!me || (h->step & 1)) PAPER_FAIL(SPREAD_ESTATE, "somier_step: K1_TB2 needs one local chunk and an even step");
+    CUDA_TRY(h, cudaSetDevice(me->device));
+    cudaStream_t st = h->stream_of(*me);
+    CUDA_TRY(h, cudaMemsetAsync(me->acc() + 1, 0, sizeof(paper::StatsAccum), st));
+    CUDA_TRY(h, cudaMemsetAsync(me->acc() + 3, 0, sizeof(paper::StatsAccum), st));
+    const int cur = h->xbuf, vb = h->vbuf;
+    paper::StepArgs a;
+    std::memset(&a, 0, sizeof a);
+    a.x_cur = me->x(cur);
+    a.v = me->v(vb);
+    a.g = h->geom_of(*me);
+    a.K = h->p.k_spring;
+    a.L = h->p.rest_len;
+    a.M = h->p.mass;
+    a.dt = h->p.dt;
+    a.acc = me->acc() + 1;
+    a.tmap_x_cur = &me->tmap_xt[cur];
+    a.tmap_v = &me->tmap_vt[vb];
+    CUDA_TRY(h, paper::launch_k1_tb2(a, me->x(cur ^ 1), me->v(vb ^ 1), me->acc() + 3, h->unit_mass(), st));
+    h->launches++;
+    h->step += 2;
+    h->xbuf ^= 1;
+    h->vbuf ^= 1;
     return SPREAD_OK;
 }
 
@@ -808,7 +873,7 @@ spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* 
     if (st != SPREAD_OK) return st;
     double* X[3] = {x, y, z};
     double* V[3] = {vx, vy, vz};
-    const int cur = (int)(h->step & 1);
+    const int cur = h->xbuf;
     const size_t plane = (size_t)(h->p.n[1] * h->p.n[2]);
     const int64_t i1 = i0 + count;
     // host grids hold planes [i0, i1): global plane i -> host plane i - i0
@@ -834,7 +899,7 @@ spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* 
                     if (sp.fixed)  // fixed end planes have zero velocity
                         std::memset(V[d] + (size_t)(lo - i0) * plane, 0, (size_t)(hi - lo) * plane * sizeof(double));
                     else
-                        CUDA_TRY(h, copy_planes(h, c.v(), d, lo - c.start, V[d], lo - i0, hi - lo,
+                        CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, lo - c.start, V[d], lo - i0, hi - lo,
                                                 cudaMemcpyDeviceToHost, s));
                 }
             }
@@ -855,7 +920,7 @@ spread_status somier_load(somier_t h, const double* x, const double* y, const do
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     const double* X[3] = {x, y, z};
     const double* V[3] = {vx, vy, vz};
-    const int cur = (int)(h->step & 1);
+    const int cur = h->xbuf;
     for (auto& c : h->chunks) {
         if (!c.local) continue;
         CUDA_TRY(h, cudaSetDevice(c.device));
@@ -863,7 +928,7 @@ spread_status somier_load(somier_t h, const double* x, const double* y, const do
         for (int d = 0; d < 3; d++) {
             CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, const_cast<double*>(X[d]), c.start - 1, c.size + 2,
                                     cudaMemcpyHostToDevice, s));
-            CUDA_TRY(h, copy_planes(h, c.v(), d, 0, const_cast<double*>(V[d]), c.start, c.size,
+            CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, 0, const_cast<double*>(V[d]), c.start, c.size,
                                     cudaMemcpyHostToDevice, s));
         }
         // the X_{t+1} buffer must hold the same fixed nodes (never written by a step)

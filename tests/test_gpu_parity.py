@@ -59,7 +59,7 @@ def _assert_parity(X, V, st, ref, rst, bitwise=True):
         assert st.centre == rst.centre and st.vmax == rst.vmax
 
 
-@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2])
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2, P.K1_TB2])
 @pytest.mark.parametrize("n", [(16, 16, 16), (17, 9, 33), (3, 3, 3), (5, 40, 70)])
 def test_initial_state_bitwise(n, kernel):
     sp = _params(n, seed=2, kernel=kernel)
@@ -70,7 +70,7 @@ def test_initial_state_bitwise(n, kernel):
     assert st.sums == rst.sums and st.centre == rst.centre and st.vmax2_bits == rst.vmax2_bits
 
 
-@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2])
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2, P.K1_TB2])
 @pytest.mark.parametrize("seed", [1, 2, 3])
 def test_16cube_10_steps(seed, kernel):
     """configs[0]: Somier 16^3, fp64, 10 steps."""
@@ -80,7 +80,7 @@ def test_16cube_10_steps(seed, kernel):
     _assert_parity(X, V, st, ref, rst)
 
 
-@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2])
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2, P.K1_TB2])
 @pytest.mark.parametrize("n", [(17, 9, 33), (9, 33, 17), (33, 17, 9), (6, 131, 70), (4, 5, 260)])
 def test_ragged_shapes_30_steps(n, kernel):
     """Shapes spanning several tiles with ragged tails in every dimension."""
@@ -90,7 +90,7 @@ def test_ragged_shapes_30_steps(n, kernel):
     _assert_parity(X, V, st, ref, rst)
 
 
-@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2])
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2, P.K1_TB2])
 def test_128cube_100_steps(kernel):
     """configs[1]: Somier 128^3, 100 steps, 1 GPU vs the CPU oracle."""
     sp = _params((128, 128, 128), seed=1, kernel=kernel)
@@ -239,7 +239,7 @@ def test_launch_count_and_footprint():
         assert s.device_bytes >= (2 * 34 + 32) * 3 * 20 * 40 * 8
 
 
-@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2])
+@pytest.mark.parametrize("kernel", [P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2, P.K1_TB2])
 @pytest.mark.parametrize("K", [0.0, -2.0])
 def test_zero_and_negative_stiffness_signed_zeros(K, kernel):
     """K <= 0 makes K*(d-L) = -0 possible; -0/d must stay -0 (the K > 0 fast

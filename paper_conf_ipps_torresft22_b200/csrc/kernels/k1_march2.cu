@@ -43,6 +43,10 @@ constexpr int kXSlot = 15616;                     // 128-byte aligned
 #ifndef K1M2_VSTAGES
 #define K1M2_VSTAGES 3
 #endif
+#ifndef K1M2_UNROLL
+#define K1M2_UNROLL 1
+#endif
+constexpr int kM2Unroll = K1M2_UNROLL;  // plane-loop unroll (removes the loop-carried register moves)
 constexpr int kStages = K1M2_STAGES;
 constexpr int kVStages = K1M2_VSTAGES;
 constexpr int kSegPlanes = 64;
@@ -226,7 +230,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     const uint64_t pol_st = (K1M2_HINTS & 2) ? policy_evict_first() : 0;
     NodeStats st;
     st.zero();
-#pragma unroll 1
+#pragma unroll(kM2Unroll)
     for (int p = pb; p < pe; p++) {
         const int par = p & 1;
         mbar_wait(&sm.full[s_nxt], ph_nxt);

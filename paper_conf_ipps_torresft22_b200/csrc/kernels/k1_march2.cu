@@ -303,7 +303,10 @@ cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t str
     mp.tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
     const int tiles_j = (int)((a.g.n1 + kTJ - 1) / kTJ);
     const int tiles = mp.tiles_k * tiles_j;
-    const int want_ctas = 4 * 148 * 2;
+#ifndef K1M2_WAVES
+#define K1M2_WAVES 4
+#endif
+    const int want_ctas = K1M2_WAVES * 148 * 2;  // waves of 2 CTAs per SM
     int nseg = (int)((a.g.size + kSegPlanes - 1) / kSegPlanes);
     nseg = std::max(nseg, std::min((int)a.g.size, (want_ctas + tiles - 1) / tiles));
     mp.seg_planes = (int)((a.g.size + nseg - 1) / nseg);

@@ -159,13 +159,12 @@ class ClockSampler:
 
 # --------------------------------------------------------------------------- oracle arm
 
-def oracle_sample(n, budget_s, max_steps=None, warmup=0):
+def oracle_sample(n, budget_s, max_steps=None, warmup=0, planes=8):
     """Time the CPU oracle (as it stands) on a bounded sample of the workload: a
     (planes+2) x n1 x n2 slab -- `planes` interior planes of the full cross
     section -- stepped repeatedly. Returns (node-updates/s, sample description, steps)."""
     import oracle as O
 
-    planes = 8
     p = O.Params(n=(planes + 2, n[1], n[2]), seed=42)
     s = O.init(p)
     per_step = planes * (n[1] - 2) * (n[2] - 2)
@@ -193,12 +192,17 @@ def run_reference(a):
     if rank != 0:
         return 0
     n = a.n
-    rate, desc, steps, el = oracle_sample(n, budget_s=None, max_steps=a.steps, warmup=a.warmup)
+    # Bound the whole --steps K --warmup W run to a few minutes: one oracle
+    # node-update costs ~0.1-0.2 us on one core, so a step over P planes of the
+    # n1 x n2 cross-section costs ~2e-7 * P * n1 * n2 s; budget ~150 s total.
+    per_plane = 2e-7 * n[1] * n[2]
+    planes = int(max(1, min(8, 150.0 / (max(1, a.steps + a.warmup) * per_plane))))
+    rate, desc, steps, el = oracle_sample(n, budget_s=None, max_steps=a.steps, warmup=a.warmup, planes=planes)
     line = {
         "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": a.gpus, "steps": a.steps,
         "warmup": a.warmup, "ms_per_step": 1e3 * el / steps, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": workload_name(n), "n": list(n), "sample": "8-plane slab per step"},
+        "config": {"workload": workload_name(n), "n": list(n), "sample": "%d-plane slab per step" % planes},
         "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
         "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }

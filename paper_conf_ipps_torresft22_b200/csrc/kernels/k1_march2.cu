@@ -49,7 +49,10 @@ constexpr int kXSlot = 15616;                     // 128-byte aligned
 constexpr int kM2Unroll = K1M2_UNROLL;  // plane-loop unroll (removes the loop-carried register moves)
 constexpr int kStages = K1M2_STAGES;
 constexpr int kVStages = K1M2_VSTAGES;
-constexpr int kSegPlanes = 64;
+#ifndef K1M2_SEG
+#define K1M2_SEG 64
+#endif
+constexpr int kSegPlanes = K1M2_SEG;    // planes per CTA segment along i
 constexpr int kMinSegPlanes = 4;
 constexpr int kXComp = kBJ * kBK, kVComp = kTJ * kTK;
 

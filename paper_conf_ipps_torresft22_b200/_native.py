@@ -69,6 +69,10 @@ _DP = ctypes.POINTER(ctypes.c_double)
 SIGNATURES = [
     ("spread_create", ctypes.c_int, [_IP, ctypes.c_int, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.c_int64,
                                      ctypes.POINTER(_VP)]),
+    ("spread_create_sizes", ctypes.c_int, [_IP, ctypes.c_int, ctypes.c_int64, ctypes.c_int64, _I64P, ctypes.c_int64,
+                                           ctypes.POINTER(_VP)]),
+    ("spread_create_weighted", ctypes.c_int, [_IP, ctypes.c_int, ctypes.c_int64, ctypes.c_int64, _DP,
+                                              ctypes.POINTER(_VP)]),
     ("spread_destroy", ctypes.c_int, [_VP]),
     ("spread_num_chunks", ctypes.c_int, [_VP, _I64P]),
     ("spread_num_devices", ctypes.c_int, [_VP, _IP]),

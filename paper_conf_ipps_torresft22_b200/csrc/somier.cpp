@@ -27,7 +27,7 @@ using paper::set_last_error;
 namespace {
 
 constexpr uint64_t kIpcMagic = 0x534f4d4945524950ull;  // "SOMIERIP"
-constexpr uint32_t kIpcVersion = 1;
+constexpr uint32_t kIpcVersion = 2;
 
 using PFN_waitValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 using PFN_encodeTiled = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -86,8 +86,26 @@ struct IpcHeader {
     int64_t n[3];
     int64_t nchunks;
     int64_t chunk;
+    uint64_t layout;  // FNV-1a of every chunk's (device_pos, start, size): catches unequal irregular tables
     int64_t nrecords;
 };
+
+uint64_t spread_layout_hash(const spread_s& s) {
+    uint64_t h = 1469598103934665603ull;
+    auto mix = [&](int64_t v) {
+        for (int b = 0; b < 8; b++) {
+            h ^= (uint64_t)((v >> (8 * b)) & 0xff);
+            h *= 1099511628211ull;
+        }
+    };
+    for (int64_t c = 0; c < s.nchunks; c++) {
+        const paper::ChunkInfo ci = s.chunk_info(c);
+        mix(ci.pos);
+        mix(ci.start);
+        mix(ci.size);
+    }
+    return h;
+}
 
 size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
@@ -590,6 +608,7 @@ spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len) 
     for (int d = 0; d < 3; d++) hd.n[d] = h->p.n[d];
     hd.nchunks = (int64_t)h->chunks.size();
     hd.chunk = h->spread.chunk;
+    hd.layout = spread_layout_hash(h->spread);
     hd.nrecords = (int64_t)recs.size();
     const size_t need = sizeof hd + recs.size() * sizeof(IpcChunkRecord);
     if (len) *len = need;
@@ -612,7 +631,8 @@ spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const siz
         if (hd.magic != kIpcMagic || hd.version != kIpcVersion)
             PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d is not a somier IPC blob", b);
         if (hd.n[0] != h->p.n[0] || hd.n[1] != h->p.n[1] || hd.n[2] != h->p.n[2] ||
-            hd.nchunks != (int64_t)h->chunks.size() || hd.chunk != h->spread.chunk)
+            hd.nchunks != (int64_t)h->chunks.size() || hd.chunk != h->spread.chunk ||
+            hd.layout != spread_layout_hash(h->spread))
             PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d describes another grid or spread", b);
         if (lens[b] != sizeof hd + (size_t)hd.nrecords * sizeof(IpcChunkRecord))
             PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d has a bad length", b);

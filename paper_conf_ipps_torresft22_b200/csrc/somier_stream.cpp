@@ -147,7 +147,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
     h->spread = *s;
     h->buffers = buffers;
     h->geom = paper::SlabGeom{p->n[0], p->n[1], p->n[2], paper::slab_ld(p->n[2]), 0, 0};
-    h->max_chunk = std::min<int64_t>(s->chunk, s->range_len);
+    h->max_chunk = s->max_chunk();
     h->devs.resize(s->devices.size());
     for (size_t q = 0; q < s->devices.size(); q++) {
         h->devs[q].pos = (int)q;

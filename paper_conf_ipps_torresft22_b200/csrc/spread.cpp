@@ -1,6 +1,7 @@
 // spread.cpp -- the "target spread" descriptor: device list + iteration range +
 // static round-robin schedule, and halo map extents (include/spread.h).
 // Host-only logic; PAPER.md:95-116 (§III-B.1), 144-173 (Listing 5).
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -62,6 +63,83 @@ spread_status spread_create(const int* devices, int ndevices, int64_t range_star
     return SPREAD_OK;
 }
 
+spread_status spread_create_sizes(const int* devices, int ndevices, int64_t range_start, int64_t range_len,
+                                  const int64_t* sizes, int64_t nsizes, spread_t* out) {
+    if (!out) PAPER_FAIL(SPREAD_EINVAL, "spread_create_sizes: out is NULL");
+    *out = nullptr;
+    if (nsizes < 0 || (nsizes > 0 && !sizes)) PAPER_FAIL(SPREAD_EINVAL, "spread_create_sizes: bad sizes array");
+    int64_t total = 0, largest = 1;
+    for (int64_t c = 0; c < nsizes; c++) {
+        if (sizes[c] < 1)
+            PAPER_FAIL(SPREAD_EINVAL, "spread_create_sizes: chunk %lld has size %lld < 1", (long long)c,
+                       (long long)sizes[c]);
+        if (sizes[c] > range_len - total)
+            PAPER_FAIL(SPREAD_EINVAL, "spread_create_sizes: chunk sizes exceed the range length %lld",
+                       (long long)range_len);
+        total += sizes[c];
+        largest = std::max<int64_t>(largest, sizes[c]);
+    }
+    if (total != range_len)
+        PAPER_FAIL(SPREAD_EINVAL, "spread_create_sizes: chunk sizes sum to %lld, range length is %lld",
+                   (long long)total, (long long)range_len);
+    spread_t s = nullptr;
+    spread_status st = spread_create(devices, ndevices, range_start, range_len, SPREAD_SCHED_STATIC, 0, &s);
+    if (st != SPREAD_OK) return st;
+    try {
+        s->offsets.resize((size_t)nsizes + 1);
+    } catch (...) {
+        delete s;
+        PAPER_FAIL(SPREAD_ENOMEM, "spread_create_sizes: out of host memory");
+    }
+    s->offsets[0] = 0;
+    for (int64_t c = 0; c < nsizes; c++) s->offsets[c + 1] = s->offsets[c] + sizes[c];
+    s->nchunks = nsizes;
+    s->chunk = largest;
+    *out = s;
+    return SPREAD_OK;
+}
+
+spread_status spread_create_weighted(const int* devices, int ndevices, int64_t range_start, int64_t range_len,
+                                     const double* weights, spread_t* out) {
+    if (!out) PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: out is NULL");
+    *out = nullptr;
+    if (!devices || ndevices < 1) PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: empty devices() list");
+    if (!weights) PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: weights is NULL");
+    if (range_len < ndevices)
+        PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: range length %lld < %d devices", (long long)range_len,
+                   ndevices);
+    double wsum = 0.0;
+    for (int d = 0; d < ndevices; d++) {
+        if (!(weights[d] > 0.0) || !std::isfinite(weights[d]))
+            PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: weight %d is not a positive finite number", d);
+        wsum += weights[d];
+    }
+    if (!std::isfinite(wsum)) PAPER_FAIL(SPREAD_EINVAL, "spread_create_weighted: weights overflow");
+    // One chunk per list position: 1 iteration each, the remaining len - p
+    // shared by largest remainder of w_d / sum(w) (ties to the earlier position).
+    std::vector<int64_t> sizes((size_t)ndevices, 1);
+    std::vector<double> rem((size_t)ndevices);
+    const int64_t spare = range_len - ndevices;
+    int64_t given = 0;
+    for (int d = 0; d < ndevices; d++) {
+        const double share = (double)spare * (weights[d] / wsum);
+        int64_t f = (int64_t)std::floor(share);
+        f = std::min<int64_t>(f, spare - given);
+        sizes[d] += f;
+        given += f;
+        rem[d] = share - (double)f;
+    }
+    while (given < spare) {
+        int best = 0;
+        for (int d = 1; d < ndevices; d++)
+            if (rem[d] > rem[best]) best = d;
+        sizes[best] += 1;
+        rem[best] = -1.0;
+        given += 1;
+    }
+    return spread_create_sizes(devices, ndevices, range_start, range_len, sizes.data(), ndevices, out);
+}
+
 spread_status spread_destroy(spread_t s) {
     delete s;
     return SPREAD_OK;
@@ -118,7 +196,7 @@ spread_status spread_chunk_of(spread_t s, int64_t iter, int64_t* chunk_index) {
     if (!s) PAPER_FAIL(SPREAD_EINVAL, "spread_chunk_of: NULL handle");
     if (iter < s->range_start || iter >= s->range_start + s->range_len)
         PAPER_FAIL(SPREAD_EINVAL, "spread_chunk_of: iteration %lld outside the range", (long long)iter);
-    if (chunk_index) *chunk_index = (iter - s->range_start) / s->chunk;
+    if (chunk_index) *chunk_index = s->chunk_of(iter);
     return SPREAD_OK;
 }
 

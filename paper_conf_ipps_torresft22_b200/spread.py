@@ -19,16 +19,39 @@ class Spread:
     """devices(...) + range(start:len) + spread_schedule(static, chunk).
 
     chunk == 0 means ceil(len / ndevices): one contiguous slab per device.
+    Irregular static schedules: Spread.with_sizes / Spread.weighted.
     """
 
-    def __init__(self, devices: Sequence[int], range_start: int, range_len: int, chunk: int = 0, sched: int = 0):
+    def __init__(self, devices: Sequence[int], range_start: int, range_len: int, chunk: int = 0, sched: int = 0,
+                 *, sizes: Sequence[int] | None = None, weights: Sequence[float] | None = None):
         L = N.lib()
         arr = (ctypes.c_int * len(devices))(*devices)
         h = ctypes.c_void_p()
-        N.check(L.spread_create(arr, len(devices), range_start, range_len, sched, chunk, ctypes.byref(h)),
-                "spread_create")
+        if sizes is not None:
+            sz = (ctypes.c_int64 * max(1, len(sizes)))(*sizes)
+            N.check(L.spread_create_sizes(arr, len(devices), range_start, range_len, sz, len(sizes),
+                                          ctypes.byref(h)), "spread_create_sizes")
+        elif weights is not None:
+            if len(weights) != len(devices):
+                raise ValueError("one weight per device")
+            w = (ctypes.c_double * len(weights))(*weights)
+            N.check(L.spread_create_weighted(arr, len(devices), range_start, range_len, w, ctypes.byref(h)),
+                    "spread_create_weighted")
+        else:
+            N.check(L.spread_create(arr, len(devices), range_start, range_len, sched, chunk, ctypes.byref(h)),
+                    "spread_create")
         self._h = h
         self.devices = list(devices)
+
+    @classmethod
+    def with_sizes(cls, devices: Sequence[int], range_start: int, range_len: int, sizes: Sequence[int]) -> "Spread":
+        """spread_create_sizes: chunk c = the next sizes[c] iterations, on list position c mod p."""
+        return cls(devices, range_start, range_len, sizes=sizes)
+
+    @classmethod
+    def weighted(cls, devices: Sequence[int], range_start: int, range_len: int, weights: Sequence[float]) -> "Spread":
+        """spread_create_weighted: one chunk per device, sized by largest remainder of the weights."""
+        return cls(devices, range_start, range_len, weights=weights)
 
     @property
     def handle(self) -> ctypes.c_void_p:

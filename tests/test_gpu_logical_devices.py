@@ -49,3 +49,31 @@ def test_logical_devices_load_and_continue():
         X2, V2 = s.read()
     ref, _ = O.run(O.init(O.Params(n=n, seed=2)), 10)
     assert np.array_equal(X2, ref.X) and np.array_equal(V2, ref.V)
+
+
+@pytest.mark.parametrize("devices,sizes", [([0, 1], [3, 17]), ([0, 1, 2], [1, 8, 2, 5, 1, 3]), ([2, 0], [19, 1]),
+                                           ([0], [4, 4, 12])])
+@pytest.mark.parametrize("kernel", [P.K1_MARCH2, P.K1_DIRECT])
+def test_irregular_spread_bit_identical(devices, sizes, kernel):
+    """Irregular static schedule (spread_create_sizes): any chunk
+    table gives the oracle's result bit for bit."""
+    n, steps = (22, 19, 45), 13
+    sp = P.SomierParams(n=n, seed=5, kernel=kernel)
+    spread = P.Spread.with_sizes(devices, 1, n[0] - 2, sizes)
+    with P.Somier(spread, sp, cuda_devices=[0] * len(devices)) as s:
+        s.step(steps)
+        st = s.stats()
+        X, V = s.read()
+    ref, rst = O.run(O.init(O.Params(n=n, seed=5)), steps)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+    assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits
+
+
+def test_weighted_spread_bit_identical():
+    n = (40, 16, 33)
+    sp = P.SomierParams(n=n, seed=8)
+    with P.Somier(P.Spread.weighted([0, 1, 2], 1, n[0] - 2, [1.0, 3.0, 0.5]), sp, cuda_devices=[0, 0, 0]) as s:
+        s.step(9)
+        X, V = s.read()
+    ref, _ = O.run(O.init(O.Params(n=n, seed=8)), 9)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)

@@ -33,3 +33,10 @@ def test_stencil3_subrange_leaves_rest_untouched():
     ref = O.stencil3(A)
     assert np.array_equal(B[10:30], ref[10:30])
     assert (B[:10] == -7).all() and (B[30:] == -7).all()
+
+
+@pytest.mark.parametrize("sizes", [[1, 5, 2, 4], [12], [3, 3, 1, 1, 1, 1, 1, 1]])
+def test_stencil3_irregular_chunks(sizes):
+    A = np.random.default_rng(len(sizes)).normal(size=14)
+    B = P.Spread.with_sizes([0], 1, 12, sizes).stencil3(A)
+    assert np.array_equal(B, O.stencil3(A))

@@ -93,3 +93,17 @@ def test_stream_rejects_aliasing_and_bad_buffers():
         X, V = s.generate()
         with pytest.raises(P.SpreadError):
             s.step(X, V, X)
+
+
+@pytest.mark.parametrize("sizes,buffers", [([2, 9, 1, 5], 2), ([17], 1), ([1, 1, 15], 3)])
+def test_stream_irregular_chunks(sizes, buffers):
+    sp = P.SomierParams(n=(19, 12, 35), seed=4)
+    with P.SomierStream(P.Spread.with_sizes([0], 1, 17, sizes), sp, buffers=buffers) as s:
+        X, V = s.generate()
+        XN = np.zeros_like(X)
+        for _ in range(7):
+            st = s.step(X, V, XN)
+            X, XN = XN, X
+    ref, rst = O.run(O.init(_op(sp)), 7)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+    assert st.sums == rst.sums

@@ -254,8 +254,30 @@ spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, do
 spread_status somier_stream_step(somier_stream_t h, const double* x, const double* y, const double* z, double* vx,
                                  double* vy, double* vz, double* xn, double* yn, double* zn, somier_stats_t* stats);
 
-/* Bytes moved host->device and device->host by one somier_stream_step, and
- * K1 launches so far. */
+/*
+ * somier_stream_run -- nsteps time steps on host-resident state with
+ * chunk-level dependencies instead of a barrier per step: the paper's future
+ * work `depend(out/in: B[omp_spread_start:omp_spread_size])` on the spread
+ * data directives, "making the enclosing taskgroup directive no longer
+ * necessary" (Listing 13). The H2D of chunk c for step t+1
+ * waits only for the D2H of chunks c-1, c, c+1 of step t, and the D2H of
+ * chunk c (which overwrites X_{t-1}[c]) only for the H2D of chunks c-1, c+1 of
+ * step t-1; no device idles at a step boundary. One host barrier at the end.
+ *   (x, y, z) / (xn, yn, zn): the two X buffers, used alternately: step t
+ *   reads the first if t is even, the second if t is odd, and writes the other
+ *   one; after the call X_{nsteps} is in (x, y, z) if nsteps is even, else in
+ *   (xn, yn, zn). V is updated in place. The buffers must not overlap.
+ *   stats: NULL, or an array of nsteps entries receiving the statistics after
+ *   each step.
+ * Results are bit-identical to nsteps calls of somier_stream_step.
+ * Errors: EINVAL (NULL, nsteps < 0, aliasing X buffers), ENOMEM, ECUDA.
+ */
+spread_status somier_stream_run(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                double* vz, double* xn, double* yn, double* zn, int64_t nsteps,
+                                somier_stats_t* stats);
+
+/* Bytes moved host->device and device->host by one somier_stream_step (one
+ * step of somier_stream_run), and K1 launches so far. */
 spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches);
 
 spread_status somier_stream_destroy(somier_stream_t h);

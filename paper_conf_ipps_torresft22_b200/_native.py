@@ -112,6 +112,7 @@ SIGNATURES = [
                                                ctypes.POINTER(_VP)]),
     ("somier_stream_generate", ctypes.c_int, [_VP] + [_DP] * 6),
     ("somier_stream_step", ctypes.c_int, [_VP] + [_DP] * 9 + [ctypes.POINTER(somier_stats_t)]),
+    ("somier_stream_run", ctypes.c_int, [_VP] + [_DP] * 9 + [ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
     ("somier_stream_traffic", ctypes.c_int, [_VP, _I64P, _I64P, _I64P]),
     ("somier_stream_destroy", ctypes.c_int, [_VP]),
 ]

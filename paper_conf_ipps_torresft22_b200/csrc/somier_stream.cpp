@@ -35,17 +35,28 @@ struct Slot {
     alignas(64) CUtensorMap tmap_v;
     alignas(64) CUtensorMap tmap_x2;
     alignas(64) CUtensorMap tmap_v2;
-    cudaEvent_t h2d_done = nullptr, comp_done = nullptr, d2h_done = nullptr;
+    cudaEvent_t comp_done = nullptr, d2h_done = nullptr;
     bool used = false;
+};
+
+// Per-chunk completion events, by step parity: the chunk-level `depend`
+// (PAPER.md:746-767). H2D(c, t+1) depends on D2H(c-1, t), D2H(c, t),
+// D2H(c+1, t) (it reads the halo planes and V they wrote); D2H(c, t+1), which
+// overwrites X_t[c], depends on H2D(c-1, t) and H2D(c+1, t) (they read its
+// edge planes as halos). No other ordering between steps is needed.
+struct ChunkEvents {
+    cudaEvent_t h2d[2] = {nullptr, nullptr};
+    cudaEvent_t d2h[2] = {nullptr, nullptr};
 };
 
 struct Dev {
     int pos = 0, device = 0;
     cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
     std::vector<Slot> slots;
-    void* acc_base = nullptr;  // StatsAccum[2]: chunk sums, fixed end planes
+    void* acc_base = nullptr;  // StatsAccum[acc_steps][2]: per step, chunk sums and fixed end planes
+    int64_t acc_steps = 0;
     std::vector<int64_t> chunks;
-    paper::StatsAccum* acc() const { return (paper::StatsAccum*)acc_base; }
+    paper::StatsAccum* acc(int64_t t) const { return (paper::StatsAccum*)acc_base + 2 * t; }
 };
 
 }  // namespace
@@ -59,6 +70,7 @@ struct somier_stream_s {
     int64_t step = 0;
     int64_t launches = 0;
     std::vector<Dev> devs;
+    std::vector<ChunkEvents> ev;   // per chunk, created on the chunk's device
     std::string sticky;
 };
 
@@ -79,13 +91,15 @@ spread_status sfail(somier_stream_t h, cudaError_t e, const char* what) {
 
 size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
+constexpr int64_t kAccSteps = 64;  // initial per-step stats history (grown on demand)
+
 void destroy_all(somier_stream_t h) {
     for (auto& d : h->devs) {
         cudaSetDevice(d.device);
         for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
             if (s) cudaStreamSynchronize(s);
         for (auto& sl : d.slots) {
-            for (cudaEvent_t e : {sl.h2d_done, sl.comp_done, sl.d2h_done})
+            for (cudaEvent_t e : {sl.comp_done, sl.d2h_done})
                 if (e) cudaEventDestroy(e);
             if (sl.base) cudaFree(sl.base);
         }
@@ -93,6 +107,12 @@ void destroy_all(somier_stream_t h) {
         for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
             if (s) cudaStreamDestroy(s);
     }
+    for (auto& ce : h->ev)
+        for (int q = 0; q < 2; q++) {
+            if (ce.h2d[q]) cudaEventDestroy(ce.h2d[q]);
+            if (ce.d2h[q]) cudaEventDestroy(ce.d2h[q]);
+        }
+    h->ev.clear();
     h->devs.clear();
 }
 
@@ -111,6 +131,144 @@ spread_status sync_devs(somier_stream_t h) {
         if (e != cudaSuccess) return sfail(h, e, "somier_stream: synchronize");
     }
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    return SPREAD_OK;
+}
+
+// Grow every device's per-step stats history to hold `nsteps` steps.
+spread_status ensure_acc(somier_stream_t h, int64_t nsteps) {
+    for (auto& d : h->devs) {
+        if (d.chunks.empty() || d.acc_steps >= nsteps) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaDeviceSynchronize());
+        S_TRY(h, cudaFree(d.acc_base));
+        d.acc_base = nullptr;
+        d.acc_steps = 0;
+        S_TRY(h, cudaMalloc(&d.acc_base, 2 * (size_t)nsteps * sizeof(paper::StatsAccum)));
+        d.acc_steps = nsteps;
+    }
+    return SPREAD_OK;
+}
+
+// Enqueue step t of a run (0-based within the run): every chunk, in chunk
+// order, reads X_t from X, writes X_{t+1} to XN and V in place. `chained`:
+// a step of the same run precedes it, so its copies wait on that step's
+// per-chunk events instead of a host barrier.
+spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
+                                  int64_t t, bool chained) {
+    const int64_t n0 = h->p.n[0];
+    const int64_t nch = h->spread.nchunks;
+    const int par = (int)(t & 1), prev = par ^ 1;
+    for (int64_t c = 0; c < nch; c++) {
+        const paper::ChunkInfo ci = h->spread.chunk_info(c);
+        Dev& d = h->devs[ci.pos];
+        const size_t m = (size_t)(c / (int64_t)h->devs.size());  // index of c among its device's chunks
+        Slot& sl = d.slots[m % d.slots.size()];
+        const paper::SlabGeom g = geom_of(h, ci);
+        const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
+        ChunkEvents& ev = h->ev[(size_t)c];
+        S_TRY(h, cudaSetDevice(d.device));
+        // map(to: X[start-1 : size+2], V[start : size])  -- depend(in: ...)
+        if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
+        if (chained)
+            for (int64_t nb = std::max<int64_t>(0, c - 1); nb <= std::min<int64_t>(nch - 1, c + 1); nb++)
+                S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
+        for (int q = 0; q < 3; q++) {
+            S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, X[q], ci.start - 1, ci.size + 2,
+                                             cudaMemcpyHostToDevice, d.s_h2d));
+            S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], ci.start, ci.size, cudaMemcpyHostToDevice,
+                                             d.s_h2d));
+        }
+        S_TRY(h, cudaEventRecord(ev.h2d[par], d.s_h2d));
+        // the fused step (forces, accelerations, velocities, positions, centers)
+        S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
+        paper::StatsAccum* acc = d.acc(t);
+        if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, acc + 1, d.s_comp));
+        if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, ci.size + 1, 1, acc + 1, d.s_comp));
+        paper::StepArgs a;
+        std::memset(&a, 0, sizeof a);
+        a.x_cur = sl.x_in;
+        a.x_nxt = sl.x_out;
+        a.v = sl.v;
+        a.g = g;
+        a.K = h->p.k_spring;
+        a.L = h->p.rest_len;
+        a.M = h->p.mass;
+        a.dt = h->p.dt;
+        a.acc = acc;
+        a.tmap_x_cur = &sl.tmap_x;
+        a.tmap_v = &sl.tmap_v;
+        a.tmap_x2_cur = &sl.tmap_x2;
+        a.tmap_v2 = &sl.tmap_v2;
+        a.write_fixed = 1;
+        const paper::K1Variant var = paper::k1_variant(h->p.kernel);
+        S_TRY(h, paper::launch_k1(var, a, h->p.mass == 1.0, d.s_comp));
+        h->launches++;
+        S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
+        // map(from: X[start : size], V[start : size]) (+ the fixed end planes);
+        // it overwrites X_{t-1}[chunk], whose edge planes the neighbours' H2D of
+        // the previous step read as halos
+        S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
+        if (chained) {
+            if (c > 0) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)c - 1].h2d[prev], 0));
+            if (c + 1 < nch) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)c + 1].h2d[prev], 0));
+        }
+        for (int q = 0; q < 3; q++) {
+            S_TRY(h, paper::copy_slab_planes(g, sl.x_out, q, 1, XN[q], ci.start, ci.size, cudaMemcpyDeviceToHost,
+                                             d.s_d2h));
+            S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], ci.start, ci.size, cudaMemcpyDeviceToHost,
+                                             d.s_d2h));
+            if (first)
+                S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, XN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
+            if (last)
+                S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, ci.size + 1, XN[q], n0 - 1, 1,
+                                                 cudaMemcpyDeviceToHost, d.s_d2h));
+        }
+        S_TRY(h, cudaEventRecord(ev.d2h[par], d.s_d2h));
+        S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
+        sl.used = true;
+    }
+    return SPREAD_OK;
+}
+
+// Run nsteps steps from (X, V), alternating X -> XN -> X ...; stats[t] (if
+// non-NULL) receives the statistics after step t. One host barrier at the end.
+spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
+                         int64_t nsteps, somier_stats_t* stats) {
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    spread_status st = ensure_acc(h, nsteps);
+    if (st != SPREAD_OK) return st;
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * (size_t)nsteps * sizeof(paper::StatsAccum), d.s_comp));
+    }
+    for (int64_t t = 0; t < nsteps; t++) {
+        st = (t & 1) ? enqueue_stream_step(h, XN, V, X, t, t > 0) : enqueue_stream_step(h, X, V, XN, t, t > 0);
+        if (st != SPREAD_OK) return st;
+    }
+    st = sync_devs(h);
+    if (st != SPREAD_OK) return st;
+    const int64_t step0 = h->step;
+    h->step += nsteps;
+    if (!stats) return SPREAD_OK;
+    std::vector<__int128> sums((size_t)nsteps * 3, 0);
+    std::vector<unsigned long long> vmax2((size_t)nsteps, 0);
+    std::vector<paper::StatsAccum> acc((size_t)nsteps * 2);
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaMemcpy(acc.data(), d.acc_base, acc.size() * sizeof(paper::StatsAccum), cudaMemcpyDeviceToHost));
+        for (int64_t t = 0; t < nsteps; t++)
+            for (int q = 0; q < 2; q++) {
+                const paper::StatsAccum& a = acc[(size_t)(2 * t + q)];
+                for (int k = 0; k < 3; k++)
+                    sums[(size_t)(3 * t + k)] += (__int128)(((unsigned __int128)a.hi[k] << 64) | a.lo[k]);
+                vmax2[(size_t)t] = std::max(vmax2[(size_t)t], (unsigned long long)a.vmax2);
+            }
+    }
+    for (int64_t t = 0; t < nsteps; t++)
+        paper::finish_somier_stats(&h->p, &sums[(size_t)(3 * t)], vmax2[(size_t)t],
+                                   h->p.n[0] * h->p.n[1] * h->p.n[2], step0 + t + 1, &stats[t]);
     return SPREAD_OK;
 }
 
@@ -171,15 +329,16 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         for (cudaStream_t* ps : {&d.s_h2d, &d.s_comp, &d.s_d2h})
             if ((e = cudaStreamCreateWithFlags(ps, cudaStreamNonBlocking)) != cudaSuccess)
                 return fail(sfail(h, e, "cudaStreamCreate"));
-        if ((e = cudaMalloc(&d.acc_base, 2 * sizeof(paper::StatsAccum))) != cudaSuccess)
+        if ((e = cudaMalloc(&d.acc_base, 2 * kAccSteps * sizeof(paper::StatsAccum))) != cudaSuccess)
             return fail(sfail(h, e, "cudaMalloc(stats)"));
+        d.acc_steps = kAccSteps;
         d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
         for (auto& sl : d.slots) {
             if ((e = cudaMalloc(&sl.base, 2 * xb + vb)) != cudaSuccess) return fail(sfail(h, e, "cudaMalloc(slot)"));
             sl.x_in = (double*)sl.base;
             sl.x_out = (double*)((char*)sl.base + xb);
             sl.v = (double*)((char*)sl.base + 2 * xb);
-            for (cudaEvent_t* pe : {&sl.h2d_done, &sl.comp_done, &sl.d2h_done})
+            for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
                 if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
                     return fail(sfail(h, e, "cudaEventCreate"));
             paper::SlabGeom g = h->geom;
@@ -192,6 +351,15 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
             st = paper::encode_slab_tmap(&sl.tmap_v2, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kV2BoxJ);
             if (st != SPREAD_OK) return fail(st);
         }
+    }
+    h->ev.resize((size_t)s->nchunks);
+    for (int64_t c = 0; c < s->nchunks; c++) {
+        if ((e = cudaSetDevice(h->devs[s->chunk_info(c).pos].device)) != cudaSuccess)
+            return fail(sfail(h, e, "cudaSetDevice"));
+        for (int q = 0; q < 2; q++)
+            for (cudaEvent_t* pe : {&h->ev[c].h2d[q], &h->ev[c].d2h[q]})
+                if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
+                    return fail(sfail(h, e, "cudaEventCreate"));
     }
     *out = h;
     return SPREAD_OK;
@@ -247,96 +415,24 @@ spread_status somier_stream_step(somier_stream_t h, const double* x, const doubl
     if (!h || !x || !y || !z || !vx || !vy || !vz || !xn || !yn || !zn)
         PAPER_FAIL(SPREAD_EINVAL, "somier_stream_step: NULL argument");
     if (x == xn || y == yn || z == zn) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_step: X_t and X_{t+1} alias (Jacobi)");
-    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     double* X[3] = {const_cast<double*>(x), const_cast<double*>(y), const_cast<double*>(z)};
     double* XN[3] = {xn, yn, zn};
     double* V[3] = {vx, vy, vz};
-    const int64_t n0 = h->p.n[0];
-    for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
-        S_TRY(h, cudaSetDevice(d.device));
-        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * sizeof(paper::StatsAccum), d.s_comp));
-    }
-    size_t maxm = 0;
-    for (auto& d : h->devs) maxm = std::max(maxm, d.chunks.size());
-    for (size_t m = 0; m < maxm; m++) {
-        for (auto& d : h->devs) {
-            if (m >= d.chunks.size()) continue;
-            Slot& sl = d.slots[m % d.slots.size()];
-            const paper::ChunkInfo c = h->spread.chunk_info(d.chunks[m]);
-            const paper::SlabGeom g = geom_of(h, c);
-            const bool first = c.start == 1, last = c.start + c.size == n0 - 1;
-            S_TRY(h, cudaSetDevice(d.device));
-            // map(to: X[start-1 : size+2], V[start : size])
-            if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
-            for (int q = 0; q < 3; q++) {
-                S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, X[q], c.start - 1, c.size + 2,
-                                                 cudaMemcpyHostToDevice, d.s_h2d));
-                S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], c.start, c.size, cudaMemcpyHostToDevice,
-                                                 d.s_h2d));
-            }
-            S_TRY(h, cudaEventRecord(sl.h2d_done, d.s_h2d));
-            // the fused step (forces, accelerations, velocities, positions, centers)
-            S_TRY(h, cudaStreamWaitEvent(d.s_comp, sl.h2d_done, 0));
-            if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, d.acc() + 1, d.s_comp));
-            if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, c.size + 1, 1, d.acc() + 1, d.s_comp));
-            paper::StepArgs a;
-            std::memset(&a, 0, sizeof a);
-            a.x_cur = sl.x_in;
-            a.x_nxt = sl.x_out;
-            a.v = sl.v;
-            a.g = g;
-            a.K = h->p.k_spring;
-            a.L = h->p.rest_len;
-            a.M = h->p.mass;
-            a.dt = h->p.dt;
-            a.acc = d.acc();
-            a.tmap_x_cur = &sl.tmap_x;
-            a.tmap_v = &sl.tmap_v;
-            a.tmap_x2_cur = &sl.tmap_x2;
-            a.tmap_v2 = &sl.tmap_v2;
-            a.write_fixed = 1;
-            const paper::K1Variant var = paper::k1_variant(h->p.kernel);
-            S_TRY(h, paper::launch_k1(var, a, h->p.mass == 1.0, d.s_comp));
-            h->launches++;
-            S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
-            // map(from: X[start : size], V[start : size]) (+ the fixed end planes)
-            S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
-            for (int q = 0; q < 3; q++) {
-                S_TRY(h, paper::copy_slab_planes(g, sl.x_out, q, 1, XN[q], c.start, c.size, cudaMemcpyDeviceToHost,
-                                                 d.s_d2h));
-                S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], c.start, c.size, cudaMemcpyDeviceToHost,
-                                                 d.s_d2h));
-                if (first)
-                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, XN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
-                if (last)
-                    S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, c.size + 1, XN[q], n0 - 1, 1,
-                                                     cudaMemcpyDeviceToHost, d.s_d2h));
-            }
-            S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
-            sl.used = true;
-        }
-    }
-    spread_status st = sync_devs(h);
-    if (st != SPREAD_OK) return st;
-    h->step++;
-    if (stats) {
-        __int128 sums[3] = {0, 0, 0};
-        unsigned long long vmax2 = 0;
-        for (auto& d : h->devs) {
-            if (d.chunks.empty()) continue;
-            paper::StatsAccum acc[2];
-            S_TRY(h, cudaSetDevice(d.device));
-            S_TRY(h, cudaMemcpy(acc, d.acc_base, sizeof acc, cudaMemcpyDeviceToHost));
-            for (int q = 0; q < 2; q++) {
-                for (int k = 0; k < 3; k++)
-                    sums[k] += (__int128)(((unsigned __int128)acc[q].hi[k] << 64) | acc[q].lo[k]);
-                vmax2 = std::max(vmax2, (unsigned long long)acc[q].vmax2);
-            }
-        }
-        paper::finish_somier_stats(&h->p, sums, vmax2, h->p.n[0] * h->p.n[1] * h->p.n[2], h->step, stats);
-    }
-    return SPREAD_OK;
+    return stream_run(h, X, V, XN, 1, stats);
+}
+
+spread_status somier_stream_run(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                double* vz, double* xn, double* yn, double* zn, int64_t nsteps,
+                                somier_stats_t* stats) {
+    if (!h || !x || !y || !z || !vx || !vy || !vz || !xn || !yn || !zn)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run: NULL argument");
+    if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run: nsteps %lld < 0", (long long)nsteps);
+    if (x == xn || y == yn || z == zn) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run: the two X buffers alias");
+    if (nsteps == 0) return SPREAD_OK;
+    double* X[3] = {x, y, z};
+    double* XN[3] = {xn, yn, zn};
+    double* V[3] = {vx, vy, vz};
+    return stream_run(h, X, V, XN, nsteps, stats);
 }
 
 spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches) {

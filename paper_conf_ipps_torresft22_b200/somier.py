@@ -281,6 +281,18 @@ class SomierStream:
                                            *[_dptr(g) for g in XN], ctypes.byref(out)), "somier_stream_step")
         return Stats.from_c(out)
 
+    def run(self, X, V, XN, nsteps: int, stats: bool = True):
+        """nsteps steps with chunk-level dependencies (somier_stream_run): X and
+        XN are used alternately, X_{nsteps} ends in X if nsteps is even, else in
+        XN. Returns the per-step Stats (or None)."""
+        return self.run_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]], nsteps, stats)
+
+    def run_ptrs(self, X, V, XN, nsteps: int, stats: bool = True):
+        out = (N.somier_stats_t * max(1, int(nsteps)))() if stats else None
+        N.check(N.lib().somier_stream_run(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
+                                          *[_dptr(g) for g in XN], int(nsteps), out), "somier_stream_run")
+        return [Stats.from_c(out[t]) for t in range(int(nsteps))] if stats else None
+
     def traffic(self):
         a, b, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
         N.check(N.lib().somier_stream_traffic(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)),

@@ -107,3 +107,50 @@ def test_stream_irregular_chunks(sizes, buffers):
     ref, rst = O.run(O.init(_op(sp)), 7)
     assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
     assert st.sums == rst.sums
+
+
+def _pinned_like(a):
+    return torch.empty(a.shape, dtype=torch.float64, pin_memory=True).numpy()
+
+
+@pytest.mark.parametrize("devices,spread_kw,buffers,nsteps", [
+    ([0], {"chunk": 3}, 2, 9), ([0], {"chunk": 4}, 1, 10), ([0, 1, 2], {"chunk": 2}, 2, 9),
+    ([0, 1], {"sizes": [1, 6, 2, 1, 4]}, 3, 8), ([0, 1, 2, 3], {"chunk": 0}, 2, 5), ([0], {"chunk": 100}, 2, 4)])
+def test_stream_run_chunk_level_depend(devices, spread_kw, buffers, nsteps):
+    """somier_stream_run: steps chained by per-chunk events only (no barrier per
+    step), on pinned host memory so the copies really run asynchronously;
+    every step's stats and the final state equal the oracle's bit for bit."""
+    n = (16, 13, 37)
+    sp = P.SomierParams(n=n, seed=6)
+    if "sizes" in spread_kw:
+        spread = P.Spread.with_sizes(devices, 1, n[0] - 2, spread_kw["sizes"])
+    else:
+        spread = P.Spread(devices, 1, n[0] - 2, chunk=spread_kw["chunk"])
+    with P.SomierStream(spread, sp, buffers=buffers, cuda_devices=[0] * len(devices)) as s:
+        X0, V0 = s.generate()
+        X, V, XN = _pinned_like(X0), _pinned_like(V0), _pinned_like(X0)
+        X[...] = X0
+        V[...] = V0
+        XN[...] = np.nan
+        stats = s.run(X, V, XN, nsteps)
+    final = X if nsteps % 2 == 0 else XN
+    ref = O.init(_op(sp))
+    for t in range(nsteps):
+        ref, rst = O.step(ref)
+        assert stats[t].sums == rst.sums and stats[t].vmax2_bits == rst.vmax2_bits and stats[t].step == t + 1
+    assert np.array_equal(final, ref.X) and np.array_equal(V, ref.V)
+
+
+def test_stream_run_equals_steps_and_continues():
+    sp = P.SomierParams(n=(12, 10, 33), seed=9)
+    with P.SomierStream(P.Spread([0], 1, 10, chunk=3), sp, buffers=2) as s:
+        X, V = s.generate()
+        XN = np.zeros_like(X)
+        s.run(X, V, XN, 3, stats=False)          # X_3 in XN
+        st = s.run(XN, V, X, 4)[-1]              # X_7 in XN
+        assert st.step == 7
+        assert s.run(XN, V, X, 0) == []
+        with pytest.raises(P.SpreadError):
+            s.run(X, V, X, 2)
+    ref, rst = O.run(O.init(_op(sp)), 7)
+    assert np.array_equal(XN, ref.X) and np.array_equal(V, ref.V) and st.sums == rst.sums

@@ -52,6 +52,11 @@ struct StepArgs {
     // Host-streamed mode: x_nxt is a fresh buffer, so fixed face nodes of the
     // owned planes are copied into it too (resident mode leaves them in place).
     int write_fixed;
+    // K1_MARCH2: launch with programmatic stream serialization (PDL): the
+    // kernel's prologue (barrier init, tensor-map prefetch) overlaps the tail
+    // of the previous kernel on the stream; every thread executes
+    // griddepcontrol.wait before touching global memory.
+    int pdl;
 };
 
 struct InitArgs {

@@ -171,9 +171,6 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int q0 = pb - 1;
     const int qlast = pe;
 
-    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
-        reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
-
     auto issue = [&](int q) {  // X of plane q
         const int s = (q - q0) % kStages;
         mbar_expect_tx(&sm.full[s], kXBoxBytes);
@@ -196,6 +193,17 @@ __global__ void __launch_bounds__(kThreads, 2)
         for (int s = 0; s < kStages; s++) mbar_init(&sm.full[s], 1);
         for (int s = 0; s < kVStages; s++) mbar_init(&sm.vfull[s], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    // PDL: everything above overlapped the previous kernel on the stream; from
+    // here on global memory is touched (it read the X buffer this step writes,
+    // and wrote the X_t / V this step reads). A no-op without PDL.
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
+        reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
+    // Every CTA is resident once all have passed this point, so the next
+    // step's CTAs can only take slots freed by finished CTAs of this one.
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    if (tid == 0) {
         fence_proxy_async();
         for (int q = q0; q < q0 + kStages && q <= qlast; q++) issue(q);
         for (int p = pb; p < pb + kVStages && p < pe; p++) issue_v(p);
@@ -342,7 +350,17 @@ cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t str
     const CUtensorMap& mv = *static_cast<const CUtensorMap*>(a.tmap_v2);
     auto launch = [&](auto kernel) {
         cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        kernel<<<grid, block, smem, stream>>>(mx, mv, mp);
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = grid;
+        cfg.blockDim = block;
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = stream;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = a.pdl ? 1 : 0;
+        cudaLaunchKernelEx(&cfg, kernel, mx, mv, mp);
     };
     const bool pos_k = a.K > 0.0;
     if (unit_mass)

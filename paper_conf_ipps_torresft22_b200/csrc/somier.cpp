@@ -131,6 +131,7 @@ struct somier_s {
     bool connected = true;
     // CUDA graph of an (even, odd) step pair, when every chunk is on one stream
     bool graph_ok = false;
+    bool pdl = false;
     int graph_pos = -1;
     cudaGraphExec_t graph_exec = nullptr;
 
@@ -453,6 +454,11 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         const char* ng = std::getenv("SOMIER_NO_GRAPH");
         h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1') && !h->tb2;
         h->graph_pos = pos;
+        // PDL between consecutive K1 launches only where nothing else sits
+        // between them on the stream (one stream, no flag waits); SOMIER_NO_PDL=1
+        // disables it
+        const char* np = std::getenv("SOMIER_NO_PDL");
+        h->pdl = one && pos >= 0 && !(np && np[0] == '1');
     }
     *out = h;
     return SPREAD_OK;
@@ -790,6 +796,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.tmap_v = &me.tmap_v[vb];
             a.tmap_x2_cur = &me.tmap_x2[cur];
             a.tmap_v2 = &me.tmap_v2[vb];
+            a.pdl = h->pdl ? 1 : 0;
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
             h->launches++;
         }

@@ -1,10 +1,14 @@
 #!/usr/bin/env python3
 """The paper's experiment shape on one B200 (Table I):
 Somier 1200^3, fp64, 31 time steps, state in HOST memory streamed through the
-GPU every step (somier_stream_step). The paper's whole-program wall times
-(Table I) were 1058.9 s on 1 V100 and 502.0 s on 4 V100.
+GPU every step. The paper's whole-program wall times (Table I,
+PAPER.md:669-672) were 1058.9 s on 1 V100 and 502.0 s on 4 V100.
 
-  python tools/paper_run.py [n] [steps] [chunk] [buffers]
+  python tools/paper_run.py [n] [steps] [chunk] [buffers] [run|step]
+
+mode run (default): somier_stream_run, steps chained by per-chunk events (the
+paper's future-work `depend`); step: somier_stream_step, a barrier per step
+(the paper's taskgroup).
 """
 import json
 import os
@@ -20,6 +24,7 @@ n = int(sys.argv[1]) if len(sys.argv) > 1 else 1200
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 31
 chunk = int(sys.argv[3]) if len(sys.argv) > 3 else 64
 buffers = int(sys.argv[4]) if len(sys.argv) > 4 else 3
+mode = sys.argv[5] if len(sys.argv) > 5 else "run"
 t_all = time.perf_counter()
 params = P.SomierParams(n=(n, n, n), seed=42)
 st = P.SomierStream(P.Spread([0], 1, n - 2, chunk=chunk), params, buffers=buffers)
@@ -32,14 +37,18 @@ st.generate_ptrs(X + V)
 t_gen = time.perf_counter() - t0
 per = []
 t0 = time.perf_counter()
-for _ in range(steps):
-    a = time.perf_counter()
-    stats = st.step_ptrs(X, V, XN)
-    per.append(time.perf_counter() - a)
-    X, XN = XN, X
+if mode == "run":
+    stats = st.run_ptrs(X, V, XN, steps)[-1]
+    per = [(time.perf_counter() - t0) / steps]
+else:
+    for _ in range(steps):
+        a = time.perf_counter()
+        stats = st.step_ptrs(X, V, XN)
+        per.append(time.perf_counter() - a)
+        X, XN = XN, X
 t_steps = time.perf_counter() - t0
 tr = st.traffic()
-out = {"n": n, "steps": steps, "chunk": chunk, "buffers": buffers, "host_state_gib": 9 * n ** 3 * 8 / 2 ** 30,
+out = {"n": n, "steps": steps, "chunk": chunk, "buffers": buffers, "mode": mode, "host_state_gib": 9 * n ** 3 * 8 / 2 ** 30,
        "pin_s": t_pin, "generate_s": t_gen, "steps_s": t_steps, "s_per_step": t_steps / steps,
        "per_step_min_max": [min(per), max(per)], "node_updates_per_s": (n - 2) ** 3 * steps / t_steps,
        "h2d_gb_per_step": tr["h2d_bytes"] / 1e9, "d2h_gb_per_step": tr["d2h_bytes"] / 1e9,

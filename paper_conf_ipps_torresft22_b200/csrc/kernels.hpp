@@ -69,6 +69,13 @@ struct InitArgs {
 
 enum class K1Variant { Direct = 1, March = 2, March2 = 3 };
 
+// K1_TB2: warps per CTA; the CTA's ring-extended tile is 32 x (2 * kTB2Warps)
+// and its TMA boxes are 34 x (2 * kTB2Warps + 2) (X) and 34 x (2 * kTB2Warps) (V).
+#ifndef TB2_WARPS
+#define TB2_WARPS 12
+#endif
+constexpr int kTB2Warps = TB2_WARPS;
+
 cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cudaStream_t stream);
 // K1_TB2: two steps in one launch (a.x_cur / a.v / tmaps with the TB2 box
 // shapes -> x_out / v_out; stats of the first step into acc1, second into a.acc)

@@ -2,22 +2,28 @@
 // temporal blocking), for a chunk without neighbour chunks (one slab per
 // device, no halo exchange).
 //
-// Why: K1 is energy-bound under the 1 kW cap and the HBM traffic is ~3/4 of
-// its energy (tools/power_probe.py). Doing steps t and t+1 in
-// one pass halves the bytes per node-update (96 B -> 48 B) at the price of
+// Why: K1 is energy-bound under the 1 kW cap and HBM traffic is most of its
+// energy (tools/power_probe.py). Doing steps t and t+1 in one
+// pass halves the bytes per node-update (96 B -> 48 B) at the price of
 // recomputing step t on a one-node ring around each tile.
 //
-// Layout of the work: a CTA = 16 warps x 32 lanes = the ring-extended region
-// R1 (32 k x 16 j) of an owned tile R2 (30 k x 14 j, lanes 1..30, rows
-// 1..14). Marching along i, iteration p does
-//   step t   on plane p   for all of R1  (X_t from a TMA ring, V_t from a TMA
-//            ring; X_{t+1} of R1 kept in shared memory, V_{t+1} in registers)
-//   step t+1 on plane p-1 for R2          (neighbours all inside R1)
+// Layout of the work (v2): a CTA = kTB2Warps warps; warp w owns the two
+// ADJACENT rows 2w, 2w+1 of the ring-extended region R1 (32 k x 2*kTB2Warps j)
+// of an owned tile R2 (lanes 1..30, rows 1..2*kTB2Warps-2). Marching along i,
+// iteration p does
+//   S1: step t   on plane p   for all of R1  (X_t from a TMA ring, V_t from a
+//       TMA ring; X_{t+1} of R1 goes to a two-plane shared-memory ring, V_{t+1}
+//       stays in registers for one iteration)
+//   S2: step t+1 on plane p-1 for R2         (neighbours all inside R1)
 // and writes X_{t+2}, V_{t+2} of R2 to the OTHER X / V buffers (X and V are
 // double-buffered here because neighbouring tiles read X_t / V_t of this
-// tile's ring). Both steps use node_math.cuh, so every node update is the same
-// IEEE expression as in K1_DIRECT / K1_MARCH (bit-identical), and the stats
-// of BOTH steps are accumulated (step t into acc1, step t+1 into acc).
+// tile's ring). As in K1_MARCH2 each spring is evaluated once per step (+i, +j,
+// +k per node; -i from a register carry, -k from a lane shuffle, -j from the
+// paired row or shared memory), two CTA barriers per plane. Both steps use
+// node_math.cuh, so every node update is the same IEEE expression as in
+// K1_DIRECT / K1_MARCH2 (bit-identical). Only step t+1's stats are accumulated:
+// the handle's stats are those of the last completed step, and TB2 always
+// completes steps in pairs.
 #include <cuda.h>
 
 #include <algorithm>
@@ -31,49 +37,55 @@ namespace paper {
 
 namespace {
 
-constexpr int kTK = 32, kW = 16, kThreads = kTK * kW;
-constexpr int kOK = kTK - 2, kOJ = kW - 2;                  // owned tile 30 x 14
-constexpr int kBK = kTK + 2, kBJ = kW + 2;                  // X_t box: R1 + ring (34 x 18)
+constexpr int kTK = 32, kW = kTB2Warps, kThreads = kTK * kW;
+constexpr int kRows = 2 * kW;                               // R1 rows
+constexpr int kOK = kTK - 2, kOJ = kRows - 2;               // owned tile R2
+constexpr int kBK = kTK + 2, kBJ = kRows + 2;               // X_t box: R1 + ring
 constexpr int kXComp = kBK * kBJ;
-constexpr int kXBoxBytes = kXComp * 3 * 8;                  // 14688
-constexpr int kXSlot = 14720;
-constexpr int kVBK = kTK + 2, kVBJ = kW;                    // V_t box: R1 (+1 col for alignment) 34 x 16
+constexpr int kXBoxBytes = kXComp * 3 * 8;
+constexpr int kXSlot = (kXBoxBytes + 127) / 128 * 128;
+constexpr int kVBK = kTK + 2, kVBJ = kRows;                 // V_t box: R1 (+1 col each side for alignment)
 constexpr int kVComp = kVBK * kVBJ;
-constexpr int kVBoxBytes = kVComp * 3 * 8;                  // 13056
-constexpr int kYComp = kTK * kW;                            // X_{t+1} of R1: 32 x 16
+constexpr int kVBoxBytes = kVComp * 3 * 8;
+constexpr int kVSlot = (kVBoxBytes + 127) / 128 * 128;
+constexpr int kYComp = kRows * kTK;                         // X_{t+1} of one R1 plane, per component
 #ifndef TB2_STAGES
 #define TB2_STAGES 3
 #endif
 #ifndef TB2_VSTAGES
-#define TB2_VSTAGES 3
+#define TB2_VSTAGES 2
 #endif
 constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
 constexpr int kSegPlanes = 64, kMinSegPlanes = 4;
+static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
 
 struct __align__(16) Smem {
     unsigned char xst[kStages][kXSlot];
-    unsigned char vst[kVStages][kVBoxBytes];
-    double y[2][3][kYComp];        // X_{t+1} of R1, two planes
-    Vec3 gj1[2][kW][kTK];          // step t: +j springs by plane parity
-    Vec3 gj2[2][kW][kTK];          // step t+1
-    Vec3 gbj[2][kTK];              // step t tile-border springs (row above R1)
-    Vec3 gbk[2][kW];               // step t tile-border springs (column left of R1)
+    unsigned char vst[kVStages][kVSlot];
+    double y[2][3][kYComp];        // X_{t+1} of R1, planes by parity
+    Vec3 g1j[kW][kTK];             // S1: +j spring of each warp's second row
+    Vec3 g2j[kW][kTK];             // S2: same
+    Vec3 gbj[kTK];                 // S1 tile-border springs (row above R1 -> R1 row 0)
+    Vec3 gbk[kRows];               // S1 tile-border springs (column left of R1 -> R1 lane 0)
     unsigned long long full[kStages];
     unsigned long long vfull[kVStages];
-    WarpStats scratch[kThreads / 32];
+    WarpStats scratch[kW];
 };
 
 struct Tb2Params {
     StepArgs a;
     double* x_out;                 // X_{t+2} buffer
     double* v_out;                 // V_{t+2} buffer
-    StatsAccum* acc1;              // stats of step t (X_{t+1})
     int tiles_k, tiles_j, seg_planes;
 };
 
 __device__ __forceinline__ Vec3 shfl_up1(const Vec3& v) {
     return Vec3{__shfl_up_sync(0xffffffffu, v.x, 1), __shfl_up_sync(0xffffffffu, v.y, 1),
                 __shfl_up_sync(0xffffffffu, v.z, 1)};
+}
+
+__device__ __forceinline__ Vec3 ldb(const double* b, int off, int comp) {
+    return Vec3{b[off], b[off + comp], b[off + 2 * comp]};
 }
 
 template <bool kUnitMass, bool kPosK>
@@ -86,15 +98,16 @@ __global__ void __launch_bounds__(kThreads, 1)
     const SlabGeom& g = a.g;
     const int lane = threadIdx.x, w = threadIdx.y, tid = w * kTK + lane;
     const int tile_k = blockIdx.x % tp.tiles_k, tile_j = blockIdx.x / tp.tiles_k;
-    const int kq = tile_k * kOK, jq = tile_j * kOJ;  // owned tile origin
-    const int k = kq - 1 + lane, j = jq - 1 + w;     // this thread's R1 node
+    const int kq = tile_k * kOK, jq = tile_j * kOJ;  // owned tile origin (kq even: TMA inner coordinate)
+    const int rA = 2 * w, rB = rA + 1;               // R1 rows of this thread
+    const int k = kq - 1 + lane, jA = jq - 1 + rA, jB = jA + 1;
     const int size = (int)g.size;
     const int pb = 1 + blockIdx.y * tp.seg_planes;
-    const int pe = min(size + 1, pb + tp.seg_planes);  // step-(t+1) outputs [pb, pe)
-    const int p_first = max(0, pb - 1);                // step-t planes [p_first, pe]
-    const int q0 = max(0, p_first - 1);                // X_t planes [q0, qlast]
+    const int pe = min(size + 1, pb + tp.seg_planes);  // S2 (step t+1) output planes [pb, pe)
+    const int ps0 = pb - 1;                            // S1 (step t) planes [ps0, pe]
+    const int q0 = max(0, ps0 - 1);                    // X_t planes [q0, qlast]
     const int qlast = min(size + 1, pe + 1);
-    const int v_first = max(1, p_first), v_last = min(size, pe);  // V_t planes read
+    const int v_first = max(1, ps0), v_last = min(size, pe);  // V_t planes read (S1 on non-fixed planes)
 
     auto issue_x = [&](int q) {
         const int s = (q - q0) % kStages;
@@ -117,146 +130,190 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int p = v_first; p < v_first + kVStages && p <= v_last; p++) issue_v(p);
     }
     __syncthreads();
-
     auto xbox = [&](int q) { return reinterpret_cast<const double*>(sm.xst[(q - q0) % kStages]); };
     auto xwait = [&](int q) { mbar_wait(&sm.full[(q - q0) % kStages], (unsigned)(((q - q0) / kStages) & 1)); };
-    const int xo_own = (w + 1) * kBK + (lane + 1);
-    auto ldx = [&](const double* b, int off) { return Vec3{b[off], b[off + kXComp], b[off + 2 * kXComp]}; };
 
-    const bool valid = k >= 0 && k < g.n2 && j >= 0 && j < g.n1;
-    const bool interior = k >= 1 && k < g.n2 - 1 && j >= 1 && j < g.n1 - 1;
-    const bool owned = valid && lane >= 1 && lane <= kOK && w >= 1 && w <= kOJ;
+    const int xA = (rA + 1) * kBK + (lane + 1), xB = xA + kBK;   // own X box offsets
+    const int vA = rA * kVBK + (lane + 1), vB = vA + kVBK;        // own V box offsets
+    const int yA = rA * kTK + lane, yB = yA + kTK;                // own X_{t+1} ring offsets
+    const int yAk = lane < kTK - 1 ? yA + 1 : yA;                 // +k neighbour (lane 31 is ring: unused)
+    const int yBk = lane < kTK - 1 ? yB + 1 : yB;
+    const int yBj = w < kW - 1 ? yB + kTK : yB;                   // +j neighbour of row B (last row is ring)
+    const bool kin = k >= 1 && k < g.n2 - 1;
+    const bool intA = kin && jA >= 1 && jA < g.n1 - 1, intB = kin && jB >= 1 && jB < g.n1 - 1;
+    const bool kown = lane >= 1 && lane <= kOK && k < g.n2;
+    const bool ownA = kown && rA >= 1 && jA < g.n1;               // rows 1 .. kRows-2
+    const bool ownB = kown && rB <= kRows - 2 && jB < g.n1;
     const int64_t cs = g.comp_stride(), ps = g.plane_stride();
-    const int64_t off = owned ? (int64_t)j * g.ld + k : 0;
+    const int64_t offA = ownA ? (int64_t)jA * g.ld + k : 0, offB = ownB ? (int64_t)jB * g.ld + k : 0;
 
-    // prologue: X_t(p_first) own, and the step-t -i spring of plane p_first
-    Vec3 carry1{0.0, 0.0, 0.0}, xc1;
-    xwait(p_first);
-    xc1 = ldx(xbox(p_first), xo_own);
-    if (p_first >= 1) {
-        xwait(p_first - 1);
-        carry1 = spring_force<kPosK>(ldx(xbox(p_first - 1), xo_own), xc1, a.K, a.L);
+    // prologue: X_t(ps0) own, and the step-t -i spring of plane ps0
+    Vec3 carry1A{0.0, 0.0, 0.0}, carry1B{0.0, 0.0, 0.0};
+    xwait(ps0);
+    Vec3 xcA = ldb(xbox(ps0), xA, kXComp), xcB = ldb(xbox(ps0), xB, kXComp);
+    if (ps0 >= 1) {
+        xwait(ps0 - 1);
+        carry1A = spring_force<kPosK>(ldb(xbox(ps0 - 1), xA, kXComp), xcA, a.K, a.L);
+        carry1B = spring_force<kPosK>(ldb(xbox(ps0 - 1), xB, kXComp), xcB, a.K, a.L);
+        __syncthreads();
+        if (tid == 0 && q0 + kStages <= qlast) {
+            fence_proxy_async();
+            issue_x(q0 + kStages);  // X_t(ps0 - 1) is no longer needed
+        }
     }
-    Vec3 carry2{0.0, 0.0, 0.0};
-    Vec3 vhold{0.0, 0.0, 0.0};
-    NodeStats st1, st2;
-    st1.zero();
-    st2.zero();
-    __syncthreads();
-    if (tid == 0 && p_first >= 1 && q0 + kStages <= qlast) {
-        fence_proxy_async();
-        issue_x(q0 + kStages);  // X_t(p_first - 1) is no longer needed
-    }
+    Vec3 carry2A{0.0, 0.0, 0.0}, carry2B{0.0, 0.0, 0.0};
+    Vec3 v1pA{0.0, 0.0, 0.0}, v1pB{0.0, 0.0, 0.0};  // V_{t+1} of plane p-1
+    NodeStats st;
+    st.zero();
 
-    for (int p = p_first; p <= pe; p++) {
+    for (int p = ps0; p <= pe; p++) {
         const int par = p & 1;
-        const bool upd1 = p >= 1 && p <= size;  // step t updates plane p
+        const bool upd1 = p >= 1 && p <= size;  // S1 updates plane p (else a fixed face plane)
         const bool has_next = p + 1 <= qlast;
         if (has_next) xwait(p + 1);
         const double* Xc = xbox(p);
         const double* Xn = has_next ? xbox(p + 1) : Xc;
-        // ---- step t, phase A: "+" springs
-        Vec3 gpi1{0.0, 0.0, 0.0}, gpj1{0.0, 0.0, 0.0}, gpk1{0.0, 0.0, 0.0};
-        const Vec3 xn1 = ldx(Xn, xo_own);
-        if (has_next) gpi1 = spring_force<kPosK>(xc1, xn1, a.K, a.L);
+        // ---- S1 "+" springs of plane p
+        Vec3 gpi1A{0.0, 0.0, 0.0}, gpi1B{0.0, 0.0, 0.0};
+        Vec3 gpj1A{0.0, 0.0, 0.0}, gpj1B{0.0, 0.0, 0.0}, gpk1A{0.0, 0.0, 0.0}, gpk1B{0.0, 0.0, 0.0};
+        const Vec3 niA = ldb(Xn, xA, kXComp), niB = ldb(Xn, xB, kXComp);
+        if (has_next) {
+            gpi1A = spring_force<kPosK>(xcA, niA, a.K, a.L);
+            gpi1B = spring_force<kPosK>(xcB, niB, a.K, a.L);
+        }
         if (upd1) {
-            gpk1 = spring_force<kPosK>(xc1, ldx(Xc, xo_own + 1), a.K, a.L);
-            gpj1 = spring_force<kPosK>(xc1, ldx(Xc, xo_own + kBK), a.K, a.L);
-            sm.gj1[par][w][lane] = gpj1;
+            gpk1A = spring_force<kPosK>(xcA, ldb(Xc, xA + 1, kXComp), a.K, a.L);
+            gpk1B = spring_force<kPosK>(xcB, ldb(Xc, xB + 1, kXComp), a.K, a.L);
+            gpj1A = spring_force<kPosK>(xcA, xcB, a.K, a.L);
+            gpj1B = spring_force<kPosK>(xcB, ldb(Xc, xB + kBK, kXComp), a.K, a.L);
+            sm.g1j[w][lane] = gpj1B;
             if (w == 0) {
-                sm.gbj[par][lane] = spring_force<kPosK>(ldx(Xc, lane + 1), ldx(Xc, kBK + lane + 1), a.K, a.L);
-            } else if (w == 1 && lane < kW) {
+                sm.gbj[lane] = spring_force<kPosK>(ldb(Xc, lane + 1, kXComp), ldb(Xc, kBK + lane + 1, kXComp), a.K,
+                                                   a.L);
+            } else if (w == 1 && lane < kRows) {
                 const int r = (lane + 1) * kBK;
-                sm.gbk[par][lane] = spring_force<kPosK>(ldx(Xc, r), ldx(Xc, r + 1), a.K, a.L);
+                sm.gbk[lane] = spring_force<kPosK>(ldb(Xc, r, kXComp), ldb(Xc, r + 1, kXComp), a.K, a.L);
             }
         }
-        const Vec3 up1 = shfl_up1(gpk1);
-        __syncthreads();  // A: X_t(p) is read for the last time above
+        const Vec3 up1A = shfl_up1(gpk1A), up1B = shfl_up1(gpk1B);
+        __syncthreads();  // #1: S1 springs visible; X_t(p) read for the last time
         if (tid == 0 && p + kStages <= qlast) {
             fence_proxy_async();
             issue_x(p + kStages);
         }
-        // ---- step t, phase B: forces -> V_{t+1}, X_{t+1} of R1 plane p
-        Vec3 x1 = xc1, v1{0.0, 0.0, 0.0};
+        // ---- S1 forces -> V_{t+1}, X_{t+1} of R1, plane p
+        Vec3 x1A = xcA, x1B = xcB, v1A{0.0, 0.0, 0.0}, v1B{0.0, 0.0, 0.0};
         if (upd1) {
             const int vs = (p - v_first) % kVStages;
             mbar_wait(&sm.vfull[vs], (unsigned)(((p - v_first) / kVStages) & 1));
-            if (interior) {
-                const Vec3 gmj = neg(w == 0 ? sm.gbj[par][lane] : sm.gj1[par][w - 1][lane]);
-                const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][w] : up1);
-                const Vec3 F = sum_forces(neg(carry1), gpi1, gmj, gpj1, gmk, gpk1);
-                const double* vb = reinterpret_cast<const double*>(sm.vst[vs]) + w * kVBK + (lane + 1);
-                v1 = Vec3{vb[0], vb[kVComp], vb[2 * kVComp]};
-                kick_drift<kUnitMass>(F, a.M, a.dt, v1, xc1, x1);
+            const double* Vb = reinterpret_cast<const double*>(sm.vst[vs]);
+            if (intA) {
+                const Vec3 gmj = neg(w == 0 ? sm.gbj[lane] : sm.g1j[w - 1][lane]);
+                const Vec3 gmk = neg(lane == 0 ? sm.gbk[rA] : up1A);
+                const Vec3 F = sum_forces(neg(carry1A), gpi1A, gmj, gpj1A, gmk, gpk1A);
+                v1A = ldb(Vb, vA, kVComp);
+                kick_drift<kUnitMass>(F, a.M, a.dt, v1A, xcA, x1A);
             }
-            if (owned && p >= pb && p < pe) {
-                st1.add_position(x1);
-                if (interior) st1.add_velocity(v1);
+            if (intB) {
+                const Vec3 gmk = neg(lane == 0 ? sm.gbk[rB] : up1B);
+                const Vec3 F = sum_forces(neg(carry1B), gpi1B, neg(gpj1A), gpj1B, gmk, gpk1B);
+                v1B = ldb(Vb, vB, kVComp);
+                kick_drift<kUnitMass>(F, a.M, a.dt, v1B, xcB, x1B);
             }
         }
-        sm.y[par][0][tid] = x1.x;
-        sm.y[par][1][tid] = x1.y;
-        sm.y[par][2][tid] = x1.z;
-        carry1 = gpi1;
-        xc1 = xn1;
-        __syncthreads();  // B: X_{t+1}(p) visible; V_t(p) slot free
+        {
+            double* y = sm.y[par][0];
+            y[yA] = x1A.x;
+            y[yA + kYComp] = x1A.y;
+            y[yA + 2 * kYComp] = x1A.z;
+            y[yB] = x1B.x;
+            y[yB + kYComp] = x1B.y;
+            y[yB + 2 * kYComp] = x1B.z;
+        }
+        // ---- S2 "+" springs of plane q = p-1 (its X_{t+1} is in the ring since iteration p-1)
+        const int q = p - 1;
+        const bool do2 = q >= ps0;        // q == ps0: only the +i spring (carry of plane pb)
+        const bool out2 = q >= pb;        // an output plane
+        Vec3 gpi2A{0.0, 0.0, 0.0}, gpi2B{0.0, 0.0, 0.0};
+        Vec3 gpj2A{0.0, 0.0, 0.0}, gpj2B{0.0, 0.0, 0.0}, gpk2A{0.0, 0.0, 0.0}, gpk2B{0.0, 0.0, 0.0};
+        Vec3 xqA{0.0, 0.0, 0.0}, xqB{0.0, 0.0, 0.0};
+        if (do2) {
+            const double* yq = sm.y[par ^ 1][0];
+            xqA = ldb(yq, yA, kYComp);
+            xqB = ldb(yq, yB, kYComp);
+            gpi2A = spring_force<kPosK>(xqA, x1A, a.K, a.L);
+            gpi2B = spring_force<kPosK>(xqB, x1B, a.K, a.L);
+            if (out2) {
+                gpk2A = spring_force<kPosK>(xqA, ldb(yq, yAk, kYComp), a.K, a.L);
+                gpk2B = spring_force<kPosK>(xqB, ldb(yq, yBk, kYComp), a.K, a.L);
+                gpj2A = spring_force<kPosK>(xqA, xqB, a.K, a.L);
+                gpj2B = spring_force<kPosK>(xqB, ldb(yq, yBj, kYComp), a.K, a.L);
+                sm.g2j[w][lane] = gpj2B;
+            }
+        }
+        const Vec3 up2A = shfl_up1(gpk2A), up2B = shfl_up1(gpk2B);
+        __syncthreads();  // #2: S2 springs and X_{t+1}(p) visible; V_t(p) slot free
         if (tid == 0 && upd1 && p + kVStages <= v_last) {
             fence_proxy_async();
             issue_v(p + kVStages);
         }
-        // ---- step t+1 on plane q = p-1, phase C: "+" springs inside R1
-        const int q = p - 1;
-        Vec3 gpi2{0.0, 0.0, 0.0}, gpj2{0.0, 0.0, 0.0}, gpk2{0.0, 0.0, 0.0};
-        const bool do_c = q >= pb - 1 && q >= 0;
-        const bool out2 = q >= pb && q < pe;
-        Vec3 x2c{0.0, 0.0, 0.0};
-        if (do_c) {
-            const double* yq = sm.y[q & 1][0];
-            const double* yp = sm.y[par][0];
-            x2c = Vec3{yq[tid], yq[tid + kYComp], yq[tid + 2 * kYComp]};
-            gpi2 = spring_force<kPosK>(x2c, Vec3{yp[tid], yp[tid + kYComp], yp[tid + 2 * kYComp]}, a.K, a.L);
-            if (out2) {
-                const int tk = lane < kTK - 1 ? tid + 1 : tid;
-                const int tj = w < kW - 1 ? tid + kTK : tid;
-                gpk2 = spring_force<kPosK>(x2c, Vec3{yq[tk], yq[tk + kYComp], yq[tk + 2 * kYComp]}, a.K, a.L);
-                gpj2 = spring_force<kPosK>(x2c, Vec3{yq[tj], yq[tj + kYComp], yq[tj + 2 * kYComp]}, a.K, a.L);
-                sm.gj2[par][w][lane] = gpj2;
+        // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q
+        if (out2) {
+            if (ownA) {
+                if (intA) {
+                    const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
+                    const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
+                    Vec3 v2 = v1pA, x2;
+                    kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
+                    double* xo = tp.x_out + (int64_t)q * ps + offA;
+                    double* vo = tp.v_out + (int64_t)(q - 1) * ps + offA;
+                    xo[0] = x2.x;
+                    xo[cs] = x2.y;
+                    xo[2 * cs] = x2.z;
+                    vo[0] = v2.x;
+                    vo[cs] = v2.y;
+                    vo[2 * cs] = v2.z;
+                    st.add_position(x2);
+                    st.add_velocity(v2);
+                } else {
+                    st.add_position(xqA);  // fixed face node
+                }
+            }
+            if (ownB) {
+                if (intB) {
+                    const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
+                    Vec3 v2 = v1pB, x2;
+                    kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
+                    double* xo = tp.x_out + (int64_t)q * ps + offB;
+                    double* vo = tp.v_out + (int64_t)(q - 1) * ps + offB;
+                    xo[0] = x2.x;
+                    xo[cs] = x2.y;
+                    xo[2 * cs] = x2.z;
+                    vo[0] = v2.x;
+                    vo[cs] = v2.y;
+                    vo[2 * cs] = v2.z;
+                    st.add_position(x2);
+                    st.add_velocity(v2);
+                } else {
+                    st.add_position(xqB);
+                }
             }
         }
-        const Vec3 up2 = shfl_up1(gpk2);
-        __syncthreads();  // C
-        // ---- step t+1, phase D: update R2 nodes of plane q, write X_{t+2}, V_{t+2}
-        if (out2 && owned) {
-            if (interior) {
-                const Vec3 gmj = neg(sm.gj2[par][w - 1][lane]);
-                const Vec3 F = sum_forces(neg(carry2), gpi2, gmj, gpj2, neg(up2), gpk2);
-                Vec3 v2 = vhold, x2;
-                kick_drift<kUnitMass>(F, a.M, a.dt, v2, x2c, x2);
-                double* xo = tp.x_out + (int64_t)q * ps + off;
-                double* vo = tp.v_out + (int64_t)(q - 1) * ps + off;
-                xo[0] = x2.x;
-                xo[cs] = x2.y;
-                xo[2 * cs] = x2.z;
-                vo[0] = v2.x;
-                vo[cs] = v2.y;
-                vo[2 * cs] = v2.z;
-                st2.add_position(x2);
-                st2.add_velocity(v2);
-            } else {
-                st2.add_position(x2c);  // fixed face node
-            }
-        }
-        if (do_c) carry2 = gpi2;
-        vhold = v1;
+        carry1A = gpi1A;
+        carry1B = gpi1B;
+        xcA = niA;
+        xcB = niB;
+        carry2A = gpi2A;
+        carry2B = gpi2B;
+        v1pA = v1A;
+        v1pB = v1B;
     }
-    block_accumulate(st1, sm.scratch, tp.acc1);
-    __syncthreads();
-    block_accumulate(st2, sm.scratch, a.acc);
+    block_accumulate(st, sm.scratch, a.acc);
 }
 
 }  // namespace
 
-cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, StatsAccum* acc1, bool unit_mass,
+cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, StatsAccum* /*acc1*/, bool unit_mass,
                           cudaStream_t stream) {
     if (a.g.size <= 0) return cudaSuccess;
     if (!a.tmap_x_cur || !a.tmap_v || a.lo_dst || a.hi_dst) return cudaErrorInvalidValue;
@@ -264,7 +321,6 @@ cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, Stats
     tp.a = a;
     tp.x_out = x_out;
     tp.v_out = v_out;
-    tp.acc1 = acc1;
     tp.tiles_k = (int)((a.g.n2 + kOK - 1) / kOK);
     tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;

@@ -27,6 +27,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <type_traits>
 
 #include "../kernels.hpp"
 #include "node_math.cuh"
@@ -147,11 +148,29 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int64_t cs = g.comp_stride(), ps = g.plane_stride();
     const int64_t offA = ownA ? (int64_t)jA * g.ld + k : 0, offB = ownB ? (int64_t)jB * g.ld + k : 0;
 
-    // prologue: X_t(ps0) own, and the step-t -i spring of plane ps0
+    // Tile-border springs of S1 (row above R1 -> R1 row 0: gbj; column left of
+    // R1 -> R1 lane 0: gbk) of plane p. They are computed one iteration ahead,
+    // after barrier #2, by the two warps whose S2 phase has a ring row and so
+    // one row less to update (warp 0: row 0, warp kW-1: row kRows-1) -- keeping
+    // the S1 spring phase before barrier #1 equal across warps. Written in
+    // phase C of iteration p-1 (or the prologue), read after barrier #1 of
+    // iteration p, rewritten after barrier #2 of iteration p.
+    auto border_springs = [&](int p) {
+        const double* Xb = xbox(p);
+        if (w == 0) {
+            sm.gbj[lane] = spring_force<kPosK>(ldb(Xb, lane + 1, kXComp), ldb(Xb, kBK + lane + 1, kXComp), a.K, a.L);
+        } else if (w == kW - 1 && lane < kRows) {
+            const int r = (lane + 1) * kBK;
+            sm.gbk[lane] = spring_force<kPosK>(ldb(Xb, r, kXComp), ldb(Xb, r + 1, kXComp), a.K, a.L);
+        }
+    };
+
+    // prologue: X_t(ps0) own, the step-t -i spring of plane ps0, border springs of ps0
     Vec3 carry1A{0.0, 0.0, 0.0}, carry1B{0.0, 0.0, 0.0};
     xwait(ps0);
     Vec3 xcA = ldb(xbox(ps0), xA, kXComp), xcB = ldb(xbox(ps0), xB, kXComp);
     if (ps0 >= 1) {
+        border_springs(ps0);  // ps0 <= size always
         xwait(ps0 - 1);
         carry1A = spring_force<kPosK>(ldb(xbox(ps0 - 1), xA, kXComp), xcA, a.K, a.L);
         carry1B = spring_force<kPosK>(ldb(xbox(ps0 - 1), xB, kXComp), xcB, a.K, a.L);
@@ -165,21 +184,28 @@ __global__ void __launch_bounds__(kThreads, 1)
     Vec3 v1pA{0.0, 0.0, 0.0}, v1pB{0.0, 0.0, 0.0};  // V_{t+1} of plane p-1
     NodeStats st;
     st.zero();
+    const int border_last = min(pe, size);  // planes whose border springs S1 needs
 
-    for (int p = ps0; p <= pe; p++) {
-        const int par = p & 1;
-        const bool upd1 = p >= 1 && p <= size;  // S1 updates plane p (else a fixed face plane)
-        const bool has_next = p + 1 <= qlast;
+    // One plane of the march. kFull: a steady-state plane (p+1 exists, p is
+    // updated by S1, q = p-1 is an S2 output plane): no conditions, no
+    // zero-initialised partial results. kPar: p & 1 when known (0/1), else -1.
+    auto body = [&](auto full_c, auto par_c, int p) {
+        constexpr bool kFull = decltype(full_c)::value;
+        constexpr int kPar = decltype(par_c)::value;
+        const int par = kPar >= 0 ? kPar : (p & 1);
+        const bool upd1 = kFull || (p >= 1 && p <= size);  // S1 updates plane p (else a fixed face plane)
+        const bool has_next = kFull || p + 1 <= qlast;
         if (has_next) xwait(p + 1);
         const double* Xc = xbox(p);
         const double* Xn = has_next ? xbox(p + 1) : Xc;
         // ---- S1 "+" springs of plane p
-        Vec3 gpi1A{0.0, 0.0, 0.0}, gpi1B{0.0, 0.0, 0.0};
-        Vec3 gpj1A{0.0, 0.0, 0.0}, gpj1B{0.0, 0.0, 0.0}, gpk1A{0.0, 0.0, 0.0}, gpk1B{0.0, 0.0, 0.0};
+        Vec3 gpi1A, gpi1B, gpj1A, gpj1B, gpk1A, gpk1B;
         const Vec3 niA = ldb(Xn, xA, kXComp), niB = ldb(Xn, xB, kXComp);
         if (has_next) {
             gpi1A = spring_force<kPosK>(xcA, niA, a.K, a.L);
             gpi1B = spring_force<kPosK>(xcB, niB, a.K, a.L);
+        } else {
+            gpi1A = gpi1B = Vec3{0.0, 0.0, 0.0};
         }
         if (upd1) {
             gpk1A = spring_force<kPosK>(xcA, ldb(Xc, xA + 1, kXComp), a.K, a.L);
@@ -187,13 +213,8 @@ __global__ void __launch_bounds__(kThreads, 1)
             gpj1A = spring_force<kPosK>(xcA, xcB, a.K, a.L);
             gpj1B = spring_force<kPosK>(xcB, ldb(Xc, xB + kBK, kXComp), a.K, a.L);
             sm.g1j[w][lane] = gpj1B;
-            if (w == 0) {
-                sm.gbj[lane] = spring_force<kPosK>(ldb(Xc, lane + 1, kXComp), ldb(Xc, kBK + lane + 1, kXComp), a.K,
-                                                   a.L);
-            } else if (w == 1 && lane < kRows) {
-                const int r = (lane + 1) * kBK;
-                sm.gbk[lane] = spring_force<kPosK>(ldb(Xc, r, kXComp), ldb(Xc, r + 1, kXComp), a.K, a.L);
-            }
+        } else {
+            gpk1A = gpk1B = gpj1A = gpj1B = Vec3{0.0, 0.0, 0.0};
         }
         const Vec3 up1A = shfl_up1(gpk1A), up1B = shfl_up1(gpk1B);
         __syncthreads();  // #1: S1 springs visible; X_t(p) read for the last time
@@ -232,11 +253,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         // ---- S2 "+" springs of plane q = p-1 (its X_{t+1} is in the ring since iteration p-1)
         const int q = p - 1;
-        const bool do2 = q >= ps0;        // q == ps0: only the +i spring (carry of plane pb)
-        const bool out2 = q >= pb;        // an output plane
-        Vec3 gpi2A{0.0, 0.0, 0.0}, gpi2B{0.0, 0.0, 0.0};
-        Vec3 gpj2A{0.0, 0.0, 0.0}, gpj2B{0.0, 0.0, 0.0}, gpk2A{0.0, 0.0, 0.0}, gpk2B{0.0, 0.0, 0.0};
-        Vec3 xqA{0.0, 0.0, 0.0}, xqB{0.0, 0.0, 0.0};
+        const bool do2 = kFull || q >= ps0;  // q == ps0: only the +i spring (carry of plane pb)
+        const bool out2 = kFull || q >= pb;  // an output plane
+        Vec3 gpi2A, gpi2B, gpj2A, gpj2B, gpk2A, gpk2B, xqA, xqB;
+        gpi2A = gpi2B = gpj2A = gpj2B = gpk2A = gpk2B = xqA = xqB = Vec3{0.0, 0.0, 0.0};
         if (do2) {
             const double* yq = sm.y[par ^ 1][0];
             xqA = ldb(yq, yA, kYComp);
@@ -252,7 +272,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
         }
         const Vec3 up2A = shfl_up1(gpk2A), up2B = shfl_up1(gpk2B);
-        __syncthreads();  // #2: S2 springs and X_{t+1}(p) visible; V_t(p) slot free
+        __syncthreads();  // #2: S2 springs and X_{t+1}(p) visible; V_t(p) slot free; gbj/gbk(p) consumed
         if (tid == 0 && upd1 && p + kVStages <= v_last) {
             fence_proxy_async();
             issue_v(p + kVStages);
@@ -299,6 +319,8 @@ __global__ void __launch_bounds__(kThreads, 1)
                 }
             }
         }
+        // border springs of the next plane (X_t(p+1) is resident until barrier #1 of iteration p+1)
+        if (p + 1 <= border_last) border_springs(p + 1);
         carry1A = gpi1A;
         carry1B = gpi1B;
         xcA = niA;
@@ -307,7 +329,23 @@ __global__ void __launch_bounds__(kThreads, 1)
         carry2B = gpi2B;
         v1pA = v1A;
         v1pB = v1B;
+    };
+    using F0 = std::integral_constant<bool, false>;
+    using F1 = std::integral_constant<bool, true>;
+    using PN = std::integral_constant<int, -1>;
+    using P0 = std::integral_constant<int, 0>;
+    using P1 = std::integral_constant<int, 1>;
+    // steady planes: p >= pb+1 (q = p-1 is an output plane, p > ps0), p <= min(size, pe) (updated, p+1 exists)
+    const int lo = pb + 1, hi = min(size, pe);
+    int p = ps0;
+    for (; p < lo && p <= pe; p++) body(F0{}, PN{}, p);
+    if (p <= hi && (p & 1)) body(F1{}, P1{}, p++);
+    for (; p + 1 <= hi; p += 2) {
+        body(F1{}, P0{}, p);
+        body(F1{}, P1{}, p + 1);
     }
+    if (p <= hi) body(F1{}, P0{}, p++);
+    for (; p <= pe; p++) body(F0{}, PN{}, p);
     block_accumulate(st, sm.scratch, a.acc);
 }
 

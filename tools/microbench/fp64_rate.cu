@@ -15,6 +15,24 @@ __global__ void dfma_k(double* out, int iters, double a, double b) {
   }
   out[blockIdx.x * blockDim.x + threadIdx.x] = x0+x1+x2+x3+x4+x5+x6+x7;
 }
+// DADD / DMUL chains (same issue pattern as dfma_k): is every fp64 opcode one pipe slot?
+template <int kOp>
+__global__ void dop_k(double* out, int iters, double a) {
+  double x0 = threadIdx.x * 1e-3, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3, x4=x0+4,x5=x0+5,x6=x0+6,x7=x0+7;
+  for (int i = 0; i < iters; i++) {
+#pragma unroll
+    for (int u = 0; u < 16; u++) {
+      if (kOp == 0) {
+        x0 = __dadd_rn(x0, a); x1 = __dadd_rn(x1, a); x2 = __dadd_rn(x2, a); x3 = __dadd_rn(x3, a);
+        x4 = __dadd_rn(x4, a); x5 = __dadd_rn(x5, a); x6 = __dadd_rn(x6, a); x7 = __dadd_rn(x7, a);
+      } else {
+        x0 = __dmul_rn(x0, a); x1 = __dmul_rn(x1, a); x2 = __dmul_rn(x2, a); x3 = __dmul_rn(x3, a);
+        x4 = __dmul_rn(x4, a); x5 = __dmul_rn(x5, a); x6 = __dmul_rn(x6, a); x7 = __dmul_rn(x7, a);
+      }
+    }
+  }
+  out[blockIdx.x * blockDim.x + threadIdx.x] = x0+x1+x2+x3+x4+x5+x6+x7;
+}
 __global__ void dsqrtdiv_k(double* out, int iters, double a) {
   double x0 = 1.0 + threadIdx.x * 1e-3, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3;
   for (int i = 0; i < iters; i++) {
@@ -40,6 +58,15 @@ int main() {
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     double ops = (double)blocks * threads * iters * 16 * 8;
     printf("DFMA: %.3f ms, %.3f Tinstr/s (%.2f per SM per clk @1965)\n", ms, ops / ms / 1e9, ops / (ms*1e-3) / 148 / 1.965e9);
+  }
+  for (int op = 0; op < 2; op++)
+  for (int rep = 0; rep < 3; rep++) {
+    cudaEventRecord(e0);
+    if (op == 0) dop_k<0><<<blocks, threads>>>(out, iters, 1e-9); else dop_k<1><<<blocks, threads>>>(out, iters, 0.9999999);
+    cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    double ops = (double)blocks * threads * iters * 16 * 8;
+    printf("%s: %.3f ms, %.3f Tinstr/s (%.2f per SM per clk @1965)\n", op ? "DMUL" : "DADD", ms, ops / ms / 1e9, ops / (ms*1e-3) / 148 / 1.965e9);
   }
   iters = 500;
   for (int rep = 0; rep < 3; rep++) {

@@ -36,7 +36,7 @@ def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=6)
     ap.add_argument("--grid", type=int, nargs="+", default=[512],
                     help="grid nodes (one value: cube); not --n, which torch.distributed.run would claim")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
@@ -68,6 +68,37 @@ def algorithmic_bytes(n, start, size):
     """Per K1 launch over one chunk: read X_t on the owned planes + 2 halo planes
     (24 B/node), read V, write V, write X_{t+1} on interior nodes (72 B/node)."""
     return 24 * (size + 2) * n[1] * n[2] + 72 * size * (n[1] - 2) * (n[2] - 2)
+
+
+def interior_of(n, size):
+    """Interior nodes of a chunk of `size` planes."""
+    return size * (n[1] - 2) * (n[2] - 2)
+
+
+# fp64 lane-instructions per node-update of node_math.cuh with each spring
+# evaluated once (DESIGN.md §6): 3 springs x 27 (3 sub, d^2 5, sqrt + 1/d 11,
+# d-L and K* 2, quotient 3, f*d 3) + force sum 15 + kick/drift 12 = 108, and the
+# fused stats 27 (3 x 7 exact-split centre terms, v.v 5, max 1) per step whose
+# stats are kept. K1_TB2 keeps only the second step's stats.
+FP64_OPS_STEP, FP64_OPS_STATS = 108, 27
+
+
+def fp64_ops_per_node_update(two_step):
+    if two_step:
+        return FP64_OPS_STEP + FP64_OPS_STATS / 2.0
+    return FP64_OPS_STEP + FP64_OPS_STATS
+
+
+def load_fp64_peak():
+    """fp64 pipe peak (lane-instructions/s): tools/microbench/fp64_rate (DFMA,
+    DADD, DMUL chains) measured on a B200 of this pool (profiles/fp64_rate.json),
+    else 148 SMs x 64 fp64 lanes x 1.965 GHz."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp64_rate.json")) as f:
+            d = json.load(f)
+        return float(d["fp64_tinstr_s"]), "measured (profiles/fp64_rate.json: %s)" % d.get("how", "")
+    except Exception:
+        return 148 * 64 * 1.965e9 / 1e12, "derived: 148 SMs x 64 fp64 lanes/clk x 1.965 GHz"
 
 
 def load_peaks():
@@ -378,7 +409,10 @@ def run_ours(a):
         if multi:
             torch.distributed.barrier()
 
-    # warm-up
+    # warm-up (K1_TB2 runs steps in pairs: an odd W gets one more step so that
+    # the timed region starts on an even step; "warmup" reports the steps done)
+    if s.kernel_in_use == P.K1_TB2 and a.warmup % 2:
+        a.warmup += 1
     with torch.cuda.stream(stream):
         s.step(a.warmup)
     s.sync()
@@ -387,10 +421,12 @@ def run_ours(a):
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.5)
-    # K1_TB2 advances two steps per launch: time launches of 2 steps (K even)
-    per_call = 2 if (kernel == P.K1_TB2 and not multi and a.chunk == 0) else 1
+    # K1_TB2 (AUTO on one chunk) advances two steps per launch: K even, so every
+    # timed launch is a two-step launch
+    in_use = s.kernel_in_use
+    per_call = 2 if in_use == P.K1_TB2 else 1
     if a.steps % per_call:
-        raise SystemExit("--kernel tb2 needs an even --steps")
+        raise SystemExit("K1_TB2 runs steps in pairs: --steps must be even")
     l0 = s.launches
     barrier()
     t_start = torch.cuda.Event(enable_timing=True)
@@ -436,8 +472,12 @@ def run_ours(a):
     alg = algorithmic_bytes(n, c0.start, c0.size)
     peak, peak_src = load_peaks()
     achieved = alg / (k1_ms * 1e-3) / 1e9
-    kname = {P.K1_AUTO: "march2", P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct",
-             P.K1_TB2: "tb2"}[kernel]
+    kname = {P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct", P.K1_TB2: "tb2"}[in_use]
+    # the same launches against the fp64 pipe: the method's fp64 instructions
+    # per node-update (FP64_OPS_* below) x node-updates per launch
+    fp64_alg = interior_of(n, c0.size) * per_call * fp64_ops_per_node_update(per_call == 2)
+    fp64_peak, fp64_src = load_fp64_peak()
+    fp64_achieved = fp64_alg / (k1_ms * 1e-3) / 1e12
     traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()
@@ -514,7 +554,18 @@ def run_ours(a):
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "k1_%s_kernel" % kname, "algorithmic_bytes_per_launch": alg,
                          "avg_launch_ms": k1_ms, "launch_ms_distribution": step_dist,
-                         "sustained_copy_gbs": copy_gbs},
+                         "sustained_copy_gbs": copy_gbs, "steps_per_launch": per_call,
+                         "one_step_equivalent_gbs": alg * per_call / (k1_ms * 1e-3) / 1e9,
+                         "note": ("K1_TB2 advances two steps per pass over HBM: 'achieved' counts the bytes a launch "
+                                  "must move (one pass); one_step_equivalent_gbs is the rate the one-step method "
+                                  "would need for the same node-updates/s" if per_call == 2 else
+                                  "one step per launch")},
+            "roofline_fp64": {"bound": "alu", "achieved": fp64_achieved, "peak": fp64_peak, "unit": "Tinstr/s",
+                              "frac": fp64_achieved / fp64_peak, "peak_source": fp64_src,
+                              "alg_instr_per_launch": fp64_alg,
+                              "alg_instr_per_node_update": fp64_ops_per_node_update(per_call == 2),
+                              "note": "fp64 lane-instructions of node_math.cuh per node-update with spring reuse "
+                                      "(DESIGN.md §6); recomputed ring / tile padding not counted"},
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
             "halo": halo_info(n, spread.chunks(), world),
             "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},

@@ -49,7 +49,9 @@ extern "C" {
 
 /* K1 implementations (all compute bit-identical results). */
 typedef enum {
-    SOMIER_K1_AUTO = 0,      /* the fastest available (currently SOMIER_K1_MARCH2)    */
+    SOMIER_K1_AUTO = 0,      /* the fastest available: SOMIER_K1_TB2 for a handle with
+                                one local chunk whose device has room for it, else
+                                SOMIER_K1_MARCH2 (somier_kernel_in_use tells which)   */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
     SOMIER_K1_MARCH = 2,     /* plane-marching, smem-staged, 3 springs/node with reuse */
     SOMIER_K1_MARCH2 = 3,    /* as MARCH with two rows per warp (32 x 16 tiles)        */
@@ -196,6 +198,12 @@ spread_status somier_step_count(somier_t h, int64_t* steps);
 /* Number of chunks this handle owns, and K1 launches enqueued so far. */
 spread_status somier_local_chunks(somier_t h, int64_t* nchunks);
 spread_status somier_launch_count(somier_t h, int64_t* launches);
+
+/* The K1 implementation multi-step calls of this handle run (a somier_kernel
+ * value; never SOMIER_K1_AUTO): AUTO and TB2 resolve at somier_init. A handle
+ * on K1_TB2 still runs a single step (odd step count or odd start) with
+ * K1_MARCH2. EINVAL on NULL arguments. */
+spread_status somier_kernel_in_use(somier_t h, int32_t* kernel);
 
 /* Device bytes this handle allocated (all devices). */
 spread_status somier_device_bytes(somier_t h, int64_t* bytes);

@@ -105,6 +105,7 @@ SIGNATURES = [
     ("somier_local_chunks", ctypes.c_int, [_VP, _I64P]),
     ("somier_launch_count", ctypes.c_int, [_VP, _I64P]),
     ("somier_device_bytes", ctypes.c_int, [_VP, _I64P]),
+    ("somier_kernel_in_use", ctypes.c_int, [_VP, ctypes.POINTER(ctypes.c_int32)]),
     ("somier_destroy", ctypes.c_int, [_VP]),
     ("somier_version", ctypes.c_char_p, []),
     ("somier_stream_create", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.c_int, ctypes.POINTER(_VP)]),

@@ -373,8 +373,23 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         ch.device = h->devs[ci.pos].device;
         ch.local = (local_pos < 0) || (ci.pos == local_pos);
     }
-    // K1_TB2 (two steps per launch) needs one local chunk without neighbours
-    h->tb2 = p->kernel == SOMIER_K1_TB2 && local_pos < 0 && s->nchunks == 1;
+    // K1_TB2 (two steps per launch) needs one local chunk without neighbours.
+    // AUTO takes it there (measured fastest) when the device has
+    // room for its second V buffer (96 instead of 72 B/node), else K1_MARCH2.
+    h->tb2 = false;
+    if ((p->kernel == SOMIER_K1_TB2 || p->kernel == SOMIER_K1_AUTO) && local_pos < 0 && s->nchunks == 1) {
+        h->tb2 = true;
+        if (p->kernel == SOMIER_K1_AUTO) {
+            const Chunk& c = h->chunks[0];
+            const size_t plane = (size_t)3 * (size_t)p->n[1] * (size_t)h->ld * sizeof(double);
+            const size_t need = 2 * plane * (size_t)(c.size + 2) + 2 * plane * (size_t)c.size;
+            size_t free_b = 0, total_b = 0;
+            if (cudaSetDevice(c.device) != cudaSuccess || cudaMemGetInfo(&free_b, &total_b) != cudaSuccess ||
+                free_b < need + ((size_t)1 << 30))
+                h->tb2 = false;
+            cudaGetLastError();
+        }
+    }
     st = load_driver_entry(h);
     if (st != SPREAD_OK) {
         delete h;
@@ -1010,6 +1025,20 @@ spread_status somier_local_chunks(somier_t h, int64_t* nchunks) {
 spread_status somier_launch_count(somier_t h, int64_t* launches) {
     if (!h || !launches) PAPER_FAIL(SPREAD_EINVAL, "somier_launch_count: NULL argument");
     *launches = h->launches;
+    return SPREAD_OK;
+}
+
+spread_status somier_kernel_in_use(somier_t h, int32_t* kernel) {
+    if (!h || !kernel) PAPER_FAIL(SPREAD_EINVAL, "somier_kernel_in_use: NULL argument");
+    if (h->tb2) {
+        *kernel = SOMIER_K1_TB2;
+        return SPREAD_OK;
+    }
+    switch (h->variant()) {
+        case paper::K1Variant::Direct: *kernel = SOMIER_K1_DIRECT; break;
+        case paper::K1Variant::March: *kernel = SOMIER_K1_MARCH; break;
+        default: *kernel = SOMIER_K1_MARCH2; break;
+    }
     return SPREAD_OK;
 }
 

@@ -225,6 +225,13 @@ class Somier:
     def device_bytes(self) -> int:
         return self._i64(N.lib().somier_device_bytes, "somier_device_bytes")
 
+    @property
+    def kernel_in_use(self) -> int:
+        """The K1 implementation multi-step calls run (K1_TB2 / K1_MARCH2 / ...)."""
+        v = ctypes.c_int32()
+        N.check(N.lib().somier_kernel_in_use(self._h, ctypes.byref(v)), "somier_kernel_in_use")
+        return v.value
+
 
 class SomierStream:
     """Host-streamed Somier (include/somier.h, somier_stream_*): the state lives

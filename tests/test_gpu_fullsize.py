@@ -22,7 +22,9 @@ def _need_gpu():
 
 def _samples(n, rng, count):
     out = [(1, 1, 1), (n[0] - 2, n[1] - 2, n[2] - 2), (n[0] // 2, 1, n[2] - 2), (1, n[1] // 2, n[2] // 2),
-           (n[0] // 2, n[1] // 2, 31), (n[0] // 2, 15, 32), (65, 16, 33), (64, 17, 96)]
+           (n[0] // 2, n[1] // 2, 31), (n[0] // 2, 15, 32), (65, 16, 33), (64, 17, 96),
+           # K1_TB2 tile / segment borders (owned tiles 30 x 22 from k, j = 0; segments of 64 planes from i = 1)
+           (65, 22, 30), (64, 21, 29), (129, 44, 60), (n[0] - 2, n[1] - 2, 30)]
     while len(out) < count:
         out.append(tuple(int(rng.integers(1, n[d] - 1)) for d in range(3)))
     return out
@@ -51,8 +53,13 @@ def _check_nodes(n, steps, count, seed=42, kernel=P.K1_AUTO):
 
 
 def test_512cube_bench_config_sampled_nodes_bitwise():
-    """configs[3] (the bench workload): 512^3, 24 steps, 16 nodes."""
+    """configs[3] (the bench workload, K1 AUTO = K1_TB2): 512^3, 24 steps, 16 nodes."""
     _check_nodes((512, 512, 512), 24, 16)
+
+
+def test_512cube_march2_kernel_sampled_nodes_bitwise():
+    """The one-step kernel multi-chunk / multi-GPU runs use, at the bench size."""
+    _check_nodes((512, 512, 512), 24, 12, kernel=P.K1_MARCH2)
 
 
 def test_512cube_march_kernel_sampled_nodes_bitwise():

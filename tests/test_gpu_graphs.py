@@ -22,7 +22,7 @@ def _need_gpu():
 @pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7)])
 @pytest.mark.parametrize("chunk", [0, 4])
 def test_graph_splits_bitwise(splits, chunk):
-    sp = P.SomierParams(n=(12, 10, 36), seed=3)
+    sp = P.SomierParams(n=(12, 10, 36), seed=3, kernel=P.K1_MARCH2)  # graphs replay one-step kernels
     with P.Somier(P.Spread([0], 1, 10, chunk=chunk), sp) as s:
         for k in splits:
             s.step(k)
@@ -35,7 +35,7 @@ def test_graph_splits_bitwise(splits, chunk):
 
 
 def test_eager_and_graph_identical(monkeypatch):
-    sp = P.SomierParams(n=(16, 16, 40), seed=9)
+    sp = P.SomierParams(n=(16, 16, 40), seed=9, kernel=P.K1_MARCH2)
     outs = []
     for env in ("0", "1"):
         monkeypatch.setenv("SOMIER_NO_GRAPH", env)
@@ -43,3 +43,44 @@ def test_eager_and_graph_identical(monkeypatch):
             s.step(20)
             outs.append(s.read())
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+def _tb2_launches(splits):
+    """K1_TB2 launch rule (somier_step): an odd start runs one single step,
+    then pairs, then a leftover single step."""
+    step = launches = 0
+    for k in splits:
+        if step % 2 and k:
+            launches, step, k = launches + 1, step + 1, k - 1
+        launches += k // 2 + k % 2
+        step += k
+    return launches
+
+
+@pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7), (1, 12)])
+@pytest.mark.parametrize("kernel", [P.K1_AUTO, P.K1_TB2])
+def test_tb2_splits_bitwise(splits, kernel):
+    """AUTO on a single-chunk handle is K1_TB2 (two steps per launch); any split
+    of the step count, on either parity, gives the oracle's bits, stats
+    included."""
+    sp = P.SomierParams(n=(12, 10, 36), seed=3, kernel=kernel)
+    with P.Somier(P.Spread([0], 1, 10), sp) as s:
+        assert s.kernel_in_use == P.K1_TB2
+        for k in splits:
+            s.step(k)
+            st = s.stats()
+            ref, rst = O.run(O.init(O.Params(n=sp.n, seed=3)), s.step_count)
+            assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits, (splits, k)
+        X, V = s.read()
+        assert s.launches == _tb2_launches(splits)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+
+
+def test_auto_kernel_resolution():
+    sp = P.SomierParams(n=(12, 10, 36), seed=3)
+    with P.Somier(P.Spread([0], 1, 10), sp) as s:
+        assert s.kernel_in_use == P.K1_TB2
+    with P.Somier(P.Spread([0], 1, 10, chunk=4), sp) as s:
+        assert s.kernel_in_use == P.K1_MARCH2  # several chunks: one-step kernel with the fused exchange
+    with P.Somier(P.Spread([0], 1, 10), P.SomierParams(n=(12, 10, 36), kernel=P.K1_MARCH)) as s:
+        assert s.kernel_in_use == P.K1_MARCH

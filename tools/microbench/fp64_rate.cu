@@ -53,11 +53,13 @@ int main() {
   double* out; CK(cudaMalloc(&out, 148*64*1024*sizeof(double)));
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   int blocks = p.multiProcessorCount * 8, threads = 256, iters = 2000;
+  double best[3] = {0, 0, 0};  // DFMA, DADD, DMUL lane-instructions/s
   for (int rep = 0; rep < 3; rep++) {
     cudaEventRecord(e0); dfma_k<<<blocks, threads>>>(out, iters, 0.999999, 1e-7); cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     double ops = (double)blocks * threads * iters * 16 * 8;
     printf("DFMA: %.3f ms, %.3f Tinstr/s (%.2f per SM per clk @1965)\n", ms, ops / ms / 1e9, ops / (ms*1e-3) / 148 / 1.965e9);
+    if (ops / ms / 1e9 > best[0]) best[0] = ops / ms / 1e9;
   }
   for (int op = 0; op < 2; op++)
   for (int rep = 0; rep < 3; rep++) {
@@ -67,6 +69,7 @@ int main() {
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     double ops = (double)blocks * threads * iters * 16 * 8;
     printf("%s: %.3f ms, %.3f Tinstr/s (%.2f per SM per clk @1965)\n", op ? "DMUL" : "DADD", ms, ops / ms / 1e9, ops / (ms*1e-3) / 148 / 1.965e9);
+    if (ops / ms / 1e9 > best[1 + op]) best[1 + op] = ops / ms / 1e9;
   }
   iters = 500;
   for (int rep = 0; rep < 3; rep++) {
@@ -82,5 +85,9 @@ int main() {
     float ms; cudaEventElapsedTime(&ms, e0, e1);
     printf("copy: %.3f ms %.1f GB/s\n", ms, 2.0 * n * 16 / ms / 1e6);
   }
+  const double peak = best[0] > best[1] ? (best[0] > best[2] ? best[0] : best[2]) : (best[1] > best[2] ? best[1] : best[2]);
+  printf("{\"fp64_tinstr_s\": %.4f, \"dfma_tinstr_s\": %.4f, \"dadd_tinstr_s\": %.4f, \"dmul_tinstr_s\": %.4f, "
+         "\"how\": \"tools/microbench/fp64_rate: 8 independent chains per thread, 1184 x 256 threads, best of 3 per opcode; "
+         "peak = the fastest opcode\"}\n", peak, best[0], best[1], best[2]);
   return 0;
 }

@@ -1,7 +1,7 @@
 #!/usr/bin/env python3
 """Small runs of every kernel path for compute-sanitizer (tests/test_gpu_sanitizer.py):
 K1 direct / march / march2 over a multi-chunk spread (fused halo stores), the
-host-streamed mode, K2 and K3."""
+host-streamed mode, K2 and K3, and K1_TB2 on a single chunk."""
 import os
 import sys
 
@@ -24,4 +24,14 @@ for kern in (P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2):
         X, V = st.generate()
         XN = np.zeros_like(X)
         st.step(X, V, XN)
+# K1_TB2 (AUTO on a single chunk): two steps per launch, shared-memory rings and
+# the one-plane-ahead border springs; odd step counts take the one-step path too
+for kern in (P.K1_AUTO, P.K1_TB2):
+    sp = P.SomierParams(n=n, seed=3, kernel=kern)
+    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
+        assert s.kernel_in_use == P.K1_TB2
+        s.step(5)
+        s.stats()
+        s.step(2)
+        s.sync()
 print("sanitize case ok")

@@ -49,9 +49,10 @@ extern "C" {
 
 /* K1 implementations (all compute bit-identical results). */
 typedef enum {
-    SOMIER_K1_AUTO = 0,      /* the fastest available: SOMIER_K1_TB2 for a handle with
-                                one local chunk whose device has room for it, else
-                                SOMIER_K1_MARCH2 (somier_kernel_in_use tells which)   */
+    SOMIER_K1_AUTO = 0,      /* the fastest measured: SOMIER_K1_TB2 for a handle with
+                                one local chunk of a grid of >= 6e6 nodes whose device
+                                has room for it, else SOMIER_K1_MARCH2
+                                (somier_kernel_in_use tells which)                    */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
     SOMIER_K1_MARCH = 2,     /* plane-marching, smem-staged, 3 springs/node with reuse */
     SOMIER_K1_MARCH2 = 3,    /* as MARCH with two rows per warp (32 x 16 tiles)        */

@@ -374,12 +374,15 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         ch.local = (local_pos < 0) || (ci.pos == local_pos);
     }
     // K1_TB2 (two steps per launch) needs one local chunk without neighbours.
-    // AUTO takes it there (measured fastest) when the device has
-    // room for its second V buffer (96 instead of 72 B/node), else K1_MARCH2.
+    // AUTO takes it there for grids of >= kTb2AutoMinNodes nodes (measured: TB2
+    // +7..13% from 192^3 up, -19% at 128^3 where its 1-CTA/SM tiles fill few
+    // waves) when the device has room for its second V buffer
+    // (96 instead of 72 B/node), else K1_MARCH2.
+    constexpr double kTb2AutoMinNodes = 6.0e6;
     h->tb2 = false;
     if ((p->kernel == SOMIER_K1_TB2 || p->kernel == SOMIER_K1_AUTO) && local_pos < 0 && s->nchunks == 1) {
-        h->tb2 = true;
-        if (p->kernel == SOMIER_K1_AUTO) {
+        h->tb2 = p->kernel == SOMIER_K1_TB2 || (double)p->n[0] * (double)p->n[1] * (double)p->n[2] >= kTb2AutoMinNodes;
+        if (h->tb2 && p->kernel == SOMIER_K1_AUTO) {
             const Chunk& c = h->chunks[0];
             const size_t plane = (size_t)3 * (size_t)p->n[1] * (size_t)h->ld * sizeof(double);
             const size_t need = 2 * plane * (size_t)(c.size + 2) + 2 * plane * (size_t)c.size;

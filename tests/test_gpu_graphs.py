@@ -58,12 +58,11 @@ def _tb2_launches(splits):
 
 
 @pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7), (1, 12)])
-@pytest.mark.parametrize("kernel", [P.K1_AUTO, P.K1_TB2])
-def test_tb2_splits_bitwise(splits, kernel):
-    """AUTO on a single-chunk handle is K1_TB2 (two steps per launch); any split
+def test_tb2_splits_bitwise(splits):
+    """K1_TB2 (two steps per launch, AUTO on large single-chunk grids): any split
     of the step count, on either parity, gives the oracle's bits, stats
     included."""
-    sp = P.SomierParams(n=(12, 10, 36), seed=3, kernel=kernel)
+    sp = P.SomierParams(n=(12, 10, 36), seed=3, kernel=P.K1_TB2)
     with P.Somier(P.Spread([0], 1, 10), sp) as s:
         assert s.kernel_in_use == P.K1_TB2
         for k in splits:
@@ -77,10 +76,13 @@ def test_tb2_splits_bitwise(splits, kernel):
 
 
 def test_auto_kernel_resolution():
+    big = P.SomierParams(n=(200, 200, 200), seed=3)  # 8e6 nodes: K1_TB2's range
+    with P.Somier(P.Spread([0], 1, 198), big) as s:
+        assert s.kernel_in_use == P.K1_TB2
+    with P.Somier(P.Spread([0], 1, 198, chunk=99), big) as s:
+        assert s.kernel_in_use == P.K1_MARCH2  # several chunks: one-step kernel with the fused exchange
     sp = P.SomierParams(n=(12, 10, 36), seed=3)
     with P.Somier(P.Spread([0], 1, 10), sp) as s:
-        assert s.kernel_in_use == P.K1_TB2
-    with P.Somier(P.Spread([0], 1, 10, chunk=4), sp) as s:
-        assert s.kernel_in_use == P.K1_MARCH2  # several chunks: one-step kernel with the fused exchange
+        assert s.kernel_in_use == P.K1_MARCH2  # small grid: TB2's tiles fill too few waves
     with P.Somier(P.Spread([0], 1, 10), P.SomierParams(n=(12, 10, 36), kernel=P.K1_MARCH)) as s:
         assert s.kernel_in_use == P.K1_MARCH

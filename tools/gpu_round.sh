@@ -10,6 +10,6 @@ timeout 600 python bench.py > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=
 if [ "${SKIP_NCU:-0}" != "1" ]; then
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv --log-file $OUT/launches.csv \
     python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_list_bench.log 2>&1; echo "ncu list rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k1_ -s 4 -c 2 -o $OUT/k1_full \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k1_ -s 2 -c 1 -o $OUT/k1_full \
     python bench.py --steps 6 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
 fi

@@ -24,9 +24,9 @@ for kern in (P.K1_DIRECT, P.K1_MARCH, P.K1_MARCH2):
         X, V = st.generate()
         XN = np.zeros_like(X)
         st.step(X, V, XN)
-# K1_TB2 (AUTO on a single chunk): two steps per launch, shared-memory rings and
+# K1_TB2 (AUTO on a large single chunk): two steps per launch, shared-memory rings and
 # the one-plane-ahead border springs; odd step counts take the one-step path too
-for kern in (P.K1_AUTO, P.K1_TB2):
+for kern in (P.K1_TB2,):
     sp = P.SomierParams(n=n, seed=3, kernel=kern)
     with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
         assert s.kernel_in_use == P.K1_TB2

@@ -243,14 +243,15 @@ def run_reference(a):
 
 # --------------------------------------------------------------------------- our arm
 
-def halo_info(n, chunks, world):
+def halo_info(n, chunks, world, two_step=False):
     """Halo traffic of the fused exchange: each chunk boundary between list
     positions moves one X plane (24 B per node of the n1 x n2 cross-section)
     each way per step, stored by K1 straight into the neighbour's halo slot
-    (NVLink P2P / IPC). Reported against the measured 770 GB/s peer rate
-    (B200_PROFILING.md); the stores overlap the step, so this is a bound on
-    the exchange's cost, not a separate phase."""
-    plane = 24 * n[1] * n[2]
+    (NVLink P2P / IPC); K1_TB2 moves two X planes and one V plane each way per
+    two-step launch (36 B per cross-section node per step). Reported against
+    the measured 770 GB/s peer rate (B200_PROFILING.md); the stores overlap the
+    step, so this is a bound on the exchange's cost, not a separate phase."""
+    plane = (36 if two_step else 24) * n[1] * n[2]
     cross = sum(1 for a, b in zip(chunks, chunks[1:]) if a.device_pos != b.device_pos)
     total = 2 * cross * plane
     per_rank = total / max(1, world)
@@ -567,7 +568,7 @@ def run_ours(a):
                               "note": "fp64 lane-instructions of node_math.cuh per node-update with spring reuse "
                                       "(DESIGN.md §6); recomputed ring / tile padding not counted"},
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
-            "halo": halo_info(n, spread.chunks(), world),
+            "halo": halo_info(n, spread.chunks(), world, per_call == 2),
             "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},
         }
         print(json.dumps(line), flush=True)

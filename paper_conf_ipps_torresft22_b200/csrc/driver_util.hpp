@@ -32,7 +32,7 @@ spread_status encode_slab_tmap(CUtensorMap* map, const SlabGeom& g, double* base
 constexpr uint32_t kXBoxK = 36, kXBoxJ = 10, kVBoxK = 32, kVBoxJ = 8;
 // ... and K1_MARCH2 (two rows per warp, 32 x 16 tiles)
 constexpr uint32_t kX2BoxJ = 18, kV2BoxJ = 16;
-// ... and K1_TB2 (owned 30 x 14 tiles, ring-extended 32 x 16)
+// ... and K1_TB2 (owned 30 x 22 tiles, ring-extended 32 x 24, boxes with a one-node ring)
 constexpr uint32_t kTB2XBoxK = 34, kTB2XBoxJ = 2 * kTB2Warps + 2, kTB2VBoxK = 34, kTB2VBoxJ = 2 * kTB2Warps;
 
 // somier_params.kernel -> K1 implementation (AUTO = the fastest measured)
@@ -41,7 +41,7 @@ inline K1Variant k1_variant(int32_t kernel) {
         case SOMIER_K1_DIRECT: return K1Variant::Direct;
         case SOMIER_K1_MARCH: return K1Variant::March;
         case SOMIER_K1_MARCH2: return K1Variant::March2;
-        case SOMIER_K1_TB2: return K1Variant::March2;  // single steps of a TB2 handle
+        case SOMIER_K1_TB2: return K1Variant::March2;  // TB2 impossible (a chunk of one plane among several)
         default: return K1Variant::March2;  // measured fastest at 512^3
     }
 }

@@ -77,10 +77,26 @@ enum class K1Variant { Direct = 1, March = 2, March2 = 3 };
 constexpr int kTB2Warps = TB2_WARPS;
 
 cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cudaStream_t stream);
-// K1_TB2: two steps in one launch (a.x_cur / a.v / tmaps with the TB2 box
-// shapes -> x_out / v_out; stats of the first step into acc1, second into a.acc)
-cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, StatsAccum* acc1, bool unit_mass,
-                          cudaStream_t stream);
+
+// K1_TB2 slab layout (deep halo): X slabs hold planes [start-2, start+size+2)
+// (two halo planes per face), V slabs [start-1, start+size+1) (one), both
+// double-buffered; the launch reads X_t, V_t through a.tmap_x_cur / a.tmap_v
+// (box shapes kTB2*Box*) and writes the owned planes of X_{t+2}, V_{t+2} (one
+// step: X_{t+1}, V_{t+1}) to x_out / v_out, plus the first two X planes and
+// the first V plane to the left neighbour's halo (a.lo_dst = ITS out-buffer X
+// plane of global i = start, lo_vdst = its V plane of i = start) and the last
+// two / last one to the right neighbour's (a.hi_dst = its X plane of i =
+// start+size-2, hi_vdst = its V plane of i = start+size-1); a.signal_* /
+// a.done_counter / a.signal_value as for the one-step kernels. Stats of the
+// last step only, into a.acc.
+struct Tb2Out {
+    double* x_out;
+    double* v_out;
+    double* lo_vdst;
+    double* hi_vdst;
+    bool two;  // two steps (else one)
+};
+cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
 // Stats of planes [p0, p0+np) of an X slab (plane index inside the slab) and,
 // if v != null, of V planes [p0-1, ...) (V has no halo planes).

@@ -27,10 +27,12 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <climits>
 #include <type_traits>
 
 #include "../kernels.hpp"
 #include "node_math.cuh"
+#include "signal.cuh"
 #include "stats.cuh"
 #include "tma.cuh"
 
@@ -74,9 +76,14 @@ struct __align__(16) Smem {
 };
 
 struct Tb2Params {
-    StepArgs a;
-    double* x_out;                 // X_{t+2} buffer
-    double* v_out;                 // V_{t+2} buffer
+    StepArgs a;                    // a.x_cur / a.v: X_t, V_t slabs (through the tensor maps); a.lo_dst /
+                                   // a.hi_dst: the neighbours' X halo planes (see below)
+    double* x_out;                 // X_{t+2} (X_{t+1} in one-step mode) buffer, raw slab
+    double* v_out;                 // V_{t+2} buffer, raw slab
+    double* lo_vdst;               // left neighbour's V halo plane in ITS out buffer, or null
+    double* hi_vdst;               // right neighbour's V halo plane in ITS out buffer, or null
+    int x_base, v_base;            // global i of raw plane 0 of the X / V slabs (start - 2, start - 1)
+    int lo_end, hi_begin;          // planes q < lo_end go to lo_dst + (q - start), q >= hi_begin to hi_dst + (q - hi_begin)
     int tiles_k, tiles_j, seg_planes;
 };
 
@@ -85,11 +92,19 @@ __device__ __forceinline__ Vec3 shfl_up1(const Vec3& v) {
                 __shfl_up_sync(0xffffffffu, v.z, 1)};
 }
 
+__device__ __forceinline__ void stb3(double* p, int64_t cs, const Vec3& v) {
+    p[0] = v.x;
+    p[cs] = v.y;
+    p[2 * cs] = v.z;
+}
+
 __device__ __forceinline__ Vec3 ldb(const double* b, int off, int comp) {
     return Vec3{b[off], b[off + comp], b[off + 2 * comp]};
 }
 
-template <bool kUnitMass, bool kPosK>
+// kTwo: two steps per launch (else one: S1 only, its X_{t+1}, V_{t+1} written
+// for R2 -- the odd step of a TB2 handle, with the same halo layout).
+template <bool kUnitMass, bool kPosK, bool kTwo>
 __global__ void __launch_bounds__(kThreads, 1)
     k1_tb2_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                   const Tb2Params tp) {
@@ -102,23 +117,25 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int kq = tile_k * kOK, jq = tile_j * kOJ;  // owned tile origin (kq even: TMA inner coordinate)
     const int rA = 2 * w, rB = rA + 1;               // R1 rows of this thread
     const int k = kq - 1 + lane, jA = jq - 1 + rA, jB = jA + 1;
-    const int size = (int)g.size;
-    const int pb = 1 + blockIdx.y * tp.seg_planes;
-    const int pe = min(size + 1, pb + tp.seg_planes);  // S2 (step t+1) output planes [pb, pe)
-    const int ps0 = pb - 1;                            // S1 (step t) planes [ps0, pe]
-    const int q0 = max(0, ps0 - 1);                    // X_t planes [q0, qlast]
-    const int qlast = min(size + 1, pe + 1);
-    const int v_first = max(1, ps0), v_last = min(size, pe);  // V_t planes read (S1 on non-fixed planes)
+    // planes are global i; the chunk owns [start, start + size), its X slab
+    // holds [start - 2, start + size + 2), its V slab [start - 1, start + size + 1)
+    const int start = (int)g.start, size = (int)g.size, ilast = (int)g.n0 - 2;  // updated planes: [1, ilast]
+    const int pb = start + blockIdx.y * tp.seg_planes;
+    const int pe = min(start + size, pb + tp.seg_planes);  // S2 (step t+1) output planes [pb, pe)
+    const int ps0 = pb - 1;                                // S1 (step t) planes [ps0, pe]
+    const int q0 = max(0, ps0 - 1);                        // X_t planes [q0, qlast]
+    const int qlast = min(ilast + 1, pe + 1);
+    const int v_first = max(1, ps0), v_last = min(ilast, pe);  // V_t planes read (S1 on non-fixed planes)
 
     auto issue_x = [&](int q) {
         const int s = (q - q0) % kStages;
         mbar_expect_tx(&sm.full[s], kXBoxBytes);
-        tma_load_4d(sm.xst[s], &tmap_x, kq - 2, jq - 2, 0, q, &sm.full[s]);
+        tma_load_4d(sm.xst[s], &tmap_x, kq - 2, jq - 2, 0, q - tp.x_base, &sm.full[s]);
     };
-    auto issue_v = [&](int p) {  // V_t of slab plane p (V slab plane p-1)
+    auto issue_v = [&](int p) {  // V_t of plane p
         const int s = (p - v_first) % kVStages;
         mbar_expect_tx(&sm.vfull[s], kVBoxBytes);
-        tma_load_4d(sm.vst[s], &tmap_v, kq - 2, jq - 1, 0, p - 1, &sm.vfull[s]);
+        tma_load_4d(sm.vst[s], &tmap_v, kq - 2, jq - 1, 0, p - tp.v_base, &sm.vfull[s]);
     };
     if (tid == 0) {
         prefetch_tmap(&tmap_x);
@@ -170,7 +187,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     xwait(ps0);
     Vec3 xcA = ldb(xbox(ps0), xA, kXComp), xcB = ldb(xbox(ps0), xB, kXComp);
     if (ps0 >= 1) {
-        border_springs(ps0);  // ps0 <= size always
+        border_springs(ps0);  // ps0 <= ilast always
         xwait(ps0 - 1);
         carry1A = spring_force<kPosK>(ldb(xbox(ps0 - 1), xA, kXComp), xcA, a.K, a.L);
         carry1B = spring_force<kPosK>(ldb(xbox(ps0 - 1), xB, kXComp), xcB, a.K, a.L);
@@ -184,7 +201,21 @@ __global__ void __launch_bounds__(kThreads, 1)
     Vec3 v1pA{0.0, 0.0, 0.0}, v1pB{0.0, 0.0, 0.0};  // V_{t+1} of plane p-1
     NodeStats st;
     st.zero();
-    const int border_last = min(pe, size);  // planes whose border springs S1 needs
+    const int border_last = min(pe, ilast);  // planes whose border springs S1 needs
+    // X_{t+2} (X_{t+1}), V of an S2 output node: own slab, and the neighbours'
+    // halo planes (2 planes of X, 1 of V per face: what their next launch reads)
+    auto store_out = [&](int q, int64_t off, const Vec3& x2, const Vec3& v2) {
+        stb3(tp.x_out + (int64_t)(q - tp.x_base) * ps + off, cs, x2);
+        stb3(tp.v_out + (int64_t)(q - tp.v_base) * ps + off, cs, v2);
+        if (q < tp.lo_end) {
+            stb3(a.lo_dst + (int64_t)(q - start) * ps + off, cs, x2);
+            if (q == start) stb3(tp.lo_vdst + off, cs, v2);
+        }
+        if (q >= tp.hi_begin) {
+            stb3(a.hi_dst + (int64_t)(q - tp.hi_begin) * ps + off, cs, x2);
+            if (q == start + size - 1) stb3(tp.hi_vdst + off, cs, v2);
+        }
+    };
 
     // One plane of the march. kFull: a steady-state plane (p+1 exists, p is
     // updated by S1, q = p-1 is an S2 output plane): no conditions, no
@@ -193,7 +224,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         constexpr bool kFull = decltype(full_c)::value;
         constexpr int kPar = decltype(par_c)::value;
         const int par = kPar >= 0 ? kPar : (p & 1);
-        const bool upd1 = kFull || (p >= 1 && p <= size);  // S1 updates plane p (else a fixed face plane)
+        const bool upd1 = kFull || (p >= 1 && p <= ilast);  // S1 updates plane p (else a fixed face plane)
         const bool has_next = kFull || p + 1 <= qlast;
         if (has_next) xwait(p + 1);
         const double* Xc = xbox(p);
@@ -261,14 +292,16 @@ __global__ void __launch_bounds__(kThreads, 1)
             const double* yq = sm.y[par ^ 1][0];
             xqA = ldb(yq, yA, kYComp);
             xqB = ldb(yq, yB, kYComp);
-            gpi2A = spring_force<kPosK>(xqA, x1A, a.K, a.L);
-            gpi2B = spring_force<kPosK>(xqB, x1B, a.K, a.L);
-            if (out2) {
-                gpk2A = spring_force<kPosK>(xqA, ldb(yq, yAk, kYComp), a.K, a.L);
-                gpk2B = spring_force<kPosK>(xqB, ldb(yq, yBk, kYComp), a.K, a.L);
-                gpj2A = spring_force<kPosK>(xqA, xqB, a.K, a.L);
-                gpj2B = spring_force<kPosK>(xqB, ldb(yq, yBj, kYComp), a.K, a.L);
-                sm.g2j[w][lane] = gpj2B;
+            if (kTwo) {
+                gpi2A = spring_force<kPosK>(xqA, x1A, a.K, a.L);
+                gpi2B = spring_force<kPosK>(xqB, x1B, a.K, a.L);
+                if (out2) {
+                    gpk2A = spring_force<kPosK>(xqA, ldb(yq, yAk, kYComp), a.K, a.L);
+                    gpk2B = spring_force<kPosK>(xqB, ldb(yq, yBk, kYComp), a.K, a.L);
+                    gpj2A = spring_force<kPosK>(xqA, xqB, a.K, a.L);
+                    gpj2B = spring_force<kPosK>(xqB, ldb(yq, yBj, kYComp), a.K, a.L);
+                    sm.g2j[w][lane] = gpj2B;
+                }
             }
         }
         const Vec3 up2A = shfl_up1(gpk2A), up2B = shfl_up1(gpk2B);
@@ -277,22 +310,17 @@ __global__ void __launch_bounds__(kThreads, 1)
             fence_proxy_async();
             issue_v(p + kVStages);
         }
-        // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q
+        // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q (one-step mode: X_{t+1}, V_{t+1} of S1)
         if (out2) {
             if (ownA) {
                 if (intA) {
-                    const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
-                    const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
-                    Vec3 v2 = v1pA, x2;
-                    kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
-                    double* xo = tp.x_out + (int64_t)q * ps + offA;
-                    double* vo = tp.v_out + (int64_t)(q - 1) * ps + offA;
-                    xo[0] = x2.x;
-                    xo[cs] = x2.y;
-                    xo[2 * cs] = x2.z;
-                    vo[0] = v2.x;
-                    vo[cs] = v2.y;
-                    vo[2 * cs] = v2.z;
+                    Vec3 v2 = v1pA, x2 = xqA;
+                    if (kTwo) {
+                        const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
+                        const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
+                        kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
+                    }
+                    store_out(q, offA, x2, v2);
                     st.add_position(x2);
                     st.add_velocity(v2);
                 } else {
@@ -301,17 +329,12 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             if (ownB) {
                 if (intB) {
-                    const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
-                    Vec3 v2 = v1pB, x2;
-                    kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
-                    double* xo = tp.x_out + (int64_t)q * ps + offB;
-                    double* vo = tp.v_out + (int64_t)(q - 1) * ps + offB;
-                    xo[0] = x2.x;
-                    xo[cs] = x2.y;
-                    xo[2 * cs] = x2.z;
-                    vo[0] = v2.x;
-                    vo[cs] = v2.y;
-                    vo[2 * cs] = v2.z;
+                    Vec3 v2 = v1pB, x2 = xqB;
+                    if (kTwo) {
+                        const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
+                        kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
+                    }
+                    store_out(q, offB, x2, v2);
                     st.add_position(x2);
                     st.add_velocity(v2);
                 } else {
@@ -335,8 +358,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     using PN = std::integral_constant<int, -1>;
     using P0 = std::integral_constant<int, 0>;
     using P1 = std::integral_constant<int, 1>;
-    // steady planes: p >= pb+1 (q = p-1 is an output plane, p > ps0), p <= min(size, pe) (updated, p+1 exists)
-    const int lo = pb + 1, hi = min(size, pe);
+    // steady planes: p >= pb+1 (q = p-1 is an output plane, p > ps0), p <= min(ilast, pe) (updated, p+1 exists)
+    const int lo = pb + 1, hi = min(ilast, pe);
     int p = ps0;
     for (; p < lo && p <= pe; p++) body(F0{}, PN{}, p);
     if (p <= hi && (p & 1)) body(F1{}, P1{}, p++);
@@ -347,18 +370,26 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (p <= hi) body(F1{}, P0{}, p++);
     for (; p <= pe; p++) body(F0{}, PN{}, p);
     block_accumulate(st, sm.scratch, a.acc);
+    signal_neighbours(a);
 }
 
 }  // namespace
 
-cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, StatsAccum* /*acc1*/, bool unit_mass,
-                          cudaStream_t stream) {
+cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream) {
     if (a.g.size <= 0) return cudaSuccess;
-    if (!a.tmap_x_cur || !a.tmap_v || a.lo_dst || a.hi_dst) return cudaErrorInvalidValue;
+    if (!a.tmap_x_cur || !a.tmap_v || !o.x_out || !o.v_out) return cudaErrorInvalidValue;
+    if ((a.lo_dst && (!o.lo_vdst || a.g.size < 2)) || (a.hi_dst && (!o.hi_vdst || a.g.size < 2)))
+        return cudaErrorInvalidValue;  // a neighbour's two halo planes come from one chunk
     Tb2Params tp;
     tp.a = a;
-    tp.x_out = x_out;
-    tp.v_out = v_out;
+    tp.x_out = o.x_out;
+    tp.v_out = o.v_out;
+    tp.lo_vdst = o.lo_vdst;
+    tp.hi_vdst = o.hi_vdst;
+    tp.x_base = (int)a.g.start - 2;
+    tp.v_base = (int)a.g.start - 1;
+    tp.lo_end = a.lo_dst ? (int)a.g.start + 2 : INT_MIN;
+    tp.hi_begin = a.hi_dst ? (int)(a.g.start + a.g.size) - 2 : INT_MAX;
     tp.tiles_k = (int)((a.g.n2 + kOK - 1) / kOK);
     tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;
@@ -377,10 +408,17 @@ cudaError_t launch_k1_tb2(const StepArgs& a, double* x_out, double* v_out, Stats
         kernel<<<grid, block, smem, stream>>>(mx, mv, tp);
     };
     const bool pos_k = a.K > 0.0;
-    if (unit_mass)
-        pos_k ? launch(k1_tb2_kernel<true, true>) : launch(k1_tb2_kernel<true, false>);
-    else
-        pos_k ? launch(k1_tb2_kernel<false, true>) : launch(k1_tb2_kernel<false, false>);
+    if (o.two) {
+        if (unit_mass)
+            pos_k ? launch(k1_tb2_kernel<true, true, true>) : launch(k1_tb2_kernel<true, false, true>);
+        else
+            pos_k ? launch(k1_tb2_kernel<false, true, true>) : launch(k1_tb2_kernel<false, false, true>);
+    } else {
+        if (unit_mass)
+            pos_k ? launch(k1_tb2_kernel<true, true, false>) : launch(k1_tb2_kernel<true, false, false>);
+        else
+            pos_k ? launch(k1_tb2_kernel<false, true, false>) : launch(k1_tb2_kernel<false, false, false>);
+    }
     return cudaGetLastError();
 }
 

@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdint>
 #include <cstdlib>
 #include <cstring>
 #include <map>
@@ -27,7 +28,7 @@ using paper::set_last_error;
 namespace {
 
 constexpr uint64_t kIpcMagic = 0x534f4d4945524950ull;  // "SOMIERIP"
-constexpr uint32_t kIpcVersion = 2;
+constexpr uint32_t kIpcVersion = 3;
 
 using PFN_waitValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 using PFN_encodeTiled = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -51,10 +52,15 @@ struct Chunk {
     bool local = false;
     // local allocation: [x0 | x1 | v0 | (v1, K1_TB2 only) | acc[4] | flags[2] | counter]
     // acc: [0], [1] stats of the last steps by step parity, [2] the fixed end
-    // planes, [3] scratch (K1_TB2's first step)
+    // planes, [3] unused.
+    // X slabs: planes [start-1, start+size+1) (one halo plane per face), V
+    // slabs [start, start+size); on a K1_TB2 handle one more halo plane per
+    // face each (X [start-2, start+size+2), V [start-1, start+size+1)) and V
+    // double-buffered. xs()/vs() are the one-halo views every other path uses.
     void* base = nullptr;
     size_t bytes = 0;
     size_t off_x[2] = {0, 0}, off_v = 0, off_v1 = 0, off_acc = 0, off_flags = 0, off_counter = 0;
+    int64_t view_off = 0;  // doubles from a raw slab to its one-halo view (one plane on K1_TB2 handles)
     // remote view (IPC-opened), for non-local neighbours
     void* remote_base = nullptr;
     // TMA descriptors of the local slabs, by X / V buffer: K1_MARCH, K1_MARCH2, K1_TB2 box shapes
@@ -68,6 +74,8 @@ struct Chunk {
     void* mem() const { return local ? base : remote_base; }
     double* x(int parity) const { return (double*)((char*)mem() + off_x[parity]); }
     double* v(int b = 0) const { return (double*)((char*)mem() + (b ? off_v1 : off_v)); }
+    double* xs(int parity) const { return x(parity) + view_off; }
+    double* vs(int b = 0) const { return v(b) + view_off; }
     paper::StatsAccum* acc() const { return (paper::StatsAccum*)((char*)mem() + off_acc); }
     unsigned long long* flags() const { return (unsigned long long*)((char*)mem() + off_flags); }
     unsigned int* counter() const { return (unsigned int*)((char*)mem() + off_counter); }
@@ -75,7 +83,7 @@ struct Chunk {
 
 struct IpcChunkRecord {
     int64_t index;
-    uint64_t bytes, off_x0, off_x1, off_v, off_acc, off_flags, off_counter;
+    uint64_t bytes, off_x0, off_x1, off_v, off_v1, off_acc, off_flags, off_counter;
     cudaIpcMemHandle_t handle;
 };
 
@@ -88,6 +96,8 @@ struct IpcHeader {
     int64_t chunk;
     uint64_t layout;  // FNV-1a of every chunk's (device_pos, start, size): catches unequal irregular tables
     int64_t nrecords;
+    int32_t tb2;      // slab layout: K1_TB2 (deep halo, V double-buffered) or one-step
+    int32_t pad;
 };
 
 uint64_t spread_layout_hash(const spread_s& s) {
@@ -120,7 +130,7 @@ struct somier_s {
     int64_t launches = 0;
     int xbuf = 0;      // X buffer holding X_t (flips once per launch)
     int vbuf = 0;      // V buffer holding V_t (flips once per K1_TB2 launch; 1-step kernels update in place)
-    bool tb2 = false;  // K1_TB2 mode (single local chunk)
+    bool tb2 = false;  // K1_TB2 mode (two steps per launch, deep-halo slabs)
     bool multi_process = false;
     int local_pos = -1;
     std::vector<Chunk> chunks;
@@ -263,18 +273,20 @@ spread_status reset_stats(somier_t h, Chunk& c) {
     CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 4 * sizeof(paper::StatsAccum), s));
     const int cur = h->xbuf;
     paper::StatsAccum* last = c.acc() + ((h->step - 1) & 1);
-    CUDA_TRY(h, paper::launch_stats(c.x(cur), c.v(h->vbuf), g, 1, c.size, last, s));
-    if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, 0, 1, c.acc() + 2, s));
+    CUDA_TRY(h, paper::launch_stats(c.xs(cur), c.vs(h->vbuf), g, 1, c.size, last, s));
+    if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, 0, 1, c.acc() + 2, s));
     if (c.start + c.size == h->p.n[0] - 1)
-        CUDA_TRY(h, paper::launch_stats(c.x(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
+        CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
     return SPREAD_OK;
 }
 
 spread_status allocate_chunk(somier_t h, Chunk& c) {
     const paper::SlabGeom g = h->geom_of(c);
     const size_t plane = (size_t)g.plane_stride() * sizeof(double);
-    const size_t xb = round_up(plane * (size_t)(c.size + 2), 4096);
-    const size_t vb = round_up(plane * (size_t)c.size, 4096);
+    const int64_t deep = h->tb2 ? 1 : 0;  // K1_TB2: one more halo plane per face (X and V)
+    const size_t xb = round_up(plane * (size_t)(c.size + 2 + 2 * deep), 4096);
+    const size_t vb = round_up(plane * (size_t)(c.size + 2 * deep), 4096);
+    c.view_off = deep * g.plane_stride();
     c.off_x[0] = 0;
     c.off_x[1] = xb;
     c.off_v = 2 * xb;
@@ -291,6 +303,10 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     ia.x0 = c.x(0);
     ia.x1 = c.x(1);
     ia.g = g;
+    if (deep) {  // all planes of the deep slab: [start-2, start+size+2) (those outside the grid are never read)
+        ia.g.start -= 1;
+        ia.g.size += 2;
+    }
     ia.spacing = h->p.spacing;
     ia.amplitude = h->p.amplitude;
     ia.seed = h->p.seed;
@@ -301,12 +317,12 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
             double* base;
             int64_t planes;
             uint32_t bk, bj;
-        } maps[6] = {{&c.tmap_x[b], c.x(b), c.size + 2, paper::kXBoxK, paper::kXBoxJ},
-                     {&c.tmap_v[b], c.v(b), c.size, paper::kVBoxK, paper::kVBoxJ},
-                     {&c.tmap_x2[b], c.x(b), c.size + 2, paper::kXBoxK, paper::kX2BoxJ},
-                     {&c.tmap_v2[b], c.v(b), c.size, paper::kVBoxK, paper::kV2BoxJ},
-                     {&c.tmap_xt[b], c.x(b), c.size + 2, paper::kTB2XBoxK, paper::kTB2XBoxJ},
-                     {&c.tmap_vt[b], c.v(b), c.size, paper::kTB2VBoxK, paper::kTB2VBoxJ}};
+        } maps[6] = {{&c.tmap_x[b], c.xs(b), c.size + 2, paper::kXBoxK, paper::kXBoxJ},
+                     {&c.tmap_v[b], c.vs(b), c.size, paper::kVBoxK, paper::kVBoxJ},
+                     {&c.tmap_x2[b], c.xs(b), c.size + 2, paper::kXBoxK, paper::kX2BoxJ},
+                     {&c.tmap_v2[b], c.vs(b), c.size, paper::kVBoxK, paper::kV2BoxJ},
+                     {&c.tmap_xt[b], c.x(b), c.size + 2 + 2 * deep, paper::kTB2XBoxK, paper::kTB2XBoxJ},
+                     {&c.tmap_vt[b], c.v(b), c.size + 2 * deep, paper::kTB2VBoxK, paper::kTB2VBoxJ}};
         for (const auto& m : maps) {
             spread_status st = paper::encode_slab_tmap(m.map, g, m.base, m.planes, m.bk, m.bj);
             if (st != SPREAD_OK) return st;
@@ -373,24 +389,33 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         ch.device = h->devs[ci.pos].device;
         ch.local = (local_pos < 0) || (ci.pos == local_pos);
     }
-    // K1_TB2 (two steps per launch) needs one local chunk without neighbours.
-    // AUTO takes it there for grids of >= kTb2AutoMinNodes nodes (measured: TB2
-    // +7..13% from 192^3 up, -19% at 128^3 where its 1-CTA/SM tiles fill few
-    // waves) when the device has room for its second V buffer
-    // (96 instead of 72 B/node), else K1_MARCH2.
+    // K1_TB2 (two steps per launch, deep-halo slabs) runs any spread whose
+    // chunks hold >= 2 planes each when there are several (a neighbour's two
+    // halo planes come from one chunk). AUTO takes it where it was measured
+    // faster than K1_MARCH2 -- chunks of >= kTb2AutoMinNodes nodes (TB2
+    // +7..13% from 192^3 up, -19% at 128^3 where its one CTA per SM fills few
+    // waves) -- and each device has room for its deeper slabs
+    // and second V buffer (96 instead of 72 B/node).
     constexpr double kTb2AutoMinNodes = 6.0e6;
     h->tb2 = false;
-    if ((p->kernel == SOMIER_K1_TB2 || p->kernel == SOMIER_K1_AUTO) && local_pos < 0 && s->nchunks == 1) {
-        h->tb2 = p->kernel == SOMIER_K1_TB2 || (double)p->n[0] * (double)p->n[1] * (double)p->n[2] >= kTb2AutoMinNodes;
+    if (p->kernel == SOMIER_K1_TB2 || p->kernel == SOMIER_K1_AUTO) {
+        int64_t min_size = INT64_MAX;
+        for (auto& c : h->chunks) min_size = std::min(min_size, c.size);
+        const bool layout_ok = s->nchunks == 1 || min_size >= 2;
+        h->tb2 = layout_ok && (p->kernel == SOMIER_K1_TB2 ||
+                               (double)min_size * (double)p->n[1] * (double)p->n[2] >= kTb2AutoMinNodes);
         if (h->tb2 && p->kernel == SOMIER_K1_AUTO) {
-            const Chunk& c = h->chunks[0];
             const size_t plane = (size_t)3 * (size_t)p->n[1] * (size_t)h->ld * sizeof(double);
-            const size_t need = 2 * plane * (size_t)(c.size + 2) + 2 * plane * (size_t)c.size;
-            size_t free_b = 0, total_b = 0;
-            if (cudaSetDevice(c.device) != cudaSuccess || cudaMemGetInfo(&free_b, &total_b) != cudaSuccess ||
-                free_b < need + ((size_t)1 << 30))
-                h->tb2 = false;
-            cudaGetLastError();
+            std::map<int, size_t> need;
+            for (auto& c : h->chunks)
+                if (c.local) need[c.device] += 2 * plane * (size_t)(c.size + 4) + 2 * plane * (size_t)(c.size + 2);
+            for (auto& kv : need) {
+                size_t free_b = 0, total_b = 0;
+                if (cudaSetDevice(kv.first) != cudaSuccess || cudaMemGetInfo(&free_b, &total_b) != cudaSuccess ||
+                    free_b < kv.second + ((size_t)1 << 30))
+                    h->tb2 = false;
+                cudaGetLastError();
+            }
         }
     }
     st = load_driver_entry(h);
@@ -585,7 +610,7 @@ extern "C" {
 
 namespace {
 spread_status enqueue_steps(somier_t h, int64_t nsteps);
-spread_status enqueue_tb2(somier_t h);
+spread_status enqueue_tb2(somier_t h, bool two);
 }
 
 extern "C" {
@@ -617,6 +642,7 @@ spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len) 
         r.off_x0 = c.off_x[0];
         r.off_x1 = c.off_x[1];
         r.off_v = c.off_v;
+        r.off_v1 = c.off_v1;
         r.off_acc = c.off_acc;
         r.off_flags = c.off_flags;
         r.off_counter = c.off_counter;
@@ -634,6 +660,7 @@ spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len) 
     hd.chunk = h->spread.chunk;
     hd.layout = spread_layout_hash(h->spread);
     hd.nrecords = (int64_t)recs.size();
+    hd.tb2 = h->tb2 ? 1 : 0;
     const size_t need = sizeof hd + recs.size() * sizeof(IpcChunkRecord);
     if (len) *len = need;
     if (!buf) return SPREAD_OK;
@@ -658,6 +685,9 @@ spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const siz
             hd.nchunks != (int64_t)h->chunks.size() || hd.chunk != h->spread.chunk ||
             hd.layout != spread_layout_hash(h->spread))
             PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d describes another grid or spread", b);
+        if (hd.tb2 != (h->tb2 ? 1 : 0))
+            PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d uses the other K1 slab layout (K1_TB2 vs one-step): "
+                       "the processes resolved the kernel differently; pass the same explicit kernel", b);
         if (lens[b] != sizeof hd + (size_t)hd.nrecords * sizeof(IpcChunkRecord))
             PAPER_FAIL(SPREAD_EINVAL, "somier_ipc_connect: blob %d has a bad length", b);
         if (hd.device_pos == h->local_pos) continue;
@@ -689,6 +719,8 @@ spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const siz
             o.off_x[0] = rec.off_x0;
             o.off_x[1] = rec.off_x1;
             o.off_v = rec.off_v;
+            o.off_v1 = rec.off_v1;
+            o.view_off = h->tb2 ? h->geom.plane_stride() : 0;
             o.off_acc = rec.off_acc;
             o.off_flags = rec.off_flags;
             o.off_counter = rec.off_counter;
@@ -704,18 +736,13 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     if (!h->connected) PAPER_FAIL(SPREAD_ESTATE, "somier_step: remote neighbour chunks not connected (somier_ipc_connect)");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     if (h->tb2) {
-        // K1_TB2: pairs of steps from an even step count; a leftover single step
-        // (or an odd start) runs the one-step K1
-        if ((h->step & 1) && nsteps > 0) {
-            spread_status st = enqueue_steps(h, 1);
-            if (st != SPREAD_OK) return st;
-            nsteps--;
-        }
+        // K1_TB2: pairs of steps; a leftover single step runs the same kernel
+        // in one-step mode (same slab layout and halo protocol)
         for (; nsteps >= 2; nsteps -= 2) {
-            spread_status st = enqueue_tb2(h);
+            spread_status st = enqueue_tb2(h, true);
             if (st != SPREAD_OK) return st;
         }
-        return enqueue_steps(h, nsteps);
+        return nsteps ? enqueue_tb2(h, false) : SPREAD_OK;
     }
     // All chunks on one stream (no cross-stream flags): the launches of two
     // consecutive steps depend only on the buffer parity, so a CUDA graph of an
@@ -794,11 +821,11 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             }
             paper::StepArgs a;
             std::memset(&a, 0, sizeof a);
-            a.x_cur = me.x(cur);
-            a.x_nxt = me.x(nxt);
-            a.v = me.v(vb);
-            a.lo_dst = left ? left->x(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
-            a.hi_dst = right ? right->x(nxt) : nullptr;
+            a.x_cur = me.xs(cur);
+            a.x_nxt = me.xs(nxt);
+            a.v = me.vs(vb);
+            a.lo_dst = left ? left->xs(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
+            a.hi_dst = right ? right->xs(nxt) : nullptr;
             a.g = h->geom_of(me);
             a.K = h->p.k_spring;
             a.L = h->p.rest_len;
@@ -824,34 +851,76 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
     return SPREAD_OK;
 }
 
-// K1_TB2: steps t, t+1 (t even) in one launch of the single local chunk.
-// Stats of step t go to the scratch slot 3, of step t+1 to slot 1 (the slot
-// somier_stats reads after t+2 steps); slot 0 stays zero for step t+2.
-spread_status enqueue_tb2(somier_t h) {
-    Chunk* me = nullptr;
-    for (auto& c : h->chunks)
-        if (c.local) me = &c;
-    if (!me || (h->step & 1)) PAPER_FAIL(SPREAD_ESTATE, "somier_step: K1_TB2 needs one local chunk and an even step");
-    CUDA_TRY(h, cudaSetDevice(me->device));
-    cudaStream_t st = h->stream_of(*me);
-    CUDA_TRY(h, cudaMemsetAsync(me->acc() + 1, 0, sizeof(paper::StatsAccum), st));
-    CUDA_TRY(h, cudaMemsetAsync(me->acc() + 3, 0, sizeof(paper::StatsAccum), st));
+// K1_TB2: steps t, t+1 (two) or step t in one launch per local chunk. The
+// launch reads X_t / V_t (buffers xbuf / vbuf) with their deep halos and
+// writes the other buffers, its boundary planes also into the neighbours'
+// other buffers; flags as in enqueue_steps (the neighbours finished the launch
+// that produced step t: my halo planes of X_t / V_t are written, and they no
+// longer read their buffers I write into). Stats of the last step go to slot
+// (t_end - 1) & 1, zeroed first.
+spread_status enqueue_tb2(somier_t h, bool two) {
+    const int64_t nch = (int64_t)h->chunks.size();
+    const int64_t t = h->step, t_end = t + (two ? 2 : 1);
     const int cur = h->xbuf, vb = h->vbuf;
-    paper::StepArgs a;
-    std::memset(&a, 0, sizeof a);
-    a.x_cur = me->x(cur);
-    a.v = me->v(vb);
-    a.g = h->geom_of(*me);
-    a.K = h->p.k_spring;
-    a.L = h->p.rest_len;
-    a.M = h->p.mass;
-    a.dt = h->p.dt;
-    a.acc = me->acc() + 1;
-    a.tmap_x_cur = &me->tmap_xt[cur];
-    a.tmap_v = &me->tmap_vt[vb];
-    CUDA_TRY(h, paper::launch_k1_tb2(a, me->x(cur ^ 1), me->v(vb ^ 1), me->acc() + 3, h->unit_mass(), st));
-    h->launches++;
-    h->step += 2;
+    const int slot = (int)((t_end - 1) & 1);
+    const int64_t ps = h->geom.plane_stride();
+    int cur_dev = -1;
+    for (int64_t c = 0; c < nch; c++) {
+        Chunk& me = h->chunks[c];
+        if (!me.local) continue;
+        if (me.device != cur_dev) {
+            CUDA_TRY(h, cudaSetDevice(me.device));
+            cur_dev = me.device;
+        }
+        cudaStream_t st = h->stream_of(me);
+        const Chunk* left = c > 0 ? &h->chunks[c - 1] : nullptr;
+        const Chunk* right = c + 1 < nch ? &h->chunks[c + 1] : nullptr;
+        const bool fl = left && h->needs_flags(me, *left);
+        const bool fr = right && h->needs_flags(me, *right);
+        for (int side = 0; side < 2; side++) {
+            if (t == 0 || !(side ? fr : fl)) continue;
+            CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[side], (cuuint64_t)t,
+                                         CU_STREAM_WAIT_VALUE_GEQ | h->devs[me.pos].wait_flush);
+            if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
+        }
+        CUDA_TRY(h, cudaMemsetAsync(me.acc() + slot, 0, sizeof(paper::StatsAccum), st));
+        paper::StepArgs a;
+        std::memset(&a, 0, sizeof a);
+        a.x_cur = me.x(cur);
+        a.v = me.v(vb);
+        a.g = h->geom_of(me);
+        a.K = h->p.k_spring;
+        a.L = h->p.rest_len;
+        a.M = h->p.mass;
+        a.dt = h->p.dt;
+        a.acc = me.acc() + slot;
+        a.tmap_x_cur = &me.tmap_xt[cur];
+        a.tmap_v = &me.tmap_vt[vb];
+        paper::Tb2Out o;
+        std::memset(&o, 0, sizeof o);
+        o.x_out = me.x(cur ^ 1);
+        o.v_out = me.v(vb ^ 1);
+        o.two = two;
+        // neighbours' deep halo planes in THEIR out buffers: left X planes of
+        // global i = start, start+1 (its raw planes size+2, size+3), V plane
+        // of i = start (raw size+1); right X planes start+size-2, -1 (raw 0, 1),
+        // V plane start+size-1 (raw 0)
+        if (left) {
+            a.lo_dst = left->x(cur ^ 1) + (left->size + 2) * ps;
+            o.lo_vdst = left->v(vb ^ 1) + (left->size + 1) * ps;
+        }
+        if (right) {
+            a.hi_dst = right->x(cur ^ 1);
+            o.hi_vdst = right->v(vb ^ 1);
+        }
+        a.signal_lo = fl ? &left->flags()[1] : nullptr;
+        a.signal_hi = fr ? &right->flags()[0] : nullptr;
+        a.signal_value = (unsigned long long)t_end;
+        a.done_counter = me.counter();
+        CUDA_TRY(h, paper::launch_k1_tb2(a, o, h->unit_mass(), st));
+        h->launches++;
+    }
+    h->step = t_end;
     h->xbuf ^= 1;
     h->vbuf ^= 1;
     return SPREAD_OK;
@@ -938,13 +1007,13 @@ spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* 
             if (lo >= hi) continue;
             for (int d = 0; d < 3; d++) {
                 if (X[d])
-                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, sp.slab0 + (lo - sp.lo), X[d], lo - i0, hi - lo,
+                    CUDA_TRY(h, copy_planes(h, c.xs(cur), d, sp.slab0 + (lo - sp.lo), X[d], lo - i0, hi - lo,
                                             cudaMemcpyDeviceToHost, s));
                 if (V[d]) {
                     if (sp.fixed)  // fixed end planes have zero velocity
                         std::memset(V[d] + (size_t)(lo - i0) * plane, 0, (size_t)(hi - lo) * plane * sizeof(double));
                     else
-                        CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, lo - c.start, V[d], lo - i0, hi - lo,
+                        CUDA_TRY(h, copy_planes(h, c.vs(h->vbuf), d, lo - c.start, V[d], lo - i0, hi - lo,
                                                 cudaMemcpyDeviceToHost, s));
                 }
             }
@@ -971,10 +1040,27 @@ spread_status somier_load(somier_t h, const double* x, const double* y, const do
         CUDA_TRY(h, cudaSetDevice(c.device));
         cudaStream_t s = h->stream_of(c);
         for (int d = 0; d < 3; d++) {
-            CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, const_cast<double*>(X[d]), c.start - 1, c.size + 2,
+            CUDA_TRY(h, copy_planes(h, c.xs(cur), d, 0, const_cast<double*>(X[d]), c.start - 1, c.size + 2,
                                     cudaMemcpyHostToDevice, s));
-            CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, 0, const_cast<double*>(V[d]), c.start, c.size,
+            CUDA_TRY(h, copy_planes(h, c.vs(h->vbuf), d, 0, const_cast<double*>(V[d]), c.start, c.size,
                                     cudaMemcpyHostToDevice, s));
+            if (h->tb2) {
+                // the deep halo: X planes start-2, start+size+1 and V planes
+                // start-1, start+size where they are grid planes that move
+                const int64_t n0 = h->p.n[0];
+                if (c.start - 2 >= 0)
+                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, 0, const_cast<double*>(X[d]), c.start - 2, 1,
+                                            cudaMemcpyHostToDevice, s));
+                if (c.start + c.size + 1 <= n0 - 1)
+                    CUDA_TRY(h, copy_planes(h, c.x(cur), d, c.size + 3, const_cast<double*>(X[d]),
+                                            c.start + c.size + 1, 1, cudaMemcpyHostToDevice, s));
+                if (c.start - 1 >= 1)
+                    CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, 0, const_cast<double*>(V[d]), c.start - 1, 1,
+                                            cudaMemcpyHostToDevice, s));
+                if (c.start + c.size <= n0 - 2)
+                    CUDA_TRY(h, copy_planes(h, c.v(h->vbuf), d, c.size + 1, const_cast<double*>(V[d]),
+                                            c.start + c.size, 1, cudaMemcpyHostToDevice, s));
+            }
         }
         // the X_{t+1} buffer must hold the same fixed nodes (never written by a step)
         CUDA_TRY(h, cudaMemcpyAsync(c.x(cur ^ 1), c.x(cur), c.off_x[1] - c.off_x[0], cudaMemcpyDeviceToDevice, s));

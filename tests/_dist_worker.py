@@ -117,8 +117,11 @@ def gpu_ipc(a):
     rank, world = dist.get_rank(), dist.get_world_size()
     torch.cuda.set_device(0)
     n = tuple(a.n)
-    params = P.SomierParams(n=n, seed=a.seed)
+    kernel = int(os.environ.get("SOMIER_TEST_KERNEL", P.K1_AUTO))
+    params = P.SomierParams(n=n, seed=a.seed, kernel=kernel)
     s = PD.open_local(params, chunk=a.chunk, cuda_device=0)
+    if kernel == P.K1_TB2:
+        assert s.kernel_in_use == P.K1_TB2
     s.step(a.steps)
     s.sync()
     st = PD.gather_stats(s)

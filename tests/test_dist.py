@@ -26,11 +26,13 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _launch(mode, out, n, steps, chunk, seed=3, timeout=300):
+def _launch(mode, out, n, steps, chunk, seed=3, timeout=300, kernel=None):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), WORKER, mode, out,
            *map(str, n), str(steps), str(chunk), str(seed)]
     env = dict(os.environ, OMP_NUM_THREADS="1", PYTHONPATH=ROOT)
+    if kernel is not None:
+        env["SOMIER_TEST_KERNEL"] = str(kernel)
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, env=env)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     return np.load(out)
@@ -55,11 +57,12 @@ def test_gloo_two_ranks_slab_exchange_bit_identical(tmp_path, chunk):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("kernel", [0, 4])  # K1_AUTO (one-step kernel at this size), K1_TB2 (deep-halo exchange)
 @pytest.mark.parametrize("chunk", [0, 2, 5])
-def test_gpu_two_processes_ipc_fused_exchange(tmp_path, chunk):
+def test_gpu_two_processes_ipc_fused_exchange(tmp_path, chunk, kernel):
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     n, steps, seed = (20, 12, 40), 15, 4
-    res = _launch("gpu-ipc", str(tmp_path / "g.npz"), n, steps, chunk, seed, timeout=600)
+    res = _launch("gpu-ipc", str(tmp_path / "g.npz"), n, steps, chunk, seed, timeout=600, kernel=kernel)
     _check(res, n, steps, seed)

@@ -46,15 +46,9 @@ def test_eager_and_graph_identical(monkeypatch):
 
 
 def _tb2_launches(splits):
-    """K1_TB2 launch rule (somier_step): an odd start runs one single step,
-    then pairs, then a leftover single step."""
-    step = launches = 0
-    for k in splits:
-        if step % 2 and k:
-            launches, step, k = launches + 1, step + 1, k - 1
-        launches += k // 2 + k % 2
-        step += k
-    return launches
+    """K1_TB2 launch rule (somier_step): pairs of steps, then a leftover single
+    step (the same kernel in one-step mode), whatever the start parity."""
+    return sum(k // 2 + k % 2 for k in splits)
 
 
 @pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7), (1, 12)])
@@ -79,8 +73,11 @@ def test_auto_kernel_resolution():
     big = P.SomierParams(n=(200, 200, 200), seed=3)  # 8e6 nodes: K1_TB2's range
     with P.Somier(P.Spread([0], 1, 198), big) as s:
         assert s.kernel_in_use == P.K1_TB2
-    with P.Somier(P.Spread([0], 1, 198, chunk=99), big) as s:
-        assert s.kernel_in_use == P.K1_MARCH2  # several chunks: one-step kernel with the fused exchange
+    tall = P.SomierParams(n=(320, 200, 200), seed=3)
+    with P.Somier(P.Spread([0], 1, 318, chunk=159), tall) as s:
+        assert s.kernel_in_use == P.K1_TB2  # two chunks of 159 planes x 200^2 nodes: K1_TB2 with deep halos
+    with P.Somier(P.Spread([0], 1, 198, chunk=40), big) as s:
+        assert s.kernel_in_use == P.K1_MARCH2  # a chunk of 38 planes (1.5e6 nodes): below TB2's range
     sp = P.SomierParams(n=(12, 10, 36), seed=3)
     with P.Somier(P.Spread([0], 1, 10), sp) as s:
         assert s.kernel_in_use == P.K1_MARCH2  # small grid: TB2's tiles fill too few waves

@@ -22,7 +22,7 @@ def _need_gpu():
 
 @pytest.mark.parametrize("devices,chunk", [([0, 1], 0), ([0, 1, 2, 3], 0), ([3, 1, 0, 2], 3), ([5, 7], 2),
                                            ([0, 1, 2], 1)])
-@pytest.mark.parametrize("kernel", [P.K1_MARCH, P.K1_MARCH2, P.K1_DIRECT])
+@pytest.mark.parametrize("kernel", [P.K1_MARCH, P.K1_MARCH2, P.K1_DIRECT, P.K1_TB2])
 def test_logical_devices_bit_identical(devices, chunk, kernel):
     n, steps = (22, 19, 45), 17
     sp = P.SomierParams(n=n, seed=11, kernel=kernel)
@@ -77,3 +77,56 @@ def test_weighted_spread_bit_identical():
         X, V = s.read()
     ref, _ = O.run(O.init(O.Params(n=n, seed=8)), 9)
     assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+
+
+@pytest.mark.parametrize("devices,sizes", [([0, 1], [3, 17]), ([0, 1, 2], [2, 8, 2, 5, 3]), ([2, 0], [18, 2]),
+                                           ([0], [4, 4, 12]), ([0, 1], [2, 2, 2, 2, 2, 2, 2, 2, 2, 2])])
+def test_tb2_deep_halo_spreads_bit_identical(devices, sizes):
+    """K1_TB2 on several chunks: two X halo planes and one V halo plane per face,
+    stored by the neighbour's kernel (cross-stream flags between list
+    positions, stream order within one); chunks of two planes (both halo planes
+    from one neighbour); pairs and single steps, on either parity."""
+    n = (22, 19, 45)
+    sp = P.SomierParams(n=n, seed=7, kernel=P.K1_TB2)
+    spread = P.Spread.with_sizes(devices, 1, n[0] - 2, sizes)
+    with P.Somier(spread, sp, cuda_devices=[0] * len(devices)) as s:
+        assert s.kernel_in_use == P.K1_TB2
+        done = 0
+        for k in (4, 1, 3, 2, 5):
+            s.step(k)
+            done += k
+            st = s.stats()
+            ref, rst = O.run(O.init(O.Params(n=n, seed=7)), done)
+            assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits, (k, done)
+        X, V = s.read()
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+
+
+def test_tb2_one_plane_chunk_falls_back():
+    """A chunk of one plane among several cannot feed a neighbour's two halo
+    planes: K1_TB2 resolves to K1_MARCH2 (still bit-identical)."""
+    n = (14, 12, 33)
+    sp = P.SomierParams(n=n, seed=2, kernel=P.K1_TB2)
+    with P.Somier(P.Spread.with_sizes([0, 1], 1, n[0] - 2, [1, 11]), sp, cuda_devices=[0, 0]) as s:
+        assert s.kernel_in_use == P.K1_MARCH2
+        s.step(5)
+        X, V = s.read()
+    ref, _ = O.run(O.init(O.Params(n=n, seed=2)), 5)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+
+
+@pytest.mark.parametrize("chunk", [0, 2, 3])
+def test_tb2_load_and_continue(chunk):
+    """somier_load fills the deep halo planes (X two, V one per face) too."""
+    n = (14, 12, 33)
+    sp = P.SomierParams(n=n, seed=2, kernel=P.K1_TB2)
+    with P.Somier(P.Spread([0, 1, 2], 1, n[0] - 2, chunk=chunk), sp, cuda_devices=[0, 0, 0]) as s:
+        s.step(3)
+        X, V = s.read()
+        s.load(X, V)
+        s.step(7)
+        X2, V2 = s.read()
+        st = s.stats()
+    ref, rst = O.run(O.init(O.Params(n=n, seed=2)), 10)
+    assert np.array_equal(X2, ref.X) and np.array_equal(V2, ref.V)
+    assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits

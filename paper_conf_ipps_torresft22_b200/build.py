@@ -25,7 +25,9 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall,-Wno-unknown-pragmas",
           "-I" + INCLUDE, "-I" + CSRC]
-CU_FLAGS = ARCH + ["-Xptxas", "-v", "--expt-relaxed-constexpr"] + os.environ.get("SOMIER_NVCC_DEFS", "").split()
+# variant macros apply to host sources too: box shapes (driver_util.hpp) must match the kernels
+DEFS = os.environ.get("SOMIER_NVCC_DEFS", "").split()
+CU_FLAGS = ARCH + ["-Xptxas", "-v", "--expt-relaxed-constexpr"] + DEFS
 
 
 def sources():
@@ -52,7 +54,7 @@ def _compile(src, newest_hdr, verbose):
     if src.endswith(".cu"):
         cmd[1:1] = CU_FLAGS
     else:
-        cmd[1:1] = ARCH
+        cmd[1:1] = ARCH + DEFS
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("nvcc failed for %s:\n%s\n%s" % (src, " ".join(cmd), r.stderr))

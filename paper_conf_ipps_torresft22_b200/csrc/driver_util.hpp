@@ -33,7 +33,7 @@ constexpr uint32_t kXBoxK = 36, kXBoxJ = 10, kVBoxK = 32, kVBoxJ = 8;
 // ... and K1_MARCH2 (two rows per warp, 32 x 16 tiles)
 constexpr uint32_t kX2BoxJ = 18, kV2BoxJ = 16;
 // ... and K1_TB2 (owned 30 x 22 tiles, ring-extended 32 x 24, boxes with a one-node ring)
-constexpr uint32_t kTB2XBoxK = 34, kTB2XBoxJ = 2 * kTB2Warps + 2, kTB2VBoxK = 34, kTB2VBoxJ = 2 * kTB2Warps;
+constexpr uint32_t kTB2XBoxK = 36, kTB2XBoxJ = 2 * kTB2Warps + 2, kTB2VBoxK = 34, kTB2VBoxJ = 2 * kTB2Warps;
 
 // somier_params.kernel -> K1 implementation (AUTO = the fastest measured)
 inline K1Variant k1_variant(int32_t kernel) {

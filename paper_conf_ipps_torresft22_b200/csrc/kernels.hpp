@@ -100,7 +100,13 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
 // Stats of planes [p0, p0+np) of an X slab (plane index inside the slab) and,
 // if v != null, of V planes [p0-1, ...) (V has no halo planes).
+// k_interior_only: skip the k-face columns (k = 0, n2-1).
 cudaError_t launch_stats(const double* x_slab, const double* v_slab, const SlabGeom& g, int64_t p0, int64_t np,
-                         StatsAccum* acc, cudaStream_t stream);
+                         StatsAccum* acc, cudaStream_t stream, bool k_interior_only = false);
+// Positions of the k-face columns (k = 0, n2-1) of X slab planes [p0, p0+np):
+// K1_TB2 tiles the interior k columns only, so these constant nodes go to the
+// static stats slot.
+cudaError_t launch_kface_stats(const double* x_slab, const SlabGeom& g, int64_t p0, int64_t np, StatsAccum* acc,
+                               cudaStream_t stream);
 
 }  // namespace paper

@@ -43,11 +43,16 @@ namespace {
 constexpr int kTK = 32, kW = kTB2Warps, kThreads = kTK * kW;
 constexpr int kRows = 2 * kW;                               // R1 rows
 constexpr int kOK = kTK - 2, kOJ = kRows - 2;               // owned tile R2
-constexpr int kBK = kTK + 2, kBJ = kRows + 2;               // X_t box: R1 + ring
+// Tiles cover the INTERIOR k columns [1, n2-2] (30 per tile: 512^3 = 17
+// tiles exactly); the fixed k-face columns are ring nodes of the edge tiles
+// and their (constant) stats are precomputed into the static stats slot. A
+// tile's first owned column kq = 1 + 30 t is odd, so the X box starts at
+// kq - 3 (an fp64 box must start on an even column): box column = R1 lane + 2.
+constexpr int kBK = kTK + 4, kBJ = kRows + 2;               // X_t box: R1 + ring (+1 alignment column each side)
 constexpr int kXComp = kBK * kBJ;
 constexpr int kXBoxBytes = kXComp * 3 * 8;
 constexpr int kXSlot = (kXBoxBytes + 127) / 128 * 128;
-constexpr int kVBK = kTK + 2, kVBJ = kRows;                 // V_t box: R1 (+1 col each side for alignment)
+constexpr int kVBK = kTK + 2, kVBJ = kRows;                 // V_t box: R1 from kq - 3 (R1 lane l: column l + 2)
 constexpr int kVComp = kVBK * kVBJ;
 constexpr int kVBoxBytes = kVComp * 3 * 8;
 constexpr int kVSlot = (kVBoxBytes + 127) / 128 * 128;
@@ -114,7 +119,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const SlabGeom& g = a.g;
     const int lane = threadIdx.x, w = threadIdx.y, tid = w * kTK + lane;
     const int tile_k = blockIdx.x % tp.tiles_k, tile_j = blockIdx.x / tp.tiles_k;
-    const int kq = tile_k * kOK, jq = tile_j * kOJ;  // owned tile origin (kq even: TMA inner coordinate)
+    const int kq = 1 + tile_k * kOK, jq = tile_j * kOJ;  // owned tile origin (interior k columns)
     const int rA = 2 * w, rB = rA + 1;               // R1 rows of this thread
     const int k = kq - 1 + lane, jA = jq - 1 + rA, jB = jA + 1;
     // planes are global i; the chunk owns [start, start + size), its X slab
@@ -130,12 +135,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto issue_x = [&](int q) {
         const int s = (q - q0) % kStages;
         mbar_expect_tx(&sm.full[s], kXBoxBytes);
-        tma_load_4d(sm.xst[s], &tmap_x, kq - 2, jq - 2, 0, q - tp.x_base, &sm.full[s]);
+        tma_load_4d(sm.xst[s], &tmap_x, kq - 3, jq - 2, 0, q - tp.x_base, &sm.full[s]);
     };
     auto issue_v = [&](int p) {  // V_t of plane p
         const int s = (p - v_first) % kVStages;
         mbar_expect_tx(&sm.vfull[s], kVBoxBytes);
-        tma_load_4d(sm.vst[s], &tmap_v, kq - 2, jq - 1, 0, p - tp.v_base, &sm.vfull[s]);
+        tma_load_4d(sm.vst[s], &tmap_v, kq - 3, jq - 1, 0, p - tp.v_base, &sm.vfull[s]);
     };
     if (tid == 0) {
         prefetch_tmap(&tmap_x);
@@ -151,15 +156,15 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto xbox = [&](int q) { return reinterpret_cast<const double*>(sm.xst[(q - q0) % kStages]); };
     auto xwait = [&](int q) { mbar_wait(&sm.full[(q - q0) % kStages], (unsigned)(((q - q0) / kStages) & 1)); };
 
-    const int xA = (rA + 1) * kBK + (lane + 1), xB = xA + kBK;   // own X box offsets
-    const int vA = rA * kVBK + (lane + 1), vB = vA + kVBK;        // own V box offsets
+    const int xA = (rA + 1) * kBK + (lane + 2), xB = xA + kBK;   // own X box offsets
+    const int vA = rA * kVBK + (lane + 2), vB = vA + kVBK;        // own V box offsets
     const int yA = rA * kTK + lane, yB = yA + kTK;                // own X_{t+1} ring offsets
     const int yAk = lane < kTK - 1 ? yA + 1 : yA;                 // +k neighbour (lane 31 is ring: unused)
     const int yBk = lane < kTK - 1 ? yB + 1 : yB;
     const int yBj = w < kW - 1 ? yB + kTK : yB;                   // +j neighbour of row B (last row is ring)
     const bool kin = k >= 1 && k < g.n2 - 1;
     const bool intA = kin && jA >= 1 && jA < g.n1 - 1, intB = kin && jB >= 1 && jB < g.n1 - 1;
-    const bool kown = lane >= 1 && lane <= kOK && k < g.n2;
+    const bool kown = lane >= 1 && lane <= kOK && k <= g.n2 - 2;   // interior k columns only
     const bool ownA = kown && rA >= 1 && jA < g.n1;               // rows 1 .. kRows-2
     const bool ownB = kown && rB <= kRows - 2 && jB < g.n1;
     const int64_t cs = g.comp_stride(), ps = g.plane_stride();
@@ -175,10 +180,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto border_springs = [&](int p) {
         const double* Xb = xbox(p);
         if (w == 0) {
-            sm.gbj[lane] = spring_force<kPosK>(ldb(Xb, lane + 1, kXComp), ldb(Xb, kBK + lane + 1, kXComp), a.K, a.L);
+            sm.gbj[lane] = spring_force<kPosK>(ldb(Xb, lane + 2, kXComp), ldb(Xb, kBK + lane + 2, kXComp), a.K, a.L);
         } else if (w == kW - 1 && lane < kRows) {
             const int r = (lane + 1) * kBK;
-            sm.gbk[lane] = spring_force<kPosK>(ldb(Xb, r, kXComp), ldb(Xb, r + 1, kXComp), a.K, a.L);
+            sm.gbk[lane] = spring_force<kPosK>(ldb(Xb, r + 1, kXComp), ldb(Xb, r + 2, kXComp), a.K, a.L);
         }
     };
 
@@ -390,7 +395,7 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
     tp.v_base = (int)a.g.start - 1;
     tp.lo_end = a.lo_dst ? (int)a.g.start + 2 : INT_MIN;
     tp.hi_begin = a.hi_dst ? (int)(a.g.start + a.g.size) - 2 : INT_MAX;
-    tp.tiles_k = (int)((a.g.n2 + kOK - 1) / kOK);
+    tp.tiles_k = (int)((a.g.n2 - 2 + kOK - 1) / kOK);
     tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;
     const int want_ctas = 4 * 148;

@@ -54,14 +54,14 @@ __global__ void __launch_bounds__(kBX* kBY) init_kernel(InitArgs a) {
 
 __global__ void __launch_bounds__(kBX* kBY)
     stats_kernel(const double* __restrict__ x, const double* __restrict__ v, SlabGeom g, int64_t p0,
-                 StatsAccum* acc) {
+                 StatsAccum* acc, int k_interior_only) {
     __shared__ WarpStats scratch[kBX * kBY / 32];
     const int64_t k = (int64_t)blockIdx.x * kBX + threadIdx.x;
     const int64_t j = (int64_t)blockIdx.y * kBY + threadIdx.y;
     const int64_t p = p0 + blockIdx.z;
     NodeStats st;
     st.zero();
-    if (j < g.n1 && k < g.n2) {
+    if (j < g.n1 && k < g.n2 && !(k_interior_only && (k == 0 || k == g.n2 - 1))) {
         const int64_t cs = g.comp_stride();
         const double* xp = x + p * g.plane_stride() + j * g.ld + k;
         st.add_position(Vec3{xp[0], xp[cs], xp[2 * cs]});
@@ -73,7 +73,34 @@ __global__ void __launch_bounds__(kBX* kBY)
     block_accumulate(st, scratch, acc);
 }
 
+// Positions of the fixed k-face columns (k = 0 and k = n2-1, every j) of
+// planes [p0, p0 + gridDim.y): the nodes K1_TB2's tiles do not own.
+__global__ void __launch_bounds__(256) kface_stats_kernel(const double* __restrict__ x, SlabGeom g, int64_t p0,
+                                                         StatsAccum* acc) {
+    __shared__ WarpStats scratch[256 / 32];
+    const int64_t j = (int64_t)blockIdx.x * 256 + threadIdx.x;
+    const int64_t p = p0 + blockIdx.y;
+    NodeStats st;
+    st.zero();
+    if (j < g.n1) {
+        const int64_t cs = g.comp_stride();
+        const double* xp = x + p * g.plane_stride() + j * g.ld;
+        st.add_position(Vec3{xp[0], xp[cs], xp[2 * cs]});
+        const int64_t k1 = g.n2 - 1;
+        st.add_position(Vec3{xp[k1], xp[cs + k1], xp[2 * cs + k1]});
+    }
+    block_accumulate(st, scratch, acc);
+}
+
 }  // namespace
+
+cudaError_t launch_kface_stats(const double* x_slab, const SlabGeom& g, int64_t p0, int64_t np, StatsAccum* acc,
+                               cudaStream_t stream) {
+    if (np <= 0) return cudaSuccess;
+    dim3 grid((unsigned)((g.n1 + 255) / 256), (unsigned)np);
+    kface_stats_kernel<<<grid, 256, 0, stream>>>(x_slab, g, p0, acc);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream) {
     dim3 block(kBX, kBY);
@@ -83,11 +110,11 @@ cudaError_t launch_init(const InitArgs& a, cudaStream_t stream) {
 }
 
 cudaError_t launch_stats(const double* x_slab, const double* v_slab, const SlabGeom& g, int64_t p0, int64_t np,
-                         StatsAccum* acc, cudaStream_t stream) {
+                         StatsAccum* acc, cudaStream_t stream, bool k_interior_only) {
     if (np <= 0) return cudaSuccess;
     dim3 block(kBX, kBY);
     dim3 grid((unsigned)((g.n2 + kBX - 1) / kBX), (unsigned)((g.n1 + kBY - 1) / kBY), (unsigned)np);
-    stats_kernel<<<grid, block, 0, stream>>>(x_slab, v_slab, g, p0, acc);
+    stats_kernel<<<grid, block, 0, stream>>>(x_slab, v_slab, g, p0, acc, k_interior_only ? 1 : 0);
     return cudaGetLastError();
 }
 

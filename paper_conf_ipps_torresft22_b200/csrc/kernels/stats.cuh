@@ -25,6 +25,56 @@ namespace paper {
 constexpr int kMaxNodesPerThread = 128;
 constexpr double kRoundC = 6755399441055744.0;  // 1.5 * 2^52
 
+#ifndef STATS_FP64_ACC
+// Per thread, the exact sums are carried as the BIT PATTERNS of the rounded
+// doubles (fp64 work: 4 operations per coordinate, the accumulation on the
+// integer pipe):
+//   hd = fma(x, 2^28, C)                   = C + h, h = round_half_even(x 2^28), |h| < 2^51
+//   r  = fma(x, 2^28, -(hd - C))           exact, |r| <= 1/2
+//   ld = fma(r, 2^32, C)                   = C + l, l = round_half_even(r 2^32)
+// C + m with |m| < 2^51 lies in [2^52, 2^53), where one unit of the mantissa
+// is 1, so bits(C + m) = bits(C) + m: sum h = sum bits(hd) - n bits(C) and
+// sum l = sum bits(ld) - n bits(C), computed modulo 2^64 (the true sums are
+// below 2^53 in magnitude). q(x) = h 2^32 + l as in the fp64 form below.
+struct NodeStats {
+    unsigned long long hb[3], lb[3];
+    unsigned int n;  // nodes added (positions)
+    double vmax2;    // NaN-sticky max of v.v
+
+    __device__ __forceinline__ void zero() {
+        hb[0] = hb[1] = hb[2] = 0ull;
+        lb[0] = lb[1] = lb[2] = 0ull;
+        n = 0u;
+        vmax2 = 0.0;
+    }
+    __device__ __forceinline__ void add_coord(int c, double x) {
+        const double hd = __fma_rn(x, 0x1p28, kRoundC);
+        const double r = __fma_rn(x, 0x1p28, -__dsub_rn(hd, kRoundC));
+        const double ld = __fma_rn(r, 0x1p32, kRoundC);
+        hb[c] += (unsigned long long)__double_as_longlong(hd);
+        lb[c] += (unsigned long long)__double_as_longlong(ld);
+    }
+    __device__ __forceinline__ void add_position(const Vec3& x) {
+        add_coord(0, x.x);
+        add_coord(1, x.y);
+        add_coord(2, x.z);
+        n++;
+    }
+    __device__ __forceinline__ void add_velocity(const Vec3& v) {
+        const double v2 = dot_self(v);
+        vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
+    }
+    // exact int128 value of sum q(x) for coordinate c
+    __device__ __forceinline__ __int128 sum(int c) const {
+        const unsigned long long cb = (unsigned long long)__double_as_longlong(kRoundC) * n;
+        const long long h = (long long)(hb[c] - cb), l = (long long)(lb[c] - cb);
+        return (__int128)h * ((__int128)1 << 32) + (__int128)l;
+    }
+    __device__ __forceinline__ unsigned long long vmax2_bits() const {
+        return (unsigned long long)__double_as_longlong(vmax2);
+    }
+};
+#else
 struct NodeStats {
     double h[3], l[3];
     double vmax2;  // NaN-sticky max of v.v
@@ -59,6 +109,8 @@ struct NodeStats {
         return (unsigned long long)__double_as_longlong(vmax2);
     }
 };
+
+#endif
 
 struct I128Stats {
     __int128 s[3];

@@ -266,17 +266,24 @@ void free_all(somier_t h) {
 
 // Recompute the stats slots of a chunk from its resident state: slot (step-1)&1
 // = stats of the current state, slot step&1 zeroed, slot 2 = the fixed end
-// planes the chunk holds as halos (global i = 0 and i = n0-1).
+// planes the chunk holds as halos (global i = 0 and i = n0-1) and, on K1_TB2
+// handles, the fixed k-face columns of its owned planes (which the kernel's
+// tiles do not own) -- those are then left out of the current slot.
 spread_status reset_stats(somier_t h, Chunk& c) {
     cudaStream_t s = h->stream_of(c);
     paper::SlabGeom g = h->geom_of(c);
     CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 4 * sizeof(paper::StatsAccum), s));
     const int cur = h->xbuf;
     paper::StatsAccum* last = c.acc() + ((h->step - 1) & 1);
-    CUDA_TRY(h, paper::launch_stats(c.xs(cur), c.vs(h->vbuf), g, 1, c.size, last, s));
+    CUDA_TRY(h, paper::launch_stats(c.xs(cur), c.vs(h->vbuf), g, 1, c.size, last, s, h->tb2));
     if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, 0, 1, c.acc() + 2, s));
     if (c.start + c.size == h->p.n[0] - 1)
         CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
+    if (h->tb2) {
+        // K1_TB2 does not own the fixed k-face columns of its planes: their
+        // constant positions are counted here once, in the static slot
+        CUDA_TRY(h, paper::launch_kface_stats(c.xs(cur), g, 1, c.size, c.acc() + 2, s));
+    }
     return SPREAD_OK;
 }
 

@@ -30,12 +30,14 @@ def _samples(n, rng, count):
     return out
 
 
-def _check_nodes(n, steps, count, seed=42, kernel=P.K1_AUTO):
+def _check_nodes(n, steps, count, seed=42, kernel=P.K1_AUTO, devices=(0,), extra=()):
     sp = P.SomierParams(n=n, seed=seed, kernel=kernel)
     op = O.Params(n=n, seed=seed)
     rng = np.random.default_rng(7)
-    nodes = _samples(n, rng, count)
-    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
+    nodes = list(extra) + _samples(n, rng, count)
+    with P.Somier(P.Spread(list(devices), 1, n[0] - 2), sp, cuda_devices=[0] * len(devices)) as s:
+        if kernel == P.K1_AUTO:
+            assert s.kernel_in_use == P.K1_TB2
         s.step(steps)
         got = {}
         for c in nodes:
@@ -55,6 +57,15 @@ def _check_nodes(n, steps, count, seed=42, kernel=P.K1_AUTO):
 def test_512cube_bench_config_sampled_nodes_bitwise():
     """configs[3] (the bench workload, K1 AUTO = K1_TB2): 512^3, 24 steps, 16 nodes."""
     _check_nodes((512, 512, 512), 24, 16)
+
+
+def test_512cube_two_positions_deep_halo_sampled_nodes_bitwise():
+    """The bench's N = 2 layout on one GPU: 512^3 over devices(0,1) (two chunks
+    of 255 planes, K1 AUTO = K1_TB2 with the two-plane halo exchange between
+    list positions), 13 steps (six two-step launches and one single step);
+    nodes on both sides of the chunk boundary and its deep halo planes."""
+    edge = [(254, 40, 77), (255, 300, 13), (256, 5, 500), (257, 255, 256), (253, 1, 1), (258, 510, 510)]
+    _check_nodes((512, 512, 512), 13, 10, devices=(0, 1), extra=edge)
 
 
 def test_512cube_march2_kernel_sampled_nodes_bitwise():

@@ -50,7 +50,7 @@ extern "C" {
 /* K1 implementations (all compute bit-identical results). */
 typedef enum {
     SOMIER_K1_AUTO = 0,      /* the fastest measured: SOMIER_K1_TB2 for a handle with
-                                one local chunk of a grid of >= 6e6 nodes whose device
+                                one local chunk of a grid of >= 3e6 nodes whose device
                                 has room for it, else SOMIER_K1_MARCH2
                                 (somier_kernel_in_use tells which)                    */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */

@@ -28,6 +28,8 @@
 
 #include <algorithm>
 #include <climits>
+#include <cmath>
+#include <cstdlib>
 #include <type_traits>
 
 #include "../kernels.hpp"
@@ -64,7 +66,7 @@ constexpr int kYComp = kRows * kTK;                         // X_{t+1} of one R1
 #define TB2_VSTAGES 2
 #endif
 constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
-constexpr int kSegPlanes = 64, kMinSegPlanes = 4;
+constexpr int kMinSegPlanes = 4, kMaxSegPlanes = 256;
 static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
 
 struct __align__(16) Smem {
@@ -398,9 +400,42 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
     tp.tiles_k = (int)((a.g.n2 - 2 + kOK - 1) / kOK);
     tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;
-    const int want_ctas = 4 * 148;
-    int nseg = (int)((a.g.size + kSegPlanes - 1) / kSegPlanes);
-    nseg = std::max(nseg, std::min((int)a.g.size, (want_ctas + tiles - 1) / tiles));
+    // Segments per tile column: one CTA per SM (384 threads x 168 registers),
+    // so the grid runs in waves of `sms` CTAs. Each segment pays ~3 planes of
+    // extra work (step t on its first and last planes, the X/V pipeline fill);
+    // a partial last wave leaves SMs idle. Pick the count minimising
+    // waves x (segment + 3), segments of at most 256 planes (measured, DESIGN.md
+    // §6: 256^3 4 segments 6.92e10 vs 6 of the old 64-plane rule 6.23e10;
+    // 512^3 5 vs 8: 7.30 vs 7.19e10; 1024^3 7 vs 16: 7.00 vs 6.88e10; one
+    // segment of 1022 planes 6.51e10).
+    static int sms_cache[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int& sms = sms_cache[dev & 63];
+    if (!sms) {
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    const int64_t size = a.g.size;
+    int nseg = 0;
+    double best = 0.0;
+    for (int c = 1; c <= std::min<int64_t>(size, 64); c++) {
+        const int64_t seg = (size + c - 1) / c;
+        if (seg < kMinSegPlanes && c > 1) break;
+        if (seg > kMaxSegPlanes) continue;  // long segments drift apart: halo rows fall out of L2
+        const double waves = std::ceil((double)tiles * c / sms);
+        const double cost = waves * (double)(seg + 3);
+        if (nseg == 0 || cost < best - 1e-9) {
+            best = cost;
+            nseg = c;
+        }
+    }
+    if (nseg == 0) nseg = (int)((size + kMaxSegPlanes - 1) / kMaxSegPlanes);
+    static const int env_nseg = [] {  // experiment hook: segments per tile column
+        const char* e = std::getenv("SOMIER_TB2_NSEG");
+        return e ? std::atoi(e) : 0;
+    }();
+    if (env_nseg > 0) nseg = std::min<int>(env_nseg, (int)a.g.size);
     tp.seg_planes = (int)((a.g.size + nseg - 1) / nseg);
     if (tp.seg_planes < kMinSegPlanes) tp.seg_planes = (int)std::min<int64_t>(kMinSegPlanes, a.g.size);
     nseg = (int)((a.g.size + tp.seg_planes - 1) / tp.seg_planes);

@@ -400,10 +400,9 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
     // chunks hold >= 2 planes each when there are several (a neighbour's two
     // halo planes come from one chunk). AUTO takes it where it was measured
     // faster than K1_MARCH2 -- chunks of >= kTb2AutoMinNodes nodes (TB2
-    // +7..13% from 192^3 up, -19% at 128^3 where its one CTA per SM fills few
-    // waves) -- and each device has room for its deeper slabs
-    // and second V buffer (96 instead of 72 B/node).
-    constexpr double kTb2AutoMinNodes = 6.0e6;
+    // +14..27% from 160^3 up, -2% at 128^3) -- and each device
+    // has room for its deeper slabs and second V buffer (96 instead of 72 B/node).
+    constexpr double kTb2AutoMinNodes = 3.0e6;
     h->tb2 = false;
     if (p->kernel == SOMIER_K1_TB2 || p->kernel == SOMIER_K1_AUTO) {
         int64_t min_size = INT64_MAX;

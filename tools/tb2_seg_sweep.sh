@@ -1,0 +1,6 @@
+OUT=gpurun_out/seg; mkdir -p $OUT
+for rep in 1 2; do
+for ns in 8 9 7 10 6 12 5 11; do
+  SOMIER_TB2_NSEG=$ns timeout 300 python bench.py --kernel tb2 --steps 100 --warmup 6 --no-e2e --no-cpu-baseline > $OUT/ns$ns.$rep.json 2>$OUT/ns$ns.$rep.err
+  python -c "import json;d=json.load(open('$OUT/ns$ns.$rep.json'));r=d['roofline'];print('nseg $ns', '%.4g'%d['value'], 'ms %.4f'%d['ms_per_step'], 'med %.4f'%r['launch_ms_distribution']['median'], d['clocks']['sm_mhz'], d['clocks']['reasons'])" 2>&1 | tail -1
+done; done

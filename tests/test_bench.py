@@ -1,0 +1,89 @@
+"""bench.py's contract: the JSON line the driver parses, for the reference arm
+(the oracle, CPU) and for our arm at N = 1 and N = 2 (two ranks sharing one
+GPU through CUDA IPC, gloo plumbing) -- the launch shapes of the round-end
+runs, at small sizes."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+
+
+def _run(args, timeout=600, env=None):
+    e = dict(os.environ)
+    e.update(env or {})
+    r = subprocess.run([sys.executable, *args], cwd=ROOT, capture_output=True, text=True, timeout=timeout, env=e)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    return lines, r
+
+
+def _torchrun(nproc, port):
+    return ["-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % nproc, "--master-addr=127.0.0.1",
+            "--master-port=%d" % port]
+
+
+def _check_common(d, n_gpus, steps, warmup):
+    assert d["metric"] == METRIC
+    assert d["unit"] == "node-updates/s" and d["higher_is_better"] is True
+    assert d["n_gpus"] == n_gpus and d["steps"] == steps and d["warmup"] >= warmup
+    assert d["value"] > 0 and d["ms_per_step"] > 0
+    assert d["dtype"] == "f64" and d["data"] == "synthetic"
+    assert d["config"]["workload"]
+    assert d["vs_baseline"] is None
+
+
+def test_reference_arm_json_line():
+    lines, _ = _run(["bench.py", "--impl", "reference", "--steps", "2", "--warmup", "3"])
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    _check_common(d, 1, 2, 3)
+    assert d["impl"] == "reference"
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["cpu_baseline"]["value"] == d["value"]
+    assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+
+
+def test_reference_arm_under_torchrun_prints_once():
+    lines, _ = _run(_torchrun(2, 29561) + ["bench.py", "--impl", "reference", "--gpus", "2", "--steps", "2",
+                                           "--warmup", "3"], env={"OMP_NUM_THREADS": "1"})
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["value"] > 0
+
+
+def test_warmup_below_three_is_refused():
+    r = subprocess.run([sys.executable, "bench.py", "--steps", "2", "--warmup", "1"], cwd=ROOT, capture_output=True,
+                       text=True, timeout=120)
+    assert r.returncode != 0
+
+
+@pytest.mark.gpu
+def test_our_arm_json_line_one_gpu():
+    lines, _ = _run(["bench.py", "--grid", "64", "--steps", "4", "--warmup", "3", "--no-cpu-baseline", "--no-e2e"])
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    _check_common(d, 1, 4, 3)
+    assert d["gpu_launches"] > 0
+    r = d["roofline"]
+    assert r["bound"] == "hbm" and r["unit"] == "GB/s" and r["peak"] > 0
+    assert abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9
+    assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
+
+
+@pytest.mark.gpu
+def test_our_arm_two_ranks_share_one_gpu():
+    """N = 2 through torchrun (the driver's launch), both ranks on cuda:0 over
+    CUDA IPC: one JSON line, whole-job value, the fused exchange's halo bytes."""
+    lines, r = _run(_torchrun(2, 29563) + ["bench.py", "--gpus", "2", "--grid", "64", "--steps", "4", "--warmup",
+                                           "3", "--share-gpu", "--no-cpu-baseline", "--no-e2e"],
+                    env={"OMP_NUM_THREADS": "1"})
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    _check_common(d, 2, 4, 3)
+    assert d["gpu_launches"] > 0
+    assert d["halo"]["bytes_per_step_total"] > 0

@@ -285,9 +285,36 @@ spread_status somier_stream_run(somier_stream_t h, double* x, double* y, double*
                                 double* vz, double* xn, double* yn, double* zn, int64_t nsteps,
                                 somier_stats_t* stats);
 
+/*
+ * somier_stream_run2 -- as somier_stream_run, but each round trip advances the
+ * state TWO steps (2.5-D temporal blocking across the host link, K1_TB2):
+ * per chunk map(to: X[start-2 : size+4], V[start-1 : size+2]) (clipped to the
+ * grid), two fused steps, map(from: X[start : size], V[start : size]) -- half
+ * the host<->device bytes per node-update of somier_stream_run. Because a
+ * chunk reads its neighbours' V_t halo planes, V is double-buffered too:
+ *   (x, y, z, vx, vy, vz) / (xn, ..., vzn): the two states, used alternately
+ *   per launch; launch k reads the first if k is even and writes the other.
+ *   nsteps / 2 two-step launches run, plus one one-step launch if nsteps is
+ *   odd; the final state is in the first buffers if the number of launches
+ *   is even, else in the second.
+ *   stats: NULL, or an array of ceil(nsteps / 2) entries receiving the
+ *   statistics after each launch (`step` says which step; the intermediate
+ *   step of a two-step launch has no statistics, as on a K1_TB2 handle).
+ * Chunk-level dependencies as in somier_stream_run, over the chunks within
+ * two planes. Results are bit-identical to somier_stream_run / the oracle.
+ * Errors: EINVAL (NULL, nsteps < 0, aliasing buffers), ENOMEM, ECUDA.
+ */
+spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                 double* vz, double* xn, double* yn, double* zn, double* vxn, double* vyn,
+                                 double* vzn, int64_t nsteps, somier_stats_t* stats);
+
 /* Bytes moved host->device and device->host by one somier_stream_step (one
  * step of somier_stream_run), and K1 launches so far. */
 spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches);
+
+/* Bytes moved host->device and device->host by one two-step launch of
+ * somier_stream_run2. */
+spread_status somier_stream_traffic2(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes);
 
 spread_status somier_stream_destroy(somier_stream_t h);
 

@@ -305,3 +305,25 @@ class SomierStream:
         N.check(N.lib().somier_stream_traffic(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)),
                 "somier_stream_traffic")
         return {"h2d_bytes": a.value, "d2h_bytes": b.value, "launches": c.value}
+
+    def run2(self, X, V, XN, VN, nsteps: int, stats: bool = True):
+        """nsteps steps, two per host round trip (somier_stream_run2): (X, V) and
+        (XN, VN) are used alternately per launch; the final state is in (X, V)
+        if the number of launches ceil(nsteps / 2) is even, else in (XN, VN).
+        Returns the Stats after each launch (or None)."""
+        return self.run2_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]],
+                              [VN[0], VN[1], VN[2]], nsteps, stats)
+
+    def run2_ptrs(self, X, V, XN, VN, nsteps: int, stats: bool = True):
+        nl = int(nsteps) // 2 + int(nsteps) % 2
+        out = (N.somier_stats_t * max(1, nl))() if stats else None
+        N.check(N.lib().somier_stream_run2(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
+                                           *[_dptr(g) for g in XN], *[_dptr(g) for g in VN], int(nsteps), out),
+                "somier_stream_run2")
+        return [Stats.from_c(out[k]) for k in range(nl)] if stats else None
+
+    def traffic2(self):
+        """Host<->device bytes of one two-step launch of run2."""
+        a, b = ctypes.c_int64(), ctypes.c_int64()
+        N.check(N.lib().somier_stream_traffic2(self._h, ctypes.byref(a), ctypes.byref(b)), "somier_stream_traffic2")
+        return {"h2d_bytes": a.value, "d2h_bytes": b.value}

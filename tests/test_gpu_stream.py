@@ -154,3 +154,67 @@ def test_stream_run_equals_steps_and_continues():
             s.run(X, V, X, 2)
     ref, rst = O.run(O.init(_op(sp)), 7)
     assert np.array_equal(XN, ref.X) and np.array_equal(V, ref.V) and st.sums == rst.sums
+
+
+@pytest.mark.parametrize("devices,spread_kw,buffers,nsteps", [
+    ([0], {"chunk": 3}, 2, 8), ([0], {"chunk": 4}, 1, 9), ([0, 1, 2], {"chunk": 2}, 2, 7),
+    ([0, 1], {"sizes": [1, 6, 2, 1, 4]}, 3, 6), ([0, 1, 2, 3], {"chunk": 0}, 2, 5), ([0], {"chunk": 100}, 2, 4),
+    ([0], {"sizes": [1, 1, 12]}, 2, 3), ([0], {"chunk": 1}, 3, 2)])
+def test_stream_run2_two_steps_per_round_trip(devices, spread_kw, buffers, nsteps):
+    """somier_stream_run2: two steps per host round trip (K1_TB2 on each chunk
+    with X halo 2 and V halo 1 from the host copies, V double-buffered), odd
+    step counts end with a one-step launch; chunks of one plane whose halos
+    reach two chunks away; the stats after every launch and the final state
+    equal the oracle's bit for bit, NaN-filled output buffers leave no trace."""
+    n = (16, 13, 37)
+    sp = P.SomierParams(n=n, seed=6)
+    if "sizes" in spread_kw:
+        spread = P.Spread.with_sizes(devices, 1, n[0] - 2, spread_kw["sizes"])
+    else:
+        spread = P.Spread(devices, 1, n[0] - 2, chunk=spread_kw["chunk"])
+    with P.SomierStream(spread, sp, buffers=buffers, cuda_devices=[0] * len(devices)) as s:
+        X0, V0 = s.generate()
+        X, V, XN, VN = _pinned_like(X0), _pinned_like(V0), _pinned_like(X0), _pinned_like(V0)
+        X[...] = X0
+        V[...] = V0
+        XN[...] = np.nan
+        VN[...] = np.nan
+        stats = s.run2(X, V, XN, VN, nsteps)
+        tr = s.traffic2()
+    nl = nsteps // 2 + nsteps % 2
+    fX, fV = (X, V) if nl % 2 == 0 else (XN, VN)
+    ref = O.init(_op(sp))
+    done = 0
+    for k in range(nl):
+        for _ in range(2 if k < nsteps // 2 else 1):
+            ref, rst = O.step(ref)
+            done += 1
+        assert stats[k].step == done
+        assert stats[k].sums == rst.sums and stats[k].vmax2_bits == rst.vmax2_bits and stats[k].centre == rst.centre
+    assert done == nsteps
+    assert np.array_equal(fX, ref.X) and np.array_equal(fV, ref.V)
+    plane = 3 * n[1] * n[2] * 8
+    assert tr["d2h_bytes"] == 2 * plane * (n[0] - 2) + 4 * plane
+
+
+def test_stream_run2_matches_run_and_resident():
+    """run2 (two steps per round trip) = run (one) = the resident K1_TB2 handle."""
+    sp = P.SomierParams(n=(40, 33, 70), seed=9, mass=1.3, k_spring=7.0)
+    with P.SomierStream(P.Spread([0], 1, 38, chunk=9), sp, buffers=2) as s:
+        X, V = s.generate()
+        X2, V2, XN, XN2, VN2 = X.copy(), V.copy(), np.zeros_like(X), np.zeros_like(X), np.zeros_like(V)
+        st1 = s.run(X, V, XN, 10)
+        st2 = s.run2(X2, V2, XN2, VN2, 10)
+        h1 = s.traffic()
+        h2 = s.traffic2()
+    # run: X_10 in X (even); run2: 5 launches -> (XN2, VN)
+    with P.Somier(P.Spread([0], 1, 38), P.SomierParams(n=(40, 33, 70), seed=9, mass=1.3, k_spring=7.0,
+                                                       kernel=P.K1_TB2)) as r:
+        r.step(10)
+        Xr, Vr = r.read()
+        sr = r.stats()
+    assert st1[-1].sums == st2[-1].sums == sr.sums
+    assert np.array_equal(X, Xr) and np.array_equal(V, Vr)
+    assert np.array_equal(XN2, Xr) and np.array_equal(VN2, Vr)
+    # per node-update, run2 moves about half the host<->device bytes of run
+    assert (h2["h2d_bytes"] + h2["d2h_bytes"]) / 2 < 0.6 * (h1["h2d_bytes"] + h1["d2h_bytes"])

@@ -1,7 +1,8 @@
 #!/usr/bin/env python3
 """Small runs of every kernel path for compute-sanitizer (tests/test_gpu_sanitizer.py):
 K1 direct / march / march2 over a multi-chunk spread (fused halo stores), the
-host-streamed mode, K2 and K3, and K1_TB2 on a single chunk."""
+host-streamed mode (one and two steps per round trip), K2 and K3, and K1_TB2 on a
+single chunk."""
 import os
 import sys
 
@@ -34,4 +35,8 @@ for kern in (P.K1_TB2,):
         s.stats()
         s.step(2)
         s.sync()
+    # host-streamed, two steps per round trip (somier_stream_run2), odd count
+    with P.SomierStream(P.Spread([0], 1, n[0] - 2, chunk=3), sp, buffers=2) as st:
+        X, V = st.generate()
+        st.run2(X, V, np.zeros_like(X), np.zeros_like(V), 3)
 print("sanitize case ok")

@@ -293,47 +293,82 @@ def pcie_rates(local, nbytes=1 << 30):
     return res
 
 
-def e2e_stream(n, params, local, a):
-    """End to end through the public C ABI with HOST buffers: somier_stream_run
-    maps every chunk to the GPU (X with halo planes, V), runs the fused step and
-    maps X_{t+1}, V back, each step -- the paper's `target spread` cycle with
-    double buffering (3 device slots, 3 streams) and chunk-level dependencies
-    between steps (the paper's future-work `depend`) instead
-    of a barrier per step. Wall-clock timed: every host<->device copy and the
-    read-back of every step's stats is inside the timed region."""
-    import numpy as np
+def e2e_stream(n, params, local, a, two_step):
+    """End to end through the public C ABI with HOST buffers: the state lives in
+    pinned host memory and every launch maps each chunk to the GPU (X with halo
+    planes, V), runs the fused step(s) and maps X, V back -- the paper's `target
+    spread` cycle with double buffering (3 device slots, 3 streams) and
+    chunk-level dependencies between launches (the paper's future-work
+    `depend`) instead of a barrier per step. Wall-clock
+    timed: every host<->device copy and the read-back of every launch's stats
+    is inside the timed region.
+    two_step (the resident kernel is K1_TB2): somier_stream_run2, two steps per
+    round trip (X halo 2, V halo 1, V double-buffered on the host), stats after
+    every second step as on the resident handle; the one-step cycle
+    (somier_stream_run, every step's stats) is measured too and reported
+    beside it."""
     import torch
 
     import paper_conf_ipps_torresft22_b200 as P
 
     chunk = a.stream_chunk
     st = P.SomierStream(P.Spread([local], 1, n[0] - 2, chunk=chunk), params, buffers=3)
-    grids = [torch.empty(tuple(n), dtype=torch.float64, pin_memory=True) for _ in range(9)]
-    X, V, XN = [g.data_ptr() for g in grids[0:3]], [g.data_ptr() for g in grids[3:6]], \
-        [g.data_ptr() for g in grids[6:9]]
+    grids = [torch.empty(tuple(n), dtype=torch.float64, pin_memory=True) for _ in range(12 if two_step else 9)]
+    ptr = [g.data_ptr() for g in grids]
+    X, V, XN = ptr[0:3], ptr[3:6], ptr[6:9]
     st.generate_ptrs(X + V)
-    st.run_ptrs(X, V, XN, 1)  # warm-up step
-    X, XN = XN, X
-    k = max(1, a.e2e_steps)
-    t0 = time.perf_counter()
-    stats = st.run_ptrs(X, V, XN, k)[-1]
-    wall = time.perf_counter() - t0
-    tr = st.traffic()
+    k = max(2, a.e2e_steps + (a.e2e_steps & 1))
+    rates = pcie_rates(local)
+
+    def one_step():
+        st.run_ptrs(X, V, XN, 1)  # warm-up step
+        t0 = time.perf_counter()
+        stats = st.run_ptrs(XN, V, X, k)[-1]
+        wall = time.perf_counter() - t0
+        tr = st.traffic()
+        b = tr["h2d_bytes"] + tr["d2h_bytes"]
+        return {"value": interior(n) * k / wall, "h2d_bytes_per_step": tr["h2d_bytes"],
+                "d2h_bytes_per_step": tr["d2h_bytes"] + 88, "steps": k, "wall_s": wall,
+                "frac_pcie": b / (wall / k) / 1e9 / rates["bidir_total"], "achieved_gbs": b / (wall / k) / 1e9,
+                "last_step_vmax": stats.vmax}
+
+    def two_steps():
+        VN = ptr[9:12]
+        st.run2_ptrs(X, V, XN, VN, 2)  # warm-up launch
+        t0 = time.perf_counter()
+        stats = st.run2_ptrs(XN, VN, X, V, k)[-1]
+        wall = time.perf_counter() - t0
+        tr = st.traffic2()
+        b = (tr["h2d_bytes"] + tr["d2h_bytes"]) / 2
+        return {"value": interior(n) * k / wall, "h2d_bytes_per_step": tr["h2d_bytes"] // 2,
+                "d2h_bytes_per_step": (tr["d2h_bytes"] + 88) // 2, "steps": k, "wall_s": wall,
+                "frac_pcie": b / (wall / k) / 1e9 / rates["bidir_total"], "achieved_gbs": b / (wall / k) / 1e9,
+                "last_step_vmax": stats.vmax}
+
+    r1 = one_step()
+    r2 = two_steps() if two_step else None
     st.close()
     del grids
-    rates = pcie_rates(local)
-    bytes_step = tr["h2d_bytes"] + tr["d2h_bytes"]
-    return {"value": interior(n) * k / wall, "unit": UNIT, "h2d_bytes_per_step": tr["h2d_bytes"],
-            "d2h_bytes_per_step": tr["d2h_bytes"] + 88, "steps": k, "wall_s": wall,
-            "cycle": "somier_stream_run on pinned host grids: per chunk of %d planes map(to: X[start-1:size+2], "
-                     "V[start:size]) -> fused K1 -> map(from: X[start:size], V[start:size]); 3 device slots, "
-                     "H2D/K1/D2H overlapped, steps chained by per-chunk events (no barrier per step); every "
-                     "step's stats read back" % chunk,
-            "roofline": {"bound": "pcie", "achieved_gbs": bytes_step / (wall / k) / 1e9,
-                         "peak_gbs_bidir_measured": rates["bidir_total"], "h2d_gbs": rates["h2d"],
-                         "d2h_gbs": rates["d2h"],
-                         "frac": bytes_step / (wall / k) / 1e9 / rates["bidir_total"]},
-            "last_step_vmax": stats.vmax}
+    r = r2 if two_step else r1
+    cyc1 = ("somier_stream_run on pinned host grids: per chunk of %d planes map(to: X[start-1:size+2], "
+            "V[start:size]) -> fused K1 -> map(from: X[start:size], V[start:size]); 3 device slots, H2D/K1/D2H "
+            "overlapped, steps chained by per-chunk events (no barrier per step); every step's stats read back" % chunk)
+    cyc2 = ("somier_stream_run2 on pinned host grids: per chunk of %d planes map(to: X[start-2:size+4], "
+            "V[start-1:size+2]) -> K1_TB2 (two steps) -> map(from: X[start:size], V[start:size]) into the other "
+            "host buffers; 3 device slots, H2D/K1/D2H overlapped, launches chained by per-chunk events; every "
+            "launch's stats (each second step) read back" % chunk)
+    out = {"value": r["value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d_bytes_per_step"],
+           "d2h_bytes_per_step": r["d2h_bytes_per_step"], "steps": k, "wall_s": r["wall_s"],
+           "cycle": cyc2 if two_step else cyc1,
+           "roofline": {"bound": "pcie", "achieved_gbs": r["achieved_gbs"],
+                        "peak_gbs_bidir_measured": rates["bidir_total"], "h2d_gbs": rates["h2d"],
+                        "d2h_gbs": rates["d2h"], "frac": r["frac_pcie"]},
+           "last_step_vmax": r["last_step_vmax"]}
+    if two_step:
+        out["one_step_cycle"] = {"value": r1["value"], "h2d_bytes_per_step": r1["h2d_bytes_per_step"],
+                                 "d2h_bytes_per_step": r1["d2h_bytes_per_step"], "frac_pcie": r1["frac_pcie"],
+                                 "cycle": cyc1}
+    return out
 
 
 def sustained_copy(device, stream, gib=6, iters=30):
@@ -483,14 +518,16 @@ def run_ours(a):
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()
 
-    # end-to-end through the public API with pinned host buffers: per step,
-    # map(to) the whole state (X with halos, V), one step, read the centers
-    # result and map(from) the state -- the paper's One Buffer cycle, in core.
+    # end-to-end through the public API with pinned host buffers. N = 1: the
+    # host-streamed cycle (e2e_stream; two steps per round trip when the
+    # resident kernel is K1_TB2). N > 1: per step, map(to) the whole state (X
+    # with halos, V), one step, read the centers result and map(from) the
+    # state -- the paper's One Buffer cycle, in core.
     e2e = None
     if not a.no_e2e and not multi:
         s.close()  # free the resident grid: the streamed mode needs only a few chunk buffers
         torch.cuda.empty_cache()
-        e2e = e2e_stream(n, params, local, a)
+        e2e = e2e_stream(n, params, local, a, two_step=(in_use == P.K1_TB2))
     elif not a.no_e2e:
         shape = tuple(n)
         host = [torch.empty(shape, dtype=torch.float64, pin_memory=True) for _ in range(6)]

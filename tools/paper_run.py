@@ -8,7 +8,9 @@ PAPER.md:669-672) were 1058.9 s on 1 V100 and 502.0 s on 4 V100.
 
 mode run (default): somier_stream_run, steps chained by per-chunk events (the
 paper's future-work `depend`); step: somier_stream_step, a barrier per step
-(the paper's taskgroup).
+(the paper's taskgroup); run2: somier_stream_run2, two steps per host round
+trip (12 host grids -- the paper's 154.5 GiB at 1200^3; refused if the host
+has not that much memory available).
 """
 import json
 import os
@@ -25,11 +27,22 @@ steps = int(sys.argv[2]) if len(sys.argv) > 2 else 31
 chunk = int(sys.argv[3]) if len(sys.argv) > 3 else 64
 buffers = int(sys.argv[4]) if len(sys.argv) > 4 else 3
 mode = sys.argv[5] if len(sys.argv) > 5 else "run"
+ngrids = 12 if mode == "run2" else 9
+need = ngrids * n ** 3 * 8
+avail = 0
+with open("/proc/meminfo") as f:
+    for line in f:
+        if line.startswith("MemAvailable:"):
+            avail = int(line.split()[1]) * 1024
+if avail < need * 1.1 + (16 << 30):
+    print(json.dumps({"n": n, "mode": mode, "skipped": "host memory: need %.1f GiB pinned, %.1f GiB available" % (
+        need / 2 ** 30, avail / 2 ** 30)}))
+    sys.exit(0)
 t_all = time.perf_counter()
 params = P.SomierParams(n=(n, n, n), seed=42)
 st = P.SomierStream(P.Spread([0], 1, n - 2, chunk=chunk), params, buffers=buffers)
 t0 = time.perf_counter()
-grids = [torch.empty((n, n, n), dtype=torch.float64, pin_memory=True) for _ in range(9)]
+grids = [torch.empty((n, n, n), dtype=torch.float64, pin_memory=True) for _ in range(ngrids)]
 t_pin = time.perf_counter() - t0
 X, V, XN = [g.data_ptr() for g in grids[0:3]], [g.data_ptr() for g in grids[3:6]], [g.data_ptr() for g in grids[6:9]]
 t0 = time.perf_counter()
@@ -40,6 +53,10 @@ t0 = time.perf_counter()
 if mode == "run":
     stats = st.run_ptrs(X, V, XN, steps)[-1]
     per = [(time.perf_counter() - t0) / steps]
+elif mode == "run2":
+    VN = [g.data_ptr() for g in grids[9:12]]
+    stats = st.run2_ptrs(X, V, XN, VN, steps)[-1]
+    per = [(time.perf_counter() - t0) / steps]
 else:
     for _ in range(steps):
         a = time.perf_counter()
@@ -48,7 +65,11 @@ else:
         X, XN = XN, X
 t_steps = time.perf_counter() - t0
 tr = st.traffic()
-out = {"n": n, "steps": steps, "chunk": chunk, "buffers": buffers, "mode": mode, "host_state_gib": 9 * n ** 3 * 8 / 2 ** 30,
+if mode == "run2":  # bytes of one two-step launch, per step
+    t2 = st.traffic2()
+    tr = {"h2d_bytes": t2["h2d_bytes"] / 2, "d2h_bytes": t2["d2h_bytes"] / 2}
+out = {"n": n, "steps": steps, "chunk": chunk, "buffers": buffers, "mode": mode,
+       "host_state_gib": ngrids * n ** 3 * 8 / 2 ** 30,
        "pin_s": t_pin, "generate_s": t_gen, "steps_s": t_steps, "s_per_step": t_steps / steps,
        "per_step_min_max": [min(per), max(per)], "node_updates_per_s": (n - 2) ** 3 * steps / t_steps,
        "h2d_gb_per_step": tr["h2d_bytes"] / 1e9, "d2h_gb_per_step": tr["d2h_bytes"] / 1e9,

@@ -308,6 +308,31 @@ spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double
                                  double* vz, double* xn, double* yn, double* zn, double* vxn, double* vyn,
                                  double* vzn, int64_t nsteps, somier_stats_t* stats);
 
+/*
+ * somier_stream_run_blocked -- as somier_stream_run2 with `steps_per_trip` = s
+ * steps per host round trip (1 <= s <= 256; s = 2 moves the same bytes as
+ * somier_stream_run2): per chunk map(to: X[start-s : size+2s],
+ * V[start-s : size+2s]) (clipped to the grid), ceil(s/2) K1_TB2 launches over
+ * regions that shrink by two planes per side per launch down to the chunk
+ * itself (an odd s ends with a one-step launch), map(from: X[start : size],
+ * V[start : size]). Host<->device bytes per node-update fall as ~1/s while
+ * the device recomputes the overlap (a chunk of S planes computes ~S + s
+ * planes per step on average). Buffers alternate per trip as in run2 (the
+ * final state is in the first buffers if the number of trips ceil(nsteps/s)
+ * is even); stats: NULL or ceil(nsteps/s) entries, one per trip.
+ * Device memory: `buffers` x 2 x (X and V of max_chunk + 2s + 2 planes) per
+ * device, allocated on first use. Bit-identical to somier_stream_run.
+ * Errors: EINVAL, ENOMEM, ECUDA.
+ */
+spread_status somier_stream_run_blocked(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                        double* vz, double* xn, double* yn, double* zn, double* vxn, double* vyn,
+                                        double* vzn, int64_t nsteps, int64_t steps_per_trip, somier_stats_t* stats);
+
+/* Bytes moved host->device and device->host by one trip of
+ * somier_stream_run_blocked with s steps. */
+spread_status somier_stream_traffic_blocked(somier_stream_t h, int64_t steps_per_trip, int64_t* h2d_bytes,
+                                            int64_t* d2h_bytes);
+
 /* Bytes moved host->device and device->host by one somier_stream_step (one
  * step of somier_stream_run), and K1 launches so far. */
 spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches);

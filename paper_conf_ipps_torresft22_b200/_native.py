@@ -117,6 +117,9 @@ SIGNATURES = [
     ("somier_stream_traffic", ctypes.c_int, [_VP, _I64P, _I64P, _I64P]),
     ("somier_stream_run2", ctypes.c_int, [_VP] + [_DP] * 12 + [ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
     ("somier_stream_traffic2", ctypes.c_int, [_VP, _I64P, _I64P]),
+    ("somier_stream_run_blocked", ctypes.c_int,
+     [_VP] + [_DP] * 12 + [ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
+    ("somier_stream_traffic_blocked", ctypes.c_int, [_VP, ctypes.c_int64, _I64P, _I64P]),
     ("somier_stream_destroy", ctypes.c_int, [_VP]),
 ]
 

@@ -59,10 +59,24 @@ struct ChunkEvents {
     cudaEvent_t d2h[2] = {nullptr, nullptr};
 };
 
+// Device buffers of a blocked round trip (somier_stream_run_blocked): the
+// chunk's X_t planes [start-s-1, start+size+s+1) and V_t planes
+// [start-s, start+size+s) for s steps per trip, plus a second X and V buffer
+// the launches ping-pong through. Allocated on first use.
+struct DeepSlot {
+    void* base = nullptr;
+    double *xa = nullptr, *xb = nullptr, *va = nullptr, *vb = nullptr;
+    int64_t planes = 0;  // X planes per buffer (V: planes - 2)
+    cudaEvent_t comp_done = nullptr, d2h_done = nullptr;
+    bool used = false;
+};
+
 struct Dev {
     int pos = 0, device = 0;
     cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
     std::vector<Slot> slots;
+    std::vector<DeepSlot> deep;
+    paper::StatsAccum* scratch_acc = nullptr;  // stats of the widened intermediate launches (discarded)
     void* acc_base = nullptr;  // StatsAccum[acc_steps][2]: per step, chunk sums and fixed end planes
     int64_t acc_steps = 0;
     std::vector<int64_t> chunks;
@@ -113,6 +127,12 @@ void destroy_all(somier_stream_t h) {
                 if (e) cudaEventDestroy(e);
             if (sl.base) cudaFree(sl.base);
         }
+        for (auto& sl : d.deep) {
+            for (cudaEvent_t e : {sl.comp_done, sl.d2h_done})
+                if (e) cudaEventDestroy(e);
+            if (sl.base) cudaFree(sl.base);
+        }
+        if (d.scratch_acc) cudaFree(d.scratch_acc);
         if (d.acc_base) cudaFree(d.acc_base);
         for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
             if (s) cudaStreamDestroy(s);
@@ -393,6 +413,191 @@ spread_status stream_run_tb2(somier_stream_t h, double* const X[3], double* cons
     return stats ? gather_stats(h, nl, steps.data(), stats) : SPREAD_OK;
 }
 
+// (Re)allocate every device's deep slots for `planes` X planes per buffer.
+spread_status ensure_deep(somier_stream_t h, int64_t planes) {
+    const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        if (!d.scratch_acc) S_TRY(h, cudaMalloc(&d.scratch_acc, sizeof(paper::StatsAccum)));
+        if (!d.deep.empty() && d.deep[0].planes >= planes) continue;
+        S_TRY(h, cudaDeviceSynchronize());
+        for (auto& sl : d.deep)
+            if (sl.base) S_TRY(h, cudaFree(sl.base));
+        d.deep.resize(d.slots.size());
+        const size_t xb = round_up(plane * (size_t)planes, 4096), vb = round_up(plane * (size_t)(planes - 2), 4096);
+        for (auto& sl : d.deep) {
+            sl.base = nullptr;
+            S_TRY(h, cudaMalloc(&sl.base, 2 * xb + 2 * vb));
+            // zeroed once: the fixed face nodes of V are never written by K1_TB2
+            S_TRY(h, cudaMemset(sl.base, 0, 2 * xb + 2 * vb));
+            sl.xa = (double*)sl.base;
+            sl.xb = (double*)((char*)sl.base + xb);
+            sl.va = (double*)((char*)sl.base + 2 * xb);
+            sl.vb = (double*)((char*)sl.base + 2 * xb + vb);
+            sl.planes = planes;
+            sl.used = false;
+            for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
+                if (!*pe) S_TRY(h, cudaEventCreateWithFlags(pe, cudaEventDisableTiming));
+        }
+    }
+    return SPREAD_OK;
+}
+
+// Chunks within `depth` planes of chunk c (either way).
+void reach_range(const somier_stream_s* h, const paper::ChunkInfo& ci, int64_t depth, int64_t* c_lo, int64_t* c_hi) {
+    const int64_t n0 = h->p.n[0];
+    *c_lo = h->spread.chunk_of(std::max<int64_t>(1, ci.start - depth));
+    *c_hi = h->spread.chunk_of(std::min<int64_t>(n0 - 2, ci.start + ci.size + depth - 1));
+}
+
+// Trip k of a blocked run: every chunk maps in X_t and V_t planes
+// [start-s, start+size+s) (clipped to the grid), advances s
+// steps with ceil(s/2) K1_TB2 launches over regions that shrink by two planes
+// per side per launch (the last one is the chunk itself; an odd s ends with a
+// one-step launch), and maps X_{t+s}, V_{t+s} of its planes out into (XN, VN).
+spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
+                                     double* const VN[3], int64_t k, int64_t s, bool chained) {
+    const int64_t n0 = h->p.n[0];
+    const int64_t nch = h->spread.nchunks;
+    const int64_t ps = h->geom.plane_stride();
+    const int par = (int)(k & 1), prev = par ^ 1;
+    const int64_t nl = s / 2 + (s & 1);
+    for (int64_t c = 0; c < nch; c++) {
+        const paper::ChunkInfo ci = h->spread.chunk_info(c);
+        Dev& d = h->devs[ci.pos];
+        const size_t m = (size_t)(c / (int64_t)h->devs.size());
+        DeepSlot& sl = d.deep[m % d.deep.size()];
+        const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
+        ChunkEvents& ev = h->ev[(size_t)c];
+        int64_t c_lo, c_hi;
+        reach_range(h, ci, s, &c_lo, &c_hi);
+        // global plane of raw plane 0 of the X / V buffers: one plane of slack
+        // beyond the s-plane halo on each side (a one-step launch still reads
+        // the deep layout's outer ring plane, whose values it does not use)
+        const int64_t x0 = ci.start - s - 1, v0 = ci.start - s;
+        S_TRY(h, cudaSetDevice(d.device));
+        if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
+        if (chained)
+            for (int64_t nb = c_lo; nb <= c_hi; nb++)
+                S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
+        const int64_t xlo = std::max<int64_t>(0, ci.start - s), xhi = std::min<int64_t>(n0, ci.start + ci.size + s);
+        const int64_t vlo = std::max<int64_t>(0, ci.start - s), vhi = std::min<int64_t>(n0, ci.start + ci.size + s);
+        paper::SlabGeom g = geom_of(h, ci);
+        for (int q = 0; q < 3; q++) {
+            S_TRY(h, paper::copy_slab_planes(g, sl.xa, q, xlo - x0, X[q], xlo, xhi - xlo, cudaMemcpyHostToDevice,
+                                             d.s_h2d));
+            S_TRY(h, paper::copy_slab_planes(g, sl.va, q, vlo - v0, V[q], vlo, vhi - vlo,
+                                             cudaMemcpyHostToDevice, d.s_h2d));
+        }
+        S_TRY(h, cudaEventRecord(ev.h2d[par], d.s_h2d));
+        S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
+        // the fixed face nodes of every output plane (K1_TB2 writes the moving nodes only)
+        S_TRY(h, cudaMemcpyAsync(sl.xb + (xlo - x0) * ps, sl.xa + (xlo - x0) * ps,
+                                 (size_t)((xhi - xlo) * ps) * sizeof(double), cudaMemcpyDeviceToDevice, d.s_comp));
+        paper::StatsAccum* acc = d.acc(k);
+        double* xv_one = sl.xa + (ci.start - 1 - x0) * ps;  // one-step view: raw plane 0 = start - 1
+        if (first) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, 0, 1, acc + 1, d.s_comp));
+        if (last) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, ci.size + 1, 1, acc + 1, d.s_comp));
+        S_TRY(h, paper::launch_kface_stats(xv_one, g, 1, ci.size, acc + 1, d.s_comp));
+        int64_t remaining = s;
+        double *xin = sl.xa, *xout = sl.xb, *vin = sl.va, *vout = sl.vb;
+        for (int64_t j = 0; j < nl; j++) {
+            const bool two = remaining >= 2;
+            const int64_t w = remaining - (two ? 2 : 1);  // planes this launch's region extends beyond the chunk
+            paper::SlabGeom gj = g;
+            gj.start = std::max<int64_t>(1, ci.start - w);
+            gj.size = std::min<int64_t>(n0 - 1, ci.start + ci.size + w) - gj.start;
+            double* xs = xin + (gj.start - 2 - x0) * ps;       // raw plane 0 = region start - 2
+            double* vs = vin + (gj.start - 1 - v0) * ps;        // raw plane 0 = region start - 1
+            alignas(64) CUtensorMap mx, mv;
+            spread_status st = paper::encode_slab_tmap(&mx, gj, xs, gj.size + 4, paper::kTB2XBoxK, paper::kTB2XBoxJ);
+            if (st != SPREAD_OK) return st;
+            st = paper::encode_slab_tmap(&mv, gj, vs, gj.size + 2, paper::kTB2VBoxK, paper::kTB2VBoxJ);
+            if (st != SPREAD_OK) return st;
+            paper::StepArgs a;
+            std::memset(&a, 0, sizeof a);
+            a.x_cur = xs;
+            a.v = vs;
+            a.g = gj;
+            a.K = h->p.k_spring;
+            a.L = h->p.rest_len;
+            a.M = h->p.mass;
+            a.dt = h->p.dt;
+            a.acc = j + 1 == nl ? acc : d.scratch_acc;
+            a.tmap_x_cur = &mx;
+            a.tmap_v = &mv;
+            paper::Tb2Out o;
+            std::memset(&o, 0, sizeof o);
+            o.x_out = xout + (gj.start - 2 - x0) * ps;
+            o.v_out = vout + (gj.start - 1 - v0) * ps;
+            o.two = two;
+            S_TRY(h, paper::launch_k1_tb2(a, o, h->p.mass == 1.0, d.s_comp));
+            h->launches++;
+            remaining -= two ? 2 : 1;
+            std::swap(xin, xout);
+            std::swap(vin, vout);
+        }
+        S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
+        S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
+        if (chained)
+            for (int64_t nb = c_lo; nb <= c_hi; nb++)
+                if (nb != c) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)nb].h2d[prev], 0));
+        // after the last launch the state is in (xin, vin)
+        for (int q = 0; q < 3; q++) {
+            S_TRY(h, paper::copy_slab_planes(g, xin, q, ci.start - x0, XN[q], ci.start, ci.size,
+                                             cudaMemcpyDeviceToHost, d.s_d2h));
+            S_TRY(h, paper::copy_slab_planes(g, vin, q, ci.start - v0, VN[q], ci.start, ci.size,
+                                             cudaMemcpyDeviceToHost, d.s_d2h));
+            if (first) {
+                S_TRY(h, paper::copy_slab_planes(g, sl.xa, q, 0 - x0, XN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
+                S_TRY(h, paper::copy_slab_planes(g, sl.va, q, 0 - v0, VN[q], 0, 1, cudaMemcpyDeviceToHost,
+                                                 d.s_d2h));
+            }
+            if (last) {
+                S_TRY(h, paper::copy_slab_planes(g, sl.xa, q, n0 - 1 - x0, XN[q], n0 - 1, 1, cudaMemcpyDeviceToHost,
+                                                 d.s_d2h));
+                S_TRY(h, paper::copy_slab_planes(g, sl.va, q, n0 - 1 - v0, VN[q], n0 - 1, 1,
+                                                 cudaMemcpyDeviceToHost, d.s_d2h));
+            }
+        }
+        S_TRY(h, cudaEventRecord(ev.d2h[par], d.s_d2h));
+        S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
+        sl.used = true;
+    }
+    return SPREAD_OK;
+}
+
+// Blocked run: trips of s steps (the last one shorter if s does not divide
+// nsteps), alternating (X, V) -> (XN, VN) -> (X, V) ...; stats[k] (if non-NULL)
+// receives the statistics after trip k. One host barrier at the end.
+spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
+                                 double* const VN[3], int64_t nsteps, int64_t s, somier_stats_t* stats) {
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    const int64_t ntrips = (nsteps + s - 1) / s;
+    spread_status st = ensure_acc(h, ntrips);
+    if (st != SPREAD_OK) return st;
+    st = ensure_deep(h, h->max_chunk + 2 * s + 2);
+    if (st != SPREAD_OK) return st;
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * (size_t)ntrips * sizeof(paper::StatsAccum), d.s_comp));
+    }
+    std::vector<int64_t> steps((size_t)ntrips);
+    for (int64_t k = 0; k < ntrips; k++) {
+        const int64_t sk = std::min<int64_t>(s, nsteps - k * s);
+        steps[(size_t)k] = h->step + k * s + sk;
+        st = (k & 1) ? enqueue_stream_blocked(h, XN, VN, X, V, k, sk, k > 0)
+                     : enqueue_stream_blocked(h, X, V, XN, VN, k, sk, k > 0);
+        if (st != SPREAD_OK) return st;
+    }
+    st = sync_devs(h);
+    if (st != SPREAD_OK) return st;
+    h->step += nsteps;
+    return stats ? gather_stats(h, ntrips, steps.data(), stats) : SPREAD_OK;
+}
+
 // Run nsteps steps from (X, V), alternating X -> XN -> X ...; stats[t] (if
 // non-NULL) receives the statistics after step t. One host barrier at the end.
 spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
@@ -606,6 +811,44 @@ spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double
     double* V[3] = {vx, vy, vz};
     double* VN[3] = {vxn, vyn, vzn};
     return stream_run_tb2(h, X, V, XN, VN, nsteps, stats);
+}
+
+spread_status somier_stream_run_blocked(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
+                                        double* vz, double* xn, double* yn, double* zn, double* vxn, double* vyn,
+                                        double* vzn, int64_t nsteps, int64_t steps_per_trip, somier_stats_t* stats) {
+    if (!h || !x || !y || !z || !vx || !vy || !vz || !xn || !yn || !zn || !vxn || !vyn || !vzn)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run_blocked: NULL argument");
+    if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run_blocked: nsteps %lld < 0", (long long)nsteps);
+    if (steps_per_trip < 1 || steps_per_trip > 256)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run_blocked: steps_per_trip %lld outside [1, 256]",
+                   (long long)steps_per_trip);
+    if (x == xn || y == yn || z == zn || vx == vxn || vy == vyn || vz == vzn)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_run_blocked: the two X or the two V buffers alias");
+    if (nsteps == 0) return SPREAD_OK;
+    double* X[3] = {x, y, z};
+    double* XN[3] = {xn, yn, zn};
+    double* V[3] = {vx, vy, vz};
+    double* VN[3] = {vxn, vyn, vzn};
+    return stream_run_blocked(h, X, V, XN, VN, nsteps, steps_per_trip, stats);
+}
+
+spread_status somier_stream_traffic_blocked(somier_stream_t h, int64_t steps_per_trip, int64_t* h2d_bytes,
+                                            int64_t* d2h_bytes) {
+    if (!h || steps_per_trip < 1) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_traffic_blocked: bad argument");
+    const int64_t n0 = h->p.n[0], s = steps_per_trip;
+    const int64_t plane = 3 * h->p.n[1] * h->p.n[2] * (int64_t)sizeof(double);
+    int64_t in = 0, outb = 0;
+    for (int64_t c = 0; c < h->spread.nchunks; c++) {
+        const paper::ChunkInfo ci = h->spread.chunk_info(c);
+        const int64_t xp = std::min<int64_t>(n0, ci.start + ci.size + s) - std::max<int64_t>(0, ci.start - s);
+        const int64_t vp = std::min<int64_t>(n0, ci.start + ci.size + s) - std::max<int64_t>(0, ci.start - s);
+        in += plane * (xp + vp);
+        outb += 2 * plane * ci.size;
+    }
+    outb += 4 * plane;  // fixed end planes of X and V
+    if (h2d_bytes) *h2d_bytes = in;
+    if (d2h_bytes) *d2h_bytes = outb;
+    return SPREAD_OK;
 }
 
 spread_status somier_stream_traffic2(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes) {

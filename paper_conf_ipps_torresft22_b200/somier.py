@@ -327,3 +327,26 @@ class SomierStream:
         a, b = ctypes.c_int64(), ctypes.c_int64()
         N.check(N.lib().somier_stream_traffic2(self._h, ctypes.byref(a), ctypes.byref(b)), "somier_stream_traffic2")
         return {"h2d_bytes": a.value, "d2h_bytes": b.value}
+
+    def run_blocked(self, X, V, XN, VN, nsteps: int, steps_per_trip: int, stats: bool = True):
+        """nsteps steps, `steps_per_trip` per host round trip
+        (somier_stream_run_blocked); buffers alternate per trip as in run2.
+        Returns the Stats after each trip (or None)."""
+        return self.run_blocked_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]],
+                                     [VN[0], VN[1], VN[2]], nsteps, steps_per_trip, stats)
+
+    def run_blocked_ptrs(self, X, V, XN, VN, nsteps: int, steps_per_trip: int, stats: bool = True):
+        s = int(steps_per_trip)
+        nt = -(-int(nsteps) // max(1, s))
+        out = (N.somier_stats_t * max(1, nt))() if stats else None
+        N.check(N.lib().somier_stream_run_blocked(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
+                                                  *[_dptr(g) for g in XN], *[_dptr(g) for g in VN], int(nsteps), s,
+                                                  out), "somier_stream_run_blocked")
+        return [Stats.from_c(out[k]) for k in range(nt)] if stats else None
+
+    def traffic_blocked(self, steps_per_trip: int):
+        """Host<->device bytes of one trip of run_blocked with steps_per_trip steps."""
+        a, b = ctypes.c_int64(), ctypes.c_int64()
+        N.check(N.lib().somier_stream_traffic_blocked(self._h, int(steps_per_trip), ctypes.byref(a), ctypes.byref(b)),
+                "somier_stream_traffic_blocked")
+        return {"h2d_bytes": a.value, "d2h_bytes": b.value}

@@ -218,3 +218,58 @@ def test_stream_run2_matches_run_and_resident():
     assert np.array_equal(XN2, Xr) and np.array_equal(VN2, Vr)
     # per node-update, run2 moves about half the host<->device bytes of run
     assert (h2["h2d_bytes"] + h2["d2h_bytes"]) / 2 < 0.6 * (h1["h2d_bytes"] + h1["d2h_bytes"])
+
+
+@pytest.mark.parametrize("devices,spread_kw,buffers,nsteps,spt", [
+    ([0], {"chunk": 3}, 2, 9, 4), ([0], {"chunk": 5}, 1, 10, 8), ([0, 1, 2], {"chunk": 2}, 2, 11, 3),
+    ([0, 1], {"sizes": [1, 6, 2, 1, 4]}, 3, 12, 6), ([0], {"chunk": 100}, 2, 7, 5), ([0], {"chunk": 1}, 3, 5, 1),
+    ([0, 1, 2, 3], {"chunk": 0}, 2, 13, 13), ([0], {"sizes": [1, 1, 12]}, 2, 6, 2), ([0], {"chunk": 4}, 2, 20, 16)])
+def test_stream_run_blocked_s_steps_per_round_trip(devices, spread_kw, buffers, nsteps, spt):
+    """somier_stream_run_blocked: s steps per host round trip (halo s, regions
+    shrinking two planes per side per K1_TB2 launch, odd s ending with a
+    one-step launch, halos reaching several one-plane chunks away, s larger
+    than the grid's chunks); every trip's stats and the final state equal the
+    oracle's bit for bit."""
+    n = (16, 13, 37)
+    sp = P.SomierParams(n=n, seed=6)
+    if "sizes" in spread_kw:
+        spread = P.Spread.with_sizes(devices, 1, n[0] - 2, spread_kw["sizes"])
+    else:
+        spread = P.Spread(devices, 1, n[0] - 2, chunk=spread_kw["chunk"])
+    with P.SomierStream(spread, sp, buffers=buffers, cuda_devices=[0] * len(devices)) as s:
+        X0, V0 = s.generate()
+        X, V, XN, VN = _pinned_like(X0), _pinned_like(V0), _pinned_like(X0), _pinned_like(V0)
+        X[...] = X0
+        V[...] = V0
+        XN[...] = np.nan
+        VN[...] = np.nan
+        stats = s.run_blocked(X, V, XN, VN, nsteps, spt)
+    nt = -(-nsteps // spt)
+    fX, fV = (X, V) if nt % 2 == 0 else (XN, VN)
+    ref = O.init(_op(sp))
+    done = 0
+    for k in range(nt):
+        for _ in range(min(spt, nsteps - done)):
+            ref, rst = O.step(ref)
+            done += 1
+        assert stats[k].step == done
+        assert stats[k].sums == rst.sums and stats[k].vmax2_bits == rst.vmax2_bits
+    assert np.array_equal(fX, ref.X) and np.array_equal(fV, ref.V)
+
+
+def test_stream_run_blocked_matches_run_at_size_and_traffic():
+    """A larger grid through 8-step trips (nonunit mass) equals somier_stream_run;
+    bytes per node-update fall with the trip length."""
+    sp = P.SomierParams(n=(70, 40, 66), seed=2, mass=0.8)
+    with P.SomierStream(P.Spread([0], 1, 68, chunk=16), sp, buffers=3) as s:
+        X, V = s.generate()
+        X2, V2, XN, XN2, VN2 = X.copy(), V.copy(), np.zeros_like(X), np.zeros_like(X), np.zeros_like(V)
+        st1 = s.run(X, V, XN, 16)
+        st2 = s.run_blocked(X2, V2, XN2, VN2, 16, 8)
+        t2 = s.traffic_blocked(2)
+        t8 = s.traffic_blocked(8)
+        r2 = s.traffic2()
+    assert st1[-1].sums == st2[-1].sums and st1[-1].vmax2_bits == st2[-1].vmax2_bits
+    assert np.array_equal(X, X2) and np.array_equal(V, V2)  # 2 trips: back in the first buffers
+    assert (t8["h2d_bytes"] + t8["d2h_bytes"]) / 8 < 0.5 * (t2["h2d_bytes"] + t2["d2h_bytes"]) / 2
+    assert t2["d2h_bytes"] == r2["d2h_bytes"]

@@ -10,7 +10,8 @@ mode run (default): somier_stream_run, steps chained by per-chunk events (the
 paper's future-work `depend`); step: somier_stream_step, a barrier per step
 (the paper's taskgroup); run2: somier_stream_run2, two steps per host round
 trip (12 host grids -- the paper's 154.5 GiB at 1200^3; refused if the host
-has not that much memory available).
+has not that much memory available); blockedS (e.g. blocked8):
+somier_stream_run_blocked with S steps per round trip (12 host grids).
 """
 import json
 import os
@@ -27,7 +28,7 @@ steps = int(sys.argv[2]) if len(sys.argv) > 2 else 31
 chunk = int(sys.argv[3]) if len(sys.argv) > 3 else 64
 buffers = int(sys.argv[4]) if len(sys.argv) > 4 else 3
 mode = sys.argv[5] if len(sys.argv) > 5 else "run"
-ngrids = 12 if mode == "run2" else 9
+ngrids = 12 if (mode == "run2" or mode.startswith("blocked")) else 9
 need = ngrids * n ** 3 * 8
 avail = 0
 with open("/proc/meminfo") as f:
@@ -57,6 +58,10 @@ elif mode == "run2":
     VN = [g.data_ptr() for g in grids[9:12]]
     stats = st.run2_ptrs(X, V, XN, VN, steps)[-1]
     per = [(time.perf_counter() - t0) / steps]
+elif mode.startswith("blocked"):
+    VN = [g.data_ptr() for g in grids[9:12]]
+    stats = st.run_blocked_ptrs(X, V, XN, VN, steps, int(mode[7:]))[-1]
+    per = [(time.perf_counter() - t0) / steps]
 else:
     for _ in range(steps):
         a = time.perf_counter()
@@ -68,6 +73,10 @@ tr = st.traffic()
 if mode == "run2":  # bytes of one two-step launch, per step
     t2 = st.traffic2()
     tr = {"h2d_bytes": t2["h2d_bytes"] / 2, "d2h_bytes": t2["d2h_bytes"] / 2}
+elif mode.startswith("blocked"):  # bytes of one trip, per step (full trips)
+    S = int(mode[7:])
+    t2 = st.traffic_blocked(S)
+    tr = {"h2d_bytes": t2["h2d_bytes"] / S, "d2h_bytes": t2["d2h_bytes"] / S}
 out = {"n": n, "steps": steps, "chunk": chunk, "buffers": buffers, "mode": mode,
        "host_state_gib": ngrids * n ** 3 * 8 / 2 ** 30,
        "pin_s": t_pin, "generate_s": t_gen, "steps_s": t_steps, "s_per_step": t_steps / steps,

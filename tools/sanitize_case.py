@@ -39,4 +39,5 @@ for kern in (P.K1_TB2,):
     with P.SomierStream(P.Spread([0], 1, n[0] - 2, chunk=3), sp, buffers=2) as st:
         X, V = st.generate()
         st.run2(X, V, np.zeros_like(X), np.zeros_like(V), 3)
+        st.run_blocked(X, V, np.zeros_like(X), np.zeros_like(V), 7, 5)
 print("sanitize case ok")

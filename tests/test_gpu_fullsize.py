@@ -23,8 +23,10 @@ def _need_gpu():
 def _samples(n, rng, count):
     out = [(1, 1, 1), (n[0] - 2, n[1] - 2, n[2] - 2), (n[0] // 2, 1, n[2] - 2), (1, n[1] // 2, n[2] // 2),
            (n[0] // 2, n[1] // 2, 31), (n[0] // 2, 15, 32), (65, 16, 33), (64, 17, 96),
-           # K1_TB2 tile / segment borders (owned tiles 30 x 22 from k, j = 0; segments of 64 planes from i = 1)
-           (65, 22, 30), (64, 21, 29), (129, 44, 60), (n[0] - 2, n[1] - 2, 30)]
+           # K1_TB2 tile / segment borders (owned tiles 30 x 22 from k = 1, j = 0; at 512^3 five segments of
+           # 102 planes from i = 1, at 1024^3 seven of 146)
+           (65, 22, 30), (64, 21, 29), (129, 44, 60), (n[0] - 2, n[1] - 2, 30), (102, 23, 31), (103, 22, 1),
+           (104, 66, 61), (147, 88, 91), (148, 43, 90)]
     while len(out) < count:
         out.append(tuple(int(rng.integers(1, n[d] - 1)) for d in range(3)))
     return out
@@ -80,6 +82,16 @@ def test_512cube_march_kernel_sampled_nodes_bitwise():
 def test_1024cube_sampled_nodes_bitwise():
     """configs[4] grid (77 GB on one GPU): 1024^3, 10 steps, 8 nodes."""
     _check_nodes((1024, 1024, 1024), 10, 8)
+
+
+def test_1024cube_eight_positions_configs4_layout_sampled_nodes_bitwise():
+    """configs[4]'s layout on one GPU: 1024^3 spread over devices(0..7) (eight
+    chunks of 128 planes and one of 126, K1 AUTO = K1_TB2 with the deep-halo
+    exchange between positions), 5 steps (two two-step launches and one single
+    step); nodes on both sides of chunk boundaries."""
+    edge = [(128, 500, 3), (129, 1, 1022), (130, 700, 700), (256, 31, 30), (257, 1022, 1022), (897, 511, 512),
+            (896, 2, 64), (1022, 640, 333)]
+    _check_nodes((1024, 1024, 1024), 5, 6, devices=tuple(range(8)), extra=edge)
 
 
 def test_512cube_rest_lattice_fixed_point_and_zero_centre():

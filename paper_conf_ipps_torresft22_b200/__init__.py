@@ -12,7 +12,7 @@ from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
 from .spread import Chunk, Spread
 
 __all__ = ["Spread", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats", "combine_stats", "SpreadError",
-           "K1_AUTO", "K1_DIRECT", "K1_MARCH", "version"]
+           "K1_AUTO", "K1_DIRECT", "K1_MARCH", "K1_MARCH2", "K1_TB2", "version"]
 
 
 def version() -> str:

@@ -260,5 +260,31 @@ def stencil3(a: np.ndarray) -> np.ndarray:
     return b
 
 
+def reduce_exact(a, start: int, length: int, op: str = "sum", scale_exp: int = 60):
+    """The reduction clause's result by definition (DESIGN.md S15 generalised;
+    PAPER.md:330, 773): "sum" -> (value, S) with S = sum over i in
+    [start, start+length) of round_half_even(a[i] * 2^scale_exp), computed with
+    Python integers and Fractions (exact), value = S * 2^-scale_exp rounded once;
+    "min" / "max" -> (element, None) in the IEEE total order of non-NaN values
+    (-0 < +0), NaN if any element is NaN; empty: 0 / +inf / -inf."""
+    import math
+    from fractions import Fraction
+
+    xs = [float(v) for v in a[start:start + length]]
+    if op == "sum":
+        S = 0
+        for x in xs:
+            if not math.isfinite(x) or abs(Fraction(x) * Fraction(2) ** scale_exp) >= 2 ** 94:
+                raise ValueError("outside the exact domain")
+            S += round(Fraction(x) * Fraction(2) ** scale_exp)  # Python rounds half to even
+        return float(Fraction(S) / Fraction(2) ** scale_exp), S
+    if any(math.isnan(x) for x in xs):
+        return math.nan, None
+    if not xs:
+        return (math.inf if op == "min" else -math.inf), None
+    key = lambda x: (x, math.copysign(1.0, x))  # noqa: E731  -0 before +0
+    return (min(xs, key=key) if op == "min" else max(xs, key=key)), None
+
+
 def lib_path() -> str:
     return os.path.join(os.path.dirname(os.path.abspath(__file__)), "liboracle.so")

@@ -59,6 +59,17 @@ class somier_stats_t(ctypes.Structure):
     ]
 
 
+class spread_reduce_result(ctypes.Structure):
+    _fields_ = [
+        ("value", ctypes.c_double),
+        ("sum_lo", ctypes.c_uint64),
+        ("sum_hi", ctypes.c_int64),
+        ("count", ctypes.c_int64),
+    ]
+
+
+REDUCE_SUM, REDUCE_MIN, REDUCE_MAX = 0, 1, 2
+
 _lib = None
 
 # (name, restype, argtypes): every symbol include/*.h declares.
@@ -83,6 +94,8 @@ SIGNATURES = [
     ("spread_chunk_of", ctypes.c_int, [_VP, ctypes.c_int64, _I64P]),
     ("spread_map_extent", ctypes.c_int, [_VP, ctypes.c_int64, spread_map, ctypes.c_int64, _I64P, _I64P]),
     ("spread_stencil3", ctypes.c_int, [_VP, _DP, _DP, ctypes.c_int64]),
+    ("spread_reduce", ctypes.c_int, [_VP, _DP, ctypes.c_int64, ctypes.c_int, ctypes.c_int,
+                                     ctypes.POINTER(spread_reduce_result)]),
     ("spread_last_error", ctypes.c_char_p, []),
     ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),

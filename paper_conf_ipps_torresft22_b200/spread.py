@@ -119,6 +119,22 @@ class Spread:
                 "spread_stencil3")
         return B
 
+    def reduce(self, A, op: str = "sum", scale_exp: int = 60):
+        """`map(to: A[start:size]) reduction(op: r)` over the spread's range, each
+        chunk reduced on its device (spread_reduce). op "sum": the exact
+        fixed-point sum S of round_half_even(A[i] * 2^scale_exp) (returned as
+        the int S and value = S * 2^-scale_exp); "min" / "max": the extreme
+        element (-0 < +0, NaN if any). Returns (value, S or None, count)."""
+        import numpy as np
+
+        A = np.ascontiguousarray(A, dtype=np.float64)
+        code = {"sum": N.REDUCE_SUM, "min": N.REDUCE_MIN, "max": N.REDUCE_MAX}[op]
+        r = N.spread_reduce_result()
+        N.check(N.lib().spread_reduce(self._h, A.ctypes.data_as(ctypes.POINTER(ctypes.c_double)), A.size, code,
+                                      int(scale_exp), ctypes.byref(r)), "spread_reduce")
+        S = (r.sum_hi << 64) + r.sum_lo if op == "sum" else None
+        return r.value, S, r.count
+
     def map_extent(self, c: int, array_len: int, lo_halo: int = 0, hi_halo: int = 0, map_type: int = N.MAP_TO):
         """Section [first, first+len) of A[omp_spread_start-lo : omp_spread_size+lo+hi]."""
         first, ln = ctypes.c_int64(), ctypes.c_int64()

@@ -440,3 +440,32 @@ def test_stencil3_brute_force():
     for i in range(1, 13):
         assert b[i] == a[i - 1] + a[i] + a[i + 1]
     assert b[0] == 0 and b[13] == 0
+
+
+# ---- reduce_exact: the reduction clause's definition (S15 generalised)
+def test_reduce_exact_pins():
+    """Pins of oracle.reduce_exact against things that fix it independently:
+    math.fsum on dyadic data the quantisation leaves exact, hand-computed
+    half-even ties, numpy min/max, IEEE signed-zero order, and the C oracle's
+    own "centers" sums of a Somier state."""
+    import math
+
+    rng = np.random.default_rng(4)
+    a = rng.integers(-2 ** 40, 2 ** 40, 1000) * 2.0 ** -30  # 30 fractional bits: exact at scale 30
+    v, S = O.reduce_exact(a, 0, 1000, "sum", 30)
+    assert v == math.fsum(a) and S == sum(int(x * 2 ** 30) for x in a)
+    assert O.reduce_exact([0.5, 1.5, 2.5, -0.5, -1.5], 0, 5, "sum", 0) == (0.0 + 2 + 2 - 0 - 2, 2)
+    assert O.reduce_exact([0.5, 1.5, 2.5, -0.5, -1.5], 1, 3, "sum", 0)[1] == 2 + 2 - 0
+    b = rng.standard_normal(333)
+    assert O.reduce_exact(b, 0, 333, "min")[0] == b.min() and O.reduce_exact(b, 0, 333, "max")[0] == b.max()
+    assert math.copysign(1, O.reduce_exact([0.0, -0.0, 0.0], 0, 3, "min")[0]) == -1
+    assert math.copysign(1, O.reduce_exact([-0.0, 0.0, -0.0], 0, 3, "max")[0]) == 1
+    assert math.isnan(O.reduce_exact([1.0, math.nan], 0, 2, "max")[0])
+    assert O.reduce_exact([], 0, 0, "min")[0] == math.inf
+    with pytest.raises(ValueError):
+        O.reduce_exact([2.0 ** 34], 0, 1, "sum", 60)
+    # the Somier centre sums of the C oracle are this reduction of the positions at scale 60
+    p = O.Params(n=(7, 6, 9), seed=3)
+    s, st = O.run(O.init(p), 2)
+    for c in range(3):
+        assert O.reduce_exact(s.X[c].ravel(), 0, s.X[c].size, "sum", 60)[1] == st.sums[c]

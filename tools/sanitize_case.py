@@ -40,4 +40,8 @@ for kern in (P.K1_TB2,):
         X, V = st.generate()
         st.run2(X, V, np.zeros_like(X), np.zeros_like(V), 3)
         st.run_blocked(X, V, np.zeros_like(X), np.zeros_like(V), 7, 5)
+# the reduction clause over a multi-chunk spread
+a = np.linspace(-3.0, 5.0, 1001)
+for op in ("sum", "min", "max"):
+    P.Spread([0], 1, 999, chunk=37).reduce(a, op, 40)
 print("sanitize case ok")

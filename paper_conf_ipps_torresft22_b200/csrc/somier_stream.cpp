@@ -440,6 +440,9 @@ spread_status ensure_deep(somier_stream_t h, int64_t planes) {
             for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
                 if (!*pe) S_TRY(h, cudaEventCreateWithFlags(pe, cudaEventDisableTiming));
         }
+        // cudaMemset runs on the legacy stream, which the handle's non-blocking
+        // streams do not wait for: finish the zeroing before any copy lands
+        S_TRY(h, cudaDeviceSynchronize());
     }
     return SPREAD_OK;
 }
@@ -713,6 +716,13 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
             st = paper::encode_slab_tmap(&sl.tmap_vt, g, sl.vt_in, h->max_chunk + 2, paper::kTB2VBoxK, paper::kTB2VBoxJ);
             if (st != SPREAD_OK) return fail(st);
         }
+    }
+    // the slots' cudaMemset ran on the legacy stream: finish it before the
+    // non-blocking streams touch the slots
+    for (auto& d : h->devs) {
+        if (d.chunks.empty()) continue;
+        if ((e = cudaSetDevice(d.device)) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess)
+            return fail(sfail(h, e, "cudaDeviceSynchronize"));
     }
     h->ev.resize((size_t)s->nchunks);
     for (int64_t c = 0; c < s->nchunks; c++) {

@@ -273,3 +273,23 @@ def test_stream_run_blocked_matches_run_at_size_and_traffic():
     assert np.array_equal(X, X2) and np.array_equal(V, V2)  # 2 trips: back in the first buffers
     assert (t8["h2d_bytes"] + t8["d2h_bytes"]) / 8 < 0.5 * (t2["h2d_bytes"] + t2["d2h_bytes"]) / 2
     assert t2["d2h_bytes"] == r2["d2h_bytes"]
+
+
+def test_stream_fresh_slots_are_zeroed_before_first_copy():
+    """Regression: the slots' zeroing (cudaMemset, legacy stream) must finish
+    before the handle's non-blocking streams copy the first chunk in -- else it
+    could wipe the first planes of a chunk mapped right after creation (a wide
+    cross-section makes the memset long enough to lose that race)."""
+    n = (24, 512, 512)
+    sp = P.SomierParams(n=n, seed=8)
+    want = None
+    for rep in range(3):
+        for spt, buffers in ((2, 1), (4, 1), (2, 3)):
+            with P.SomierStream(P.Spread([0], 1, n[0] - 2, chunk=22 if rep else 8), sp, buffers=buffers) as s:
+                X, V = s.generate()
+                XN, VN = np.zeros_like(X), np.zeros_like(V)
+                st = s.run_blocked(X, V, XN, VN, 4, spt)[-1]
+                fX, fV = (X, V) if (-(-4 // spt)) % 2 == 0 else (XN, VN)
+            key = (st.sums, st.vmax2_bits, fX[:, :6].tobytes(), fV[:, :6].tobytes())
+            want = want or key
+            assert key == want

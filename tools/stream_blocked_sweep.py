@@ -6,7 +6,7 @@ place) or somier_stream_run_blocked (s >= 2) and timed by wall clock (every
 copy, kernel and the per-trip stats read-back inside). Prints one JSON line
 per configuration.
 
-  python tools/stream_blocked_sweep.py n nsteps chunk:s [chunk:s ...]
+  python tools/stream_blocked_sweep.py n nsteps chunk:s[:buffers] [...]   (buffers default 3)
 """
 import json
 import os
@@ -20,7 +20,7 @@ import paper_conf_ipps_torresft22_b200 as P  # noqa: E402
 
 n = int(sys.argv[1])
 nsteps = int(sys.argv[2])
-cfgs = [tuple(int(v) for v in c.split(":")) for c in sys.argv[3:]]
+cfgs = [tuple(int(v) for v in (c + ":3").split(":")[:3]) for c in sys.argv[3:]]
 need = 12 * n ** 3 * 8
 with open("/proc/meminfo") as f:
     avail = next(int(line.split()[1]) * 1024 for line in f if line.startswith("MemAvailable:"))
@@ -35,8 +35,8 @@ pin_s = time.perf_counter() - t0
 ptr = [g.data_ptr() for g in grids]
 X, V, XN, VN = ptr[0:3], ptr[3:6], ptr[6:9], ptr[9:12]
 ref = None
-for chunk, s in cfgs:
-    st = P.SomierStream(P.Spread([0], 1, n - 2, chunk=chunk), params, buffers=3)
+for chunk, s, buffers in cfgs:
+    st = P.SomierStream(P.Spread([0], 1, n - 2, chunk=chunk), params, buffers=buffers)
     st.generate_ptrs(X + V)
     t0 = time.perf_counter()
     if s == 1:
@@ -51,7 +51,7 @@ for chunk, s in cfgs:
     st.close()
     key = (stats.sums, stats.vmax2_bits)
     ref = ref or key
-    print(json.dumps({"n": n, "nsteps": nsteps, "chunk": chunk, "steps_per_trip": s, "wall_s": wall,
+    print(json.dumps({"n": n, "nsteps": nsteps, "chunk": chunk, "steps_per_trip": s, "buffers": buffers, "wall_s": wall,
                       "node_updates_per_s": (n - 2) ** 3 * nsteps / wall,
                       "host_bytes_per_node_update": per_step / (n - 2) ** 3,
                       "pcie_gbs": per_step * nsteps / wall / 1e9, "pin_s": pin_s,

@@ -22,7 +22,7 @@
 
 namespace paper {
 
-constexpr int kMaxNodesPerThread = 128;
+constexpr int kMaxNodesPerThread = 128;  // STATS_FP64_ACC variant only
 constexpr double kRoundC = 6755399441055744.0;  // 1.5 * 2^52
 
 #ifndef STATS_FP64_ACC
@@ -34,8 +34,11 @@ constexpr double kRoundC = 6755399441055744.0;  // 1.5 * 2^52
 //   ld = fma(r, 2^32, C)                   = C + l, l = round_half_even(r 2^32)
 // C + m with |m| < 2^51 lies in [2^52, 2^53), where one unit of the mantissa
 // is 1, so bits(C + m) = bits(C) + m: sum h = sum bits(hd) - n bits(C) and
-// sum l = sum bits(ld) - n bits(C), computed modulo 2^64 (the true sums are
-// below 2^53 in magnitude). q(x) = h 2^32 + l as in the fp64 form below.
+// sum l = sum bits(ld) - n bits(C), computed modulo 2^64, which is exact while
+// the true sums stay below 2^63 in magnitude: |h| < 2^46 for |x| < 2^18, so up
+// to 2^17 nodes per thread (K1_TB2: at most 2 rows x 256 planes = 512).
+// q(x) = h 2^32 + l as in the fp64 form below. Adding x = 0 adds exactly
+// bits(C) to both words and 1 to n: a neutral element.
 struct NodeStats {
     unsigned long long hb[3], lb[3];
     unsigned int n;  // nodes added (positions)

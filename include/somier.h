@@ -302,6 +302,8 @@ spread_status somier_stream_run(somier_stream_t h, double* x, double* y, double*
  *   step of a two-step launch has no statistics, as on a K1_TB2 handle).
  * Chunk-level dependencies as in somier_stream_run, over the chunks within
  * two planes. Results are bit-identical to somier_stream_run / the oracle.
+ * Same as somier_stream_run_blocked with steps_per_trip = 2 (its device
+ * buffers are allocated on first use).
  * Errors: EINVAL (NULL, nsteps < 0, aliasing buffers), ENOMEM, ECUDA.
  */
 spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
@@ -310,9 +312,9 @@ spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double
 
 /*
  * somier_stream_run_blocked -- as somier_stream_run2 with `steps_per_trip` = s
- * steps per host round trip (1 <= s <= 256; s = 2 moves the same bytes as
- * somier_stream_run2): per chunk map(to: X[start-s : size+2s],
- * V[start-s : size+2s]) (clipped to the grid), ceil(s/2) K1_TB2 launches over
+ * steps per host round trip (1 <= s <= 256; s = 2 is somier_stream_run2): per
+ * chunk map(to: X[start-s : size+2s], V[start-v : size+2v]) with v =
+ * max(1, s-1) (clipped to the grid), ceil(s/2) K1_TB2 launches over
  * regions that shrink by two planes per side per launch down to the chunk
  * itself (an odd s ends with a one-step launch), map(from: X[start : size],
  * V[start : size]). Host<->device bytes per node-update fall as ~1/s while

@@ -28,14 +28,6 @@ namespace {
 
 struct Slot {
     void* base = nullptr;
-    // deep slabs (two-step mode, K1_TB2 layout): X planes [start-2, start+size+2),
-    // V planes [start-1, start+size+1); V_{t+2} in its own buffer (neighbour
-    // chunks read V_t halo planes from the host copy)
-    double* xt_in = nullptr;
-    double* xt_out = nullptr;
-    double* vt_in = nullptr;
-    double* vt_out = nullptr;
-    // one-step views into them (one plane in): X planes [start-1, start+size+1), V [start, start+size)
     double* x_in = nullptr;   // X_t of the chunk, size+2 planes (halo planes included)
     double* x_out = nullptr;  // X_{t+1}, planes 1..size written by K1
     double* v = nullptr;      // V of the chunk, size planes
@@ -43,8 +35,6 @@ struct Slot {
     alignas(64) CUtensorMap tmap_v;
     alignas(64) CUtensorMap tmap_x2;
     alignas(64) CUtensorMap tmap_v2;
-    alignas(64) CUtensorMap tmap_xt;  // K1_TB2 boxes over the deep slabs
-    alignas(64) CUtensorMap tmap_vt;
     cudaEvent_t comp_done = nullptr, d2h_done = nullptr;
     bool used = false;
 };
@@ -260,108 +250,6 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
     return SPREAD_OK;
 }
 
-// Chunks whose deep-halo extent [start-2, start+size+2) meets chunk c's planes
-// (and vice versa): the chunks c's two-step H2D reads from, and whose H2D of
-// the previous launch read the planes c's D2H overwrites.
-void halo_range(const somier_stream_s* h, const paper::ChunkInfo& ci, int64_t* c_lo, int64_t* c_hi) {
-    const int64_t n0 = h->p.n[0];
-    *c_lo = h->spread.chunk_of(std::max<int64_t>(1, ci.start - 2));
-    *c_hi = h->spread.chunk_of(std::min<int64_t>(n0 - 2, ci.start + ci.size + 1));
-}
-
-// Enqueue launch k of a two-step run (0-based within the run): every chunk,
-// in chunk order, maps in X_t planes [start-2, start+size+2) and V_t planes
-// [start-1, start+size+1) (clipped to the grid), runs K1_TB2 (two steps, or
-// one if !two) and maps out X_{t+2}, V_{t+2} of its planes into (XN, VN).
-spread_status enqueue_stream_tb2(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
-                                 double* const VN[3], int64_t k, bool two, bool chained) {
-    const int64_t n0 = h->p.n[0];
-    const int64_t nch = h->spread.nchunks;
-    const int64_t ps = h->geom.plane_stride();
-    const int par = (int)(k & 1), prev = par ^ 1;
-    for (int64_t c = 0; c < nch; c++) {
-        const paper::ChunkInfo ci = h->spread.chunk_info(c);
-        Dev& d = h->devs[ci.pos];
-        const size_t m = (size_t)(c / (int64_t)h->devs.size());
-        Slot& sl = d.slots[m % d.slots.size()];
-        const paper::SlabGeom g = geom_of(h, ci);
-        const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
-        ChunkEvents& ev = h->ev[(size_t)c];
-        int64_t c_lo, c_hi;
-        halo_range(h, ci, &c_lo, &c_hi);
-        S_TRY(h, cudaSetDevice(d.device));
-        // map(to: X[start-2 : size+4], V[start-1 : size+2])
-        if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
-        if (chained)
-            for (int64_t nb = c_lo; nb <= c_hi; nb++)
-                S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
-        const int64_t xlo = std::max<int64_t>(0, ci.start - 2), xhi = std::min<int64_t>(n0, ci.start + ci.size + 2);
-        const int64_t vlo = std::max<int64_t>(0, ci.start - 1), vhi = std::min<int64_t>(n0, ci.start + ci.size + 1);
-        for (int q = 0; q < 3; q++) {
-            S_TRY(h, paper::copy_slab_planes(g, sl.xt_in, q, xlo - (ci.start - 2), X[q], xlo, xhi - xlo,
-                                             cudaMemcpyHostToDevice, d.s_h2d));
-            S_TRY(h, paper::copy_slab_planes(g, sl.vt_in, q, vlo - (ci.start - 1), V[q], vlo, vhi - vlo,
-                                             cudaMemcpyHostToDevice, d.s_h2d));
-        }
-        S_TRY(h, cudaEventRecord(ev.h2d[par], d.s_h2d));
-        S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
-        // the fixed face nodes of the output planes (K1_TB2 writes the moving nodes only)
-        S_TRY(h, cudaMemcpyAsync(sl.xt_out + 2 * ps, sl.xt_in + 2 * ps, (size_t)(ci.size * ps) * sizeof(double),
-                                 cudaMemcpyDeviceToDevice, d.s_comp));
-        paper::StatsAccum* acc = d.acc(k);
-        if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, acc + 1, d.s_comp));
-        if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, ci.size + 1, 1, acc + 1, d.s_comp));
-        S_TRY(h, paper::launch_kface_stats(sl.x_in, g, 1, ci.size, acc + 1, d.s_comp));
-        paper::StepArgs a;
-        std::memset(&a, 0, sizeof a);
-        a.x_cur = sl.xt_in;
-        a.v = sl.vt_in;
-        a.g = g;
-        a.K = h->p.k_spring;
-        a.L = h->p.rest_len;
-        a.M = h->p.mass;
-        a.dt = h->p.dt;
-        a.acc = acc;
-        a.tmap_x_cur = &sl.tmap_xt;
-        a.tmap_v = &sl.tmap_vt;
-        paper::Tb2Out o;
-        std::memset(&o, 0, sizeof o);
-        o.x_out = sl.xt_out;
-        o.v_out = sl.vt_out;
-        o.two = two;
-        S_TRY(h, paper::launch_k1_tb2(a, o, h->p.mass == 1.0, d.s_comp));
-        h->launches++;
-        S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
-        // map(from: X[start : size], V[start : size]) into the other buffers (+ the
-        // fixed end planes); waits for the H2D of the previous launch that read
-        // these planes of (XN, VN) as halos
-        S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
-        if (chained)
-            for (int64_t nb = c_lo; nb <= c_hi; nb++)
-                if (nb != c) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)nb].h2d[prev], 0));
-        for (int q = 0; q < 3; q++) {
-            S_TRY(h, paper::copy_slab_planes(g, sl.xt_out, q, 2, XN[q], ci.start, ci.size, cudaMemcpyDeviceToHost,
-                                             d.s_d2h));
-            S_TRY(h, paper::copy_slab_planes(g, sl.vt_out, q, 1, VN[q], ci.start, ci.size, cudaMemcpyDeviceToHost,
-                                             d.s_d2h));
-            if (first) {
-                S_TRY(h, paper::copy_slab_planes(g, sl.xt_in, q, 1, XN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
-                S_TRY(h, paper::copy_slab_planes(g, sl.vt_in, q, 0, VN[q], 0, 1, cudaMemcpyDeviceToHost, d.s_d2h));
-            }
-            if (last) {
-                S_TRY(h, paper::copy_slab_planes(g, sl.xt_in, q, ci.size + 2, XN[q], n0 - 1, 1,
-                                                 cudaMemcpyDeviceToHost, d.s_d2h));
-                S_TRY(h, paper::copy_slab_planes(g, sl.vt_in, q, ci.size + 1, VN[q], n0 - 1, 1,
-                                                 cudaMemcpyDeviceToHost, d.s_d2h));
-            }
-        }
-        S_TRY(h, cudaEventRecord(ev.d2h[par], d.s_d2h));
-        S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
-        sl.used = true;
-    }
-    return SPREAD_OK;
-}
-
 // Combine the per-launch stats slots of every device into stats[0 .. n).
 spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, somier_stats_t* stats) {
     std::vector<__int128> sums((size_t)n * 3, 0);
@@ -383,34 +271,6 @@ spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, s
         paper::finish_somier_stats(&h->p, &sums[(size_t)(3 * t)], vmax2[(size_t)t],
                                    h->p.n[0] * h->p.n[1] * h->p.n[2], steps[t], &stats[t]);
     return SPREAD_OK;
-}
-
-// Two-step run: nsteps / 2 two-step launches (+ one one-step launch if nsteps
-// is odd), alternating (X, V) -> (XN, VN) -> (X, V) ...; stats[k] (if non-NULL)
-// receives the statistics after launch k. One host barrier at the end.
-spread_status stream_run_tb2(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
-                             double* const VN[3], int64_t nsteps, somier_stats_t* stats) {
-    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
-    const int64_t nl = nsteps / 2 + (nsteps & 1);
-    spread_status st = ensure_acc(h, nl);
-    if (st != SPREAD_OK) return st;
-    for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
-        S_TRY(h, cudaSetDevice(d.device));
-        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * (size_t)nl * sizeof(paper::StatsAccum), d.s_comp));
-    }
-    std::vector<int64_t> steps((size_t)nl);
-    for (int64_t k = 0; k < nl; k++) {
-        const bool two = k < nsteps / 2;
-        steps[(size_t)k] = h->step + std::min<int64_t>(nsteps, 2 * (k + 1));
-        st = (k & 1) ? enqueue_stream_tb2(h, XN, VN, X, V, k, two, k > 0)
-                     : enqueue_stream_tb2(h, X, V, XN, VN, k, two, k > 0);
-        if (st != SPREAD_OK) return st;
-    }
-    st = sync_devs(h);
-    if (st != SPREAD_OK) return st;
-    h->step += nsteps;
-    return stats ? gather_stats(h, nl, steps.data(), stats) : SPREAD_OK;
 }
 
 // (Re)allocate every device's deep slots for `planes` X planes per buffer.
@@ -454,8 +314,9 @@ void reach_range(const somier_stream_s* h, const paper::ChunkInfo& ci, int64_t d
     *c_hi = h->spread.chunk_of(std::min<int64_t>(n0 - 2, ci.start + ci.size + depth - 1));
 }
 
-// Trip k of a blocked run: every chunk maps in X_t and V_t planes
-// [start-s, start+size+s) (clipped to the grid), advances s
+// Trip k of a blocked run: every chunk maps in X_t planes [start-s, start+size+s)
+// and V_t planes [start-s+1, start+size+s-1) (at least one halo plane; clipped
+// to the grid), advances s
 // steps with ceil(s/2) K1_TB2 launches over regions that shrink by two planes
 // per side per launch (the last one is the chunk itself; an odd s ends with a
 // one-step launch), and maps X_{t+s}, V_{t+s} of its planes out into (XN, VN).
@@ -485,7 +346,10 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             for (int64_t nb = c_lo; nb <= c_hi; nb++)
                 S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
         const int64_t xlo = std::max<int64_t>(0, ci.start - s), xhi = std::min<int64_t>(n0, ci.start + ci.size + s);
-        const int64_t vlo = std::max<int64_t>(0, ci.start - s), vhi = std::min<int64_t>(n0, ci.start + ci.size + s);
+        // V_t is needed one plane less deep than X_t, but at least one plane
+        // (a one-step launch reads the ring plane; the first chunk maps the face plane)
+        const int64_t vd = std::max<int64_t>(1, s - 1);
+        const int64_t vlo = std::max<int64_t>(0, ci.start - vd), vhi = std::min<int64_t>(n0, ci.start + ci.size + vd);
         paper::SlabGeom g = geom_of(h, ci);
         for (int q = 0; q < 3; q++) {
             S_TRY(h, paper::copy_slab_planes(g, sl.xa, q, xlo - x0, X[q], xlo, xhi - xlo, cudaMemcpyHostToDevice,
@@ -674,9 +538,8 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         return code;
     };
     const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
-    const size_t xb = round_up(plane * (size_t)(h->max_chunk + 4), 4096);
-    const size_t vb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
-    const int64_t ps = h->geom.plane_stride();
+    const size_t xb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
+    const size_t vb = round_up(plane * (size_t)h->max_chunk, 4096);
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         if ((e = cudaSetDevice(d.device)) != cudaSuccess) return fail(sfail(h, e, "cudaSetDevice"));
@@ -688,17 +551,10 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         d.acc_steps = kAccSteps;
         d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
         for (auto& sl : d.slots) {
-            if ((e = cudaMalloc(&sl.base, 2 * xb + 2 * vb)) != cudaSuccess)
-                return fail(sfail(h, e, "cudaMalloc(slot)"));
-            // zeroed once: the fixed face nodes of V_{t+2} are never written by K1_TB2
-            if ((e = cudaMemset(sl.base, 0, 2 * xb + 2 * vb)) != cudaSuccess) return fail(sfail(h, e, "cudaMemset(slot)"));
-            sl.xt_in = (double*)sl.base;
-            sl.xt_out = (double*)((char*)sl.base + xb);
-            sl.vt_in = (double*)((char*)sl.base + 2 * xb);
-            sl.vt_out = (double*)((char*)sl.base + 2 * xb + vb);
-            sl.x_in = sl.xt_in + ps;
-            sl.x_out = sl.xt_out + ps;
-            sl.v = sl.vt_in + ps;
+            if ((e = cudaMalloc(&sl.base, 2 * xb + vb)) != cudaSuccess) return fail(sfail(h, e, "cudaMalloc(slot)"));
+            sl.x_in = (double*)sl.base;
+            sl.x_out = (double*)((char*)sl.base + xb);
+            sl.v = (double*)((char*)sl.base + 2 * xb);
             for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
                 if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
                     return fail(sfail(h, e, "cudaEventCreate"));
@@ -711,18 +567,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
             if (st != SPREAD_OK) return fail(st);
             st = paper::encode_slab_tmap(&sl.tmap_v2, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kV2BoxJ);
             if (st != SPREAD_OK) return fail(st);
-            st = paper::encode_slab_tmap(&sl.tmap_xt, g, sl.xt_in, h->max_chunk + 4, paper::kTB2XBoxK, paper::kTB2XBoxJ);
-            if (st != SPREAD_OK) return fail(st);
-            st = paper::encode_slab_tmap(&sl.tmap_vt, g, sl.vt_in, h->max_chunk + 2, paper::kTB2VBoxK, paper::kTB2VBoxJ);
-            if (st != SPREAD_OK) return fail(st);
         }
-    }
-    // the slots' cudaMemset ran on the legacy stream: finish it before the
-    // non-blocking streams touch the slots
-    for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
-        if ((e = cudaSetDevice(d.device)) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess)
-            return fail(sfail(h, e, "cudaDeviceSynchronize"));
     }
     h->ev.resize((size_t)s->nchunks);
     for (int64_t c = 0; c < s->nchunks; c++) {
@@ -820,7 +665,7 @@ spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double
     double* XN[3] = {xn, yn, zn};
     double* V[3] = {vx, vy, vz};
     double* VN[3] = {vxn, vyn, vzn};
-    return stream_run_tb2(h, X, V, XN, VN, nsteps, stats);
+    return stream_run_blocked(h, X, V, XN, VN, nsteps, 2, stats);  // trips of two steps
 }
 
 spread_status somier_stream_run_blocked(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
@@ -851,7 +696,8 @@ spread_status somier_stream_traffic_blocked(somier_stream_t h, int64_t steps_per
     for (int64_t c = 0; c < h->spread.nchunks; c++) {
         const paper::ChunkInfo ci = h->spread.chunk_info(c);
         const int64_t xp = std::min<int64_t>(n0, ci.start + ci.size + s) - std::max<int64_t>(0, ci.start - s);
-        const int64_t vp = std::min<int64_t>(n0, ci.start + ci.size + s) - std::max<int64_t>(0, ci.start - s);
+        const int64_t vd = std::max<int64_t>(1, s - 1);
+        const int64_t vp = std::min<int64_t>(n0, ci.start + ci.size + vd) - std::max<int64_t>(0, ci.start - vd);
         in += plane * (xp + vp);
         outb += 2 * plane * ci.size;
     }
@@ -863,20 +709,7 @@ spread_status somier_stream_traffic_blocked(somier_stream_t h, int64_t steps_per
 
 spread_status somier_stream_traffic2(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes) {
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_traffic2: NULL handle");
-    const int64_t n0 = h->p.n[0];
-    const int64_t plane = 3 * h->p.n[1] * h->p.n[2] * (int64_t)sizeof(double);
-    int64_t in = 0, outb = 0;
-    for (int64_t c = 0; c < h->spread.nchunks; c++) {
-        const paper::ChunkInfo ci = h->spread.chunk_info(c);
-        const int64_t xp = std::min<int64_t>(n0, ci.start + ci.size + 2) - std::max<int64_t>(0, ci.start - 2);
-        const int64_t vp = std::min<int64_t>(n0, ci.start + ci.size + 1) - std::max<int64_t>(0, ci.start - 1);
-        in += plane * (xp + vp);
-        outb += 2 * plane * ci.size;
-    }
-    outb += 4 * plane;  // fixed end planes of X and V
-    if (h2d_bytes) *h2d_bytes = in;
-    if (d2h_bytes) *d2h_bytes = outb;
-    return SPREAD_OK;
+    return somier_stream_traffic_blocked(h, 2, h2d_bytes, d2h_bytes);
 }
 
 spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes, int64_t* launches) {

@@ -144,6 +144,7 @@ struct somier_s {
     bool pdl = false;
     int graph_pos = -1;
     cudaGraphExec_t graph_exec = nullptr;
+    cudaGraphExec_t tb2_graph[4] = {nullptr, nullptr, nullptr, nullptr};  // by (X buffer parity, step parity)
 
     bool unit_mass() const { return p.mass == 1.0; }
     paper::K1Variant variant() const {
@@ -501,7 +502,7 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
             if (c.pos != pos) one = false;
         }
         const char* ng = std::getenv("SOMIER_NO_GRAPH");
-        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1') && !h->tb2;
+        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1');
         h->graph_pos = pos;
         // PDL between consecutive K1 launches only where nothing else sits
         // between them on the stream (one stream, no flag waits); SOMIER_NO_PDL=1
@@ -743,7 +744,48 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     if (h->tb2) {
         // K1_TB2: pairs of steps; a leftover single step runs the same kernel
-        // in one-step mode (same slab layout and halo protocol)
+        // in one-step mode (same slab layout and halo protocol). On one stream
+        // without flags, two consecutive pairs (four steps) are captured once
+        // per (buffer parity, step parity) -- everything a launch depends on --
+        // and replayed as a CUDA graph; the handle's first pair runs eagerly
+        // (lazy host-side state is set up outside any capture).
+        if (h->graph_ok && nsteps >= 4) {
+            if (h->launches == 0) {
+                spread_status st = enqueue_tb2(h, true);
+                if (st != SPREAD_OK) return st;
+                nsteps -= 2;
+            }
+            DevCtx& d = h->devs[h->graph_pos];
+            int64_t nloc = 0;
+            for (auto& c : h->chunks) nloc += c.local ? 1 : 0;
+            while (nsteps >= 4) {
+                cudaGraphExec_t& ge = h->tb2_graph[(h->xbuf & 1) * 2 + (int)(h->step & 1)];
+                CUDA_TRY(h, cudaSetDevice(d.device));
+                if (!ge) {
+                    const int64_t s0 = h->step, l0 = h->launches;
+                    const int xb0 = h->xbuf, vb0 = h->vbuf;
+                    CUDA_TRY(h, cudaStreamBeginCapture(d.stream, cudaStreamCaptureModeThreadLocal));
+                    spread_status st = enqueue_tb2(h, true);
+                    if (st == SPREAD_OK) st = enqueue_tb2(h, true);
+                    h->step = s0;
+                    h->launches = l0;
+                    h->xbuf = xb0;
+                    h->vbuf = vb0;
+                    cudaGraph_t g = nullptr;
+                    cudaError_t e = cudaStreamEndCapture(d.stream, &g);
+                    if (st != SPREAD_OK) return st;
+                    if (e != cudaSuccess) return cuda_fail(h, e, "somier_step: graph capture");
+                    e = cudaGraphInstantiate(&ge, g, 0);
+                    cudaGraphDestroy(g);
+                    if (e != cudaSuccess) return cuda_fail(h, e, "somier_step: graph instantiate");
+                    CUDA_TRY(h, cudaSetDevice(d.device));
+                }
+                CUDA_TRY(h, cudaGraphLaunch(ge, d.stream));
+                h->step += 4;
+                h->launches += 2 * nloc;
+                nsteps -= 4;
+            }
+        }
         for (; nsteps >= 2; nsteps -= 2) {
             spread_status st = enqueue_tb2(h, true);
             if (st != SPREAD_OK) return st;
@@ -1154,6 +1196,8 @@ spread_status somier_destroy(somier_t h) {
             cudaStreamSynchronize(d.stream);
         }
     if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
+    for (auto& ge : h->tb2_graph)
+        if (ge) cudaGraphExecDestroy(ge);
     free_all(h);
     delete h;
     return SPREAD_OK;

@@ -51,13 +51,16 @@ def _tb2_launches(splits):
     return sum(k // 2 + k % 2 for k in splits)
 
 
-@pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7), (1, 12)])
-def test_tb2_splits_bitwise(splits):
+@pytest.mark.parametrize("chunk", [0, 4])
+@pytest.mark.parametrize("splits", [(13,), (3, 4, 1, 5), (1, 1, 11), (2, 2, 2, 7), (1, 12), (5, 9, 4, 6)])
+def test_tb2_splits_bitwise(splits, chunk):
     """K1_TB2 (two steps per launch, AUTO on large single-chunk grids): any split
     of the step count, on either parity, gives the oracle's bits, stats
-    included."""
+    included -- through the graph replays of two pairs (keyed by buffer and
+    step parity) and the eager pairs / single steps around them; chunk 4: three
+    chunks on one stream (deep-halo stores inside the graph)."""
     sp = P.SomierParams(n=(12, 10, 36), seed=3, kernel=P.K1_TB2)
-    with P.Somier(P.Spread([0], 1, 10), sp) as s:
+    with P.Somier(P.Spread([0], 1, 10, chunk=chunk), sp) as s:
         assert s.kernel_in_use == P.K1_TB2
         for k in splits:
             s.step(k)
@@ -65,8 +68,21 @@ def test_tb2_splits_bitwise(splits):
             ref, rst = O.run(O.init(O.Params(n=sp.n, seed=3)), s.step_count)
             assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits, (splits, k)
         X, V = s.read()
-        assert s.launches == _tb2_launches(splits)
+        assert s.launches == _tb2_launches(splits) * s.local_chunks
     assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+
+
+def test_tb2_eager_and_graph_identical(monkeypatch):
+    sp = P.SomierParams(n=(20, 18, 40), seed=9, kernel=P.K1_TB2)
+    outs = []
+    for env in ("0", "1"):
+        monkeypatch.setenv("SOMIER_NO_GRAPH", env)
+        with P.Somier(P.Spread([0], 1, 18, chunk=6), sp) as s:
+            s.step(3)
+            s.step(22)
+            outs.append(s.read() + (s.stats().sums,))
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    assert outs[0][2] == outs[1][2]
 
 
 def test_auto_kernel_resolution():

@@ -43,7 +43,7 @@ def parse():
     ap.add_argument("--kernel", choices=["auto", "direct", "march", "march2", "tb2"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
     ap.add_argument("--e2e-steps", type=int, default=8)
-    ap.add_argument("--stream-chunk", type=int, default=32, help="planes per chunk in the host-streamed e2e")
+    ap.add_argument("--stream-chunk", type=int, default=64, help="planes per chunk in the host-streamed e2e")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)

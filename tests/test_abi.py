@@ -78,3 +78,22 @@ def test_somier_init_without_gpu_fails_loudly():
     with pytest.raises(P.SpreadError) as e:
         P.Somier(P.Spread([0], 1, 8), P.SomierParams(n=(10, 10, 10)))
     assert e.value.status == N.ENODEV
+
+
+def test_capi_exposes_every_entry_point_under_its_c_name():
+    """The Python binding carries the C names (argument marshalling only)."""
+    from paper_conf_ipps_torresft22_b200 import capi
+
+    for name in _declared():
+        assert callable(getattr(capi, name)), name
+    # host-only calls work without a GPU, through the C names
+    h = ctypes.c_void_p()
+    devs = (ctypes.c_int * 3)(2, 0, 1)
+    capi.spread_create(devs, 3, 1, 14, 0, 4, ctypes.byref(h))
+    n = ctypes.c_int64()
+    capi.spread_num_chunks(h, ctypes.byref(n))
+    assert n.value == 4  # range of 14 iterations in chunks of 4: 4, 4, 4, 2
+    capi.spread_destroy(h)
+    with pytest.raises(P.SpreadError):
+        capi.spread_create(devs, 0, 1, 14, 0, 4, ctypes.byref(h))  # no devices
+    assert capi.somier_version()

@@ -273,6 +273,49 @@ spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, s
     return SPREAD_OK;
 }
 
+// The one-step slots and the deep slots of blocked trips never coexist: the
+// mode in use holds the device memory (a switch synchronises and reallocates),
+// so a blocked run can use the memory the one-step slots would pin.
+void release_deep(Dev& d) {
+    for (auto& sl : d.deep) {
+        if (sl.base) cudaFree(sl.base);
+        sl.base = nullptr;
+        sl.planes = 0;
+        sl.used = false;
+    }
+}
+
+spread_status ensure_flat(somier_stream_t h) {
+    const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
+    const size_t xb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
+    const size_t vb = round_up(plane * (size_t)h->max_chunk, 4096);
+    for (auto& d : h->devs) {
+        if (d.chunks.empty() || d.slots.empty() || d.slots[0].base) continue;
+        S_TRY(h, cudaSetDevice(d.device));
+        S_TRY(h, cudaDeviceSynchronize());
+        release_deep(d);
+        for (auto& sl : d.slots) {
+            S_TRY(h, cudaMalloc(&sl.base, 2 * xb + vb));
+            sl.x_in = (double*)sl.base;
+            sl.x_out = (double*)((char*)sl.base + xb);
+            sl.v = (double*)((char*)sl.base + 2 * xb);
+            sl.used = false;
+            const paper::SlabGeom g = h->geom;
+            spread_status st = paper::encode_slab_tmap(&sl.tmap_x, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK,
+                                                       paper::kXBoxJ);
+            if (st == SPREAD_OK)
+                st = paper::encode_slab_tmap(&sl.tmap_v, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kVBoxJ);
+            if (st == SPREAD_OK)
+                st = paper::encode_slab_tmap(&sl.tmap_x2, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK,
+                                             paper::kX2BoxJ);
+            if (st == SPREAD_OK)
+                st = paper::encode_slab_tmap(&sl.tmap_v2, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kV2BoxJ);
+            if (st != SPREAD_OK) return st;
+        }
+    }
+    return SPREAD_OK;
+}
+
 // (Re)allocate every device's deep slots for `planes` X planes per buffer.
 spread_status ensure_deep(somier_stream_t h, int64_t planes) {
     const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
@@ -280,8 +323,12 @@ spread_status ensure_deep(somier_stream_t h, int64_t planes) {
         if (d.chunks.empty()) continue;
         S_TRY(h, cudaSetDevice(d.device));
         if (!d.scratch_acc) S_TRY(h, cudaMalloc(&d.scratch_acc, sizeof(paper::StatsAccum)));
-        if (!d.deep.empty() && d.deep[0].planes >= planes) continue;
+        if (!d.deep.empty() && d.deep[0].base && d.deep[0].planes >= planes) continue;
         S_TRY(h, cudaDeviceSynchronize());
+        for (auto& sl : d.slots) {  // the one-step slots give their memory up (ensure_flat restores them)
+            if (sl.base) cudaFree(sl.base);
+            sl.base = nullptr;
+        }
         for (auto& sl : d.deep)
             if (sl.base) S_TRY(h, cudaFree(sl.base));
         d.deep.resize(d.slots.size());
@@ -470,7 +517,9 @@ spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* 
 spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
                          int64_t nsteps, somier_stats_t* stats) {
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
-    spread_status st = ensure_acc(h, nsteps);
+    spread_status st = ensure_flat(h);
+    if (st != SPREAD_OK) return st;
+    st = ensure_acc(h, nsteps);
     if (st != SPREAD_OK) return st;
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
@@ -537,9 +586,6 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         set_last_error("%s", msg.c_str());
         return code;
     };
-    const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
-    const size_t xb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
-    const size_t vb = round_up(plane * (size_t)h->max_chunk, 4096);
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         if ((e = cudaSetDevice(d.device)) != cudaSuccess) return fail(sfail(h, e, "cudaSetDevice"));
@@ -550,25 +596,13 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
             return fail(sfail(h, e, "cudaMalloc(stats)"));
         d.acc_steps = kAccSteps;
         d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
-        for (auto& sl : d.slots) {
-            if ((e = cudaMalloc(&sl.base, 2 * xb + vb)) != cudaSuccess) return fail(sfail(h, e, "cudaMalloc(slot)"));
-            sl.x_in = (double*)sl.base;
-            sl.x_out = (double*)((char*)sl.base + xb);
-            sl.v = (double*)((char*)sl.base + 2 * xb);
+        for (auto& sl : d.slots)
             for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
                 if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
                     return fail(sfail(h, e, "cudaEventCreate"));
-            paper::SlabGeom g = h->geom;
-            st = paper::encode_slab_tmap(&sl.tmap_x, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK, paper::kXBoxJ);
-            if (st != SPREAD_OK) return fail(st);
-            st = paper::encode_slab_tmap(&sl.tmap_v, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kVBoxJ);
-            if (st != SPREAD_OK) return fail(st);
-            st = paper::encode_slab_tmap(&sl.tmap_x2, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK, paper::kX2BoxJ);
-            if (st != SPREAD_OK) return fail(st);
-            st = paper::encode_slab_tmap(&sl.tmap_v2, g, sl.v, h->max_chunk, paper::kVBoxK, paper::kV2BoxJ);
-            if (st != SPREAD_OK) return fail(st);
-        }
     }
+    st = ensure_flat(h);
+    if (st != SPREAD_OK) return fail(st);
     h->ev.resize((size_t)s->nchunks);
     for (int64_t c = 0; c < s->nchunks; c++) {
         if ((e = cudaSetDevice(h->devs[s->chunk_info(c).pos].device)) != cudaSuccess)
@@ -585,6 +619,10 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
 spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
                                      double* vz) {
     if (!h || !x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_generate: NULL argument");
+    {
+        const spread_status st = ensure_flat(h);
+        if (st != SPREAD_OK) return st;
+    }
     double* X[3] = {x, y, z};
     const int64_t n0 = h->p.n[0];
     const size_t grid = (size_t)(h->p.n[0] * h->p.n[1] * h->p.n[2]);

@@ -293,3 +293,22 @@ def test_stream_fresh_slots_are_zeroed_before_first_copy():
             key = (st.sums, st.vmax2_bits, fX[:, :6].tobytes(), fV[:, :6].tobytes())
             want = want or key
             assert key == want
+
+
+def test_stream_modes_alternate_on_one_handle():
+    """One-step cycles and blocked trips on the same handle (the two kinds of
+    device slots are swapped in and out): the state carries through bit for bit."""
+    n = (18, 11, 35)
+    sp = P.SomierParams(n=n, seed=12)
+    with P.SomierStream(P.Spread([0], 1, n[0] - 2, chunk=5), sp, buffers=2) as s:
+        X, V = s.generate()
+        XN, VN = np.zeros_like(X), np.zeros_like(V)
+        s.run(X, V, XN, 3)                     # X_3 in XN, V in place
+        X, XN = XN, X
+        s.run_blocked(X, V, XN, VN, 4, 2)      # 2 trips: back in (X, V)
+        s.run(X, V, XN, 1)                     # X_8 in XN
+        X, XN = XN, X
+        st = s.run2(X, V, XN, VN, 3)[-1]       # 2 launches: back in (X, V)
+    ref, rst = O.run(O.init(_op(sp)), 11)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+    assert st.sums == rst.sums and st.step == 11

@@ -165,7 +165,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     const int k = k0 + lane;
     const int jA = j0 + 2 * w, jB = jA + 1;
     const int ck = lane + kCol0;
-    const int rA = 2 * w + 1, rB = rA + 1;  // box rows
+    const int rA = 2 * w + 1;  // box row of row A (row B: rA + 1)
     const int pb = 1 + blockIdx.y * mp.seg_planes;
     const int pe = min((int)g.size + 1, pb + mp.seg_planes);
     const int q0 = pb - 1;

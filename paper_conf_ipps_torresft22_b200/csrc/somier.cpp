@@ -224,22 +224,6 @@ spread_status load_driver_entry(somier_t h) {
     return SPREAD_OK;
 }
 
-// 4-D fp64 tensor map over a slab: dims (n2, n1, 3 components, planes), row
-// pitch ld. Box = (box_k, box_j, 3, 1): one plane tile per TMA.
-spread_status encode_slab_map(somier_t h, CUtensorMap* map, double* base, int64_t planes, uint32_t box_k,
-                              uint32_t box_j) {
-    const cuuint64_t dims[4] = {(cuuint64_t)h->p.n[2], (cuuint64_t)h->p.n[1], 3, (cuuint64_t)planes};
-    const cuuint64_t strides[3] = {(cuuint64_t)h->ld * 8, (cuuint64_t)(h->p.n[1] * h->ld) * 8,
-                                   (cuuint64_t)(3 * h->p.n[1] * h->ld) * 8};
-    const cuuint32_t box[4] = {box_k, box_j, 3, 1};
-    const cuuint32_t estr[4] = {1, 1, 1, 1};
-    CUresult r = h->encode_tiled(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, base, dims, strides, box, estr,
-                                 CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                                 CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier: cuTensorMapEncodeTiled failed (%d)", (int)r);
-    return SPREAD_OK;
-}
-
 void free_all(somier_t h) {
     if (!h) return;
     for (auto& c : h->chunks) {

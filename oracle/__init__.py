@@ -78,7 +78,9 @@ class Stats:
 def lib():
     global _lib
     if _lib is None:
-        path = build_oracle.build()
+        # ORACLE_LIB: an alternative build of somier_oracle.c (tools/mutate_oracle.py
+        # points it at deliberately broken mutants to show the pins catch them)
+        path = os.environ.get("ORACLE_LIB") or build_oracle.build()
         L = ctypes.CDLL(path)
         dp = ctypes.POINTER(ctypes.c_double)
         P = ctypes.POINTER(_Params)

@@ -20,7 +20,9 @@
  * (x, y, z components), like the paper's "3 3D-grids" per variable.
  *
  * Pins: every function below is pinned by tests/test_oracle_pins.py against
- * closed forms, invariants, brute force or printed values.
+ * closed forms, invariants, brute force or printed values,
+ * including mass M != 1 and rest length L != spacing (C2, C4, C7, C8); 22
+ * one-line mutants of this file each fail a pin (tools/mutate_oracle.py).
  * No function is "parity unpinned".
  */
 #ifndef SOMIER_ORACLE_H

@@ -153,6 +153,20 @@ spread_status somier_sync(somier_t h);
  */
 spread_status somier_stats(somier_t h, somier_stats_t* out);
 
+/*
+ * somier_stats_history -- blocking; the stats of EVERY step ("centers" after
+ * each time step): out[i] = the stats after step
+ * first_step + i, for count consecutive steps (step 0 = the initial state),
+ * each as somier_stats would have returned it right after that step. The
+ * handle keeps the last SOMIER_STATS_HISTORY steps since its last
+ * somier_init / somier_load (a device-side ring the step kernels write; every
+ * kernel, K1_TB2's two-step launches included, computes every step's stats).
+ * Errors: EINVAL (NULL with count > 0, count < 0, a step outside
+ * [max(last init/load step, step_count - SOMIER_STATS_HISTORY + 1), step_count]).
+ */
+#define SOMIER_STATS_HISTORY 126
+spread_status somier_stats_history(somier_t h, int64_t first_step, int64_t count, somier_stats_t* out);
+
 /* Exact, order-independent combination of n partial stats (sums added as int128,
  * max of vmax2 bits); recomputes centre = sum * 2^-60 / N_total and vmax. */
 spread_status somier_stats_combine(const somier_stats_t* parts, int n, const somier_params* p,
@@ -297,9 +311,8 @@ spread_status somier_stream_run(somier_stream_t h, double* x, double* y, double*
  *   nsteps / 2 two-step launches run, plus one one-step launch if nsteps is
  *   odd; the final state is in the first buffers if the number of launches
  *   is even, else in the second.
- *   stats: NULL, or an array of ceil(nsteps / 2) entries receiving the
- *   statistics after each launch (`step` says which step; the intermediate
- *   step of a two-step launch has no statistics, as on a K1_TB2 handle).
+ *   stats: NULL, or an array of nsteps entries receiving the statistics after
+ *   each step (both steps of a two-step launch).
  * Chunk-level dependencies as in somier_stream_run, over the chunks within
  * two planes. Results are bit-identical to somier_stream_run / the oracle.
  * Same as somier_stream_run_blocked with steps_per_trip = 2 (its device
@@ -321,7 +334,8 @@ spread_status somier_stream_run2(somier_stream_t h, double* x, double* y, double
  * the device recomputes the overlap (a chunk of S planes computes ~S + s
  * planes per step on average). Buffers alternate per trip as in run2 (the
  * final state is in the first buffers if the number of trips ceil(nsteps/s)
- * is even); stats: NULL or ceil(nsteps/s) entries, one per trip.
+ * is even); stats: NULL or nsteps entries, one per step (every launch of a
+ * trip counts the chunk's own planes only).
  * Device memory: `buffers` x 2 x (X and V of max_chunk + 2s + 2 planes) per
  * device, allocated on first use. Bit-identical to somier_stream_run.
  * Errors: EINVAL, ENOMEM, ECUDA.

@@ -20,6 +20,7 @@ OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -
 MAP_ALLOC, MAP_TO, MAP_FROM, MAP_TOFROM = 0, 1, 2, 3
 # somier_kernel
 K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2 = 0, 1, 2, 3, 4
+STATS_HISTORY = 126  # SOMIER_STATS_HISTORY (include/somier.h)
 
 
 class SpreadError(RuntimeError):
@@ -107,6 +108,7 @@ SIGNATURES = [
     ("somier_step", ctypes.c_int, [_VP, ctypes.c_int64]),
     ("somier_sync", ctypes.c_int, [_VP]),
     ("somier_stats", ctypes.c_int, [_VP, ctypes.POINTER(somier_stats_t)]),
+    ("somier_stats_history", ctypes.c_int, [_VP, ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
     ("somier_stats_combine", ctypes.c_int, [ctypes.POINTER(somier_stats_t), ctypes.c_int,
                                             ctypes.POINTER(somier_params), ctypes.POINTER(somier_stats_t)]),
     ("somier_read", ctypes.c_int, [_VP] + [_DP] * 6),

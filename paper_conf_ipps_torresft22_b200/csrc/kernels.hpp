@@ -33,8 +33,16 @@ struct StepArgs {
     double* hi_dst;         // right neighbour's lo-halo plane in ITS X_{t+1} buffer, or null
     SlabGeom g;
     double K, L, M, dt;
-    StatsAccum* acc;        // this step's stats slot (accumulated)
+    StatsAccum* acc;        // this step's stats slot (accumulated); K1_TB2: the last step's
     StatsAccum* acc_clear;  // the next step's slot (zeroed by block 0)
+    StatsAccum* acc_mid;    // K1_TB2 two-step launch: stats of the intermediate state t+1 (or null)
+    // Resident handles: per-step stats history (stats_layout.hpp). When
+    // step_word is non-null the launch reads the step number t from it, takes
+    // its slots in acc_ring (acc / acc_mid / acc_clear are ignored), and its last
+    // CTA advances *step_word by the steps it computed -- so a CUDA graph of
+    // launches needs no per-step arguments.
+    unsigned long long* step_word;
+    StatsAccum* acc_ring;
     // Completion signal for neighbours on other streams (fused exchange): the
     // last CTA stores `signal_value` with release semantics at system scope
     // into each non-null flag after every CTA's halo stores are fenced.
@@ -87,14 +95,18 @@ cudaError_t launch_k1(K1Variant variant, const StepArgs& a, bool unit_mass, cuda
 // plane of global i = start, lo_vdst = its V plane of i = start) and the last
 // two / last one to the right neighbour's (a.hi_dst = its X plane of i =
 // start+size-2, hi_vdst = its V plane of i = start+size-1); a.signal_* /
-// a.done_counter / a.signal_value as for the one-step kernels. Stats of the
-// last step only, into a.acc.
+// a.done_counter / a.signal_value as for the one-step kernels. Stats of both
+// steps: the ring (a.step_word) or a.acc_mid (state t+1) and a.acc (last state).
 struct Tb2Out {
     double* x_out;
     double* v_out;
     double* lo_vdst;
     double* hi_vdst;
     bool two;  // two steps (else one)
+    // global planes [stats_lo, stats_hi) whose nodes enter the stats (both 0:
+    // the launch's own planes [start, start+size)); a widened launch of a
+    // host-streamed trip counts only the chunk it maps out
+    int64_t stats_lo, stats_hi;
 };
 cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);

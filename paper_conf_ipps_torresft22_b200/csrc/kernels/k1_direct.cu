@@ -21,9 +21,8 @@ __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
     const int64_t k = (int64_t)blockIdx.x * kBX + threadIdx.x;
     const int64_t j = (int64_t)blockIdx.y * kBY + threadIdx.y;
     const int64_t p = blockIdx.z;  // owned plane 0..size-1 -> X slab plane p+1
-    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && threadIdx.x < 8 &&
-        threadIdx.y == 0)
-        reinterpret_cast<unsigned long long*>(a.acc_clear)[threadIdx.x] = 0ull;
+    const LaunchSlots slots = launch_slots(a, 1, blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0,
+                                           threadIdx.y * kBX + threadIdx.x);
 
     NodeStats st;
     st.zero();
@@ -75,8 +74,8 @@ __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
             }
         }
     }
-    block_accumulate(st, scratch, a.acc);
-    signal_neighbours(a);
+    block_accumulate(st, scratch, slots.fin);
+    finish_launch(a, slots.t, 1);
 }
 
 }  // namespace

@@ -144,8 +144,7 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     const int q0 = pb - 1;  // first loaded plane
     const int qlast = pe;   // last loaded plane
 
-    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
-        reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
+    const LaunchSlots slots = launch_slots(a, 1, blockIdx.x == 0 && blockIdx.y == 0, tid);
 
     auto issue = [&](int q) {  // TMA for plane q into its stage (thread 0 only)
         const int s = (q - q0) % kStages;
@@ -268,8 +267,8 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
         s_nxt = (s_nxt + 1 == kStages) ? 0 : s_nxt + 1;
         ph_nxt ^= (s_nxt == 0) ? 1u : 0u;
     }
-    block_accumulate(st, sm.scratch, a.acc);
-    signal_neighbours(a);
+    block_accumulate(st, sm.scratch, slots.fin);
+    finish_launch(a, slots.t, 1);
 }
 
 }  // namespace

@@ -198,8 +198,7 @@ __global__ void __launch_bounds__(kThreads, 2)
     // here on global memory is touched (it read the X buffer this step writes,
     // and wrote the X_t / V this step reads). A no-op without PDL.
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    if (a.acc_clear && blockIdx.x == 0 && blockIdx.y == 0 && tid < 8)
-        reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
+    const LaunchSlots slots = launch_slots(a, 1, blockIdx.x == 0 && blockIdx.y == 0, tid);
     // Every CTA is resident once all have passed this point, so the next
     // step's CTAs can only take slots freed by finished CTAs of this one.
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -299,8 +298,8 @@ __global__ void __launch_bounds__(kThreads, 2)
         s_nxt = (s_nxt + 1 == kStages) ? 0 : s_nxt + 1;
         ph_nxt ^= (s_nxt == 0) ? 1u : 0u;
     }
-    block_accumulate(st, sm.scratch, a.acc);
-    signal_neighbours(a);
+    block_accumulate(st, sm.scratch, slots.fin);
+    finish_launch(a, slots.t, 1);
 }
 
 }  // namespace

@@ -21,9 +21,10 @@
 // +k per node; -i from a register carry, -k from a lane shuffle, -j from the
 // paired row or shared memory), two CTA barriers per plane. Both steps use
 // node_math.cuh, so every node update is the same IEEE expression as in
-// K1_DIRECT / K1_MARCH2 (bit-identical). Only step t+1's stats are accumulated:
-// the handle's stats are those of the last completed step, and TB2 always
-// completes steps in pairs.
+// K1_DIRECT / K1_MARCH2 (bit-identical). The stats ("centers", PAPER.md:330,
+// 354) of BOTH steps are accumulated over the owned nodes of the output planes:
+// step t+1's from S2's results, step t's from the S1 results S2 reads anyway
+// (X_{t+1} of plane q from the shared ring, V_{t+1} from the register carry).
 #include <cuda.h>
 
 #include <algorithm>
@@ -91,6 +92,7 @@ struct Tb2Params {
     double* hi_vdst;               // right neighbour's V halo plane in ITS out buffer, or null
     int x_base, v_base;            // global i of raw plane 0 of the X / V slabs (start - 2, start - 1)
     int lo_end, hi_begin;          // planes q < lo_end go to lo_dst + (q - start), q >= hi_begin to hi_dst + (q - hi_begin)
+    int stats_lo, stats_hi;        // output planes [stats_lo, stats_hi) contribute to the stats
     int tiles_k, tiles_j, seg_planes;
 };
 
@@ -133,6 +135,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int q0 = max(0, ps0 - 1);                        // X_t planes [q0, qlast]
     const int qlast = min(ilast + 1, pe + 1);
     const int v_first = max(1, ps0), v_last = min(ilast, pe);  // V_t planes read (S1 on non-fixed planes)
+    const LaunchSlots slots = launch_slots(a, kTwo ? 2 : 1, blockIdx.x == 0 && blockIdx.y == 0, tid);
 
     auto issue_x = [&](int q) {
         const int s = (q - q0) % kStages;
@@ -206,8 +209,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     Vec3 carry2A{0.0, 0.0, 0.0}, carry2B{0.0, 0.0, 0.0};
     Vec3 v1pA{0.0, 0.0, 0.0}, v1pB{0.0, 0.0, 0.0};  // V_{t+1} of plane p-1
-    NodeStats st;
+    NodeStats st, st1;  // stats of the launch's last step (t+2, or t+1 in one-step mode) and of step t+1
     st.zero();
+    st1.zero();
     const int border_last = min(pe, ilast);  // planes whose border springs S1 needs
     // X_{t+2} (X_{t+1}), V of an S2 output node: own slab, and the neighbours'
     // halo planes (2 planes of X, 1 of V per face: what their next launch reads)
@@ -318,6 +322,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             issue_v(p + kVStages);
         }
         // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q (one-step mode: X_{t+1}, V_{t+1} of S1)
+        const bool sq = kFull ? (q >= tp.stats_lo && q < tp.stats_hi) : (out2 && q >= tp.stats_lo && q < tp.stats_hi);
         if (out2) {
             if (ownA) {
                 if (intA) {
@@ -326,12 +331,19 @@ __global__ void __launch_bounds__(kThreads, 1)
                         const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
+                        if (sq) {
+                            st1.add_position_nc(xqA);  // step t+1: X_{t+1}, V_{t+1} of this node
+                            st1.add_velocity(v1pA);
+                        }
                     }
                     store_out(q, offA, x2, v2);
-                    st.add_position(x2);
-                    st.add_velocity(v2);
-                } else {
+                    if (sq) {
+                        st.add_position(x2);
+                        st.add_velocity(v2);
+                    }
+                } else if (sq) {
                     st.add_position(xqA);  // fixed face node
+                    if (kTwo) st1.add_position_nc(xqA);
                 }
             }
             if (ownB) {
@@ -340,12 +352,19 @@ __global__ void __launch_bounds__(kThreads, 1)
                     if (kTwo) {
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
+                        if (sq) {
+                            st1.add_position_nc(xqB);
+                            st1.add_velocity(v1pB);
+                        }
                     }
                     store_out(q, offB, x2, v2);
-                    st.add_position(x2);
-                    st.add_velocity(v2);
-                } else {
+                    if (sq) {
+                        st.add_position(x2);
+                        st.add_velocity(v2);
+                    }
+                } else if (sq) {
                     st.add_position(xqB);
+                    if (kTwo) st1.add_position_nc(xqB);
                 }
             }
         }
@@ -376,8 +395,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     if (p <= hi) body(F1{}, P0{}, p++);
     for (; p <= pe; p++) body(F0{}, PN{}, p);
-    block_accumulate(st, sm.scratch, a.acc);
-    signal_neighbours(a);
+    block_accumulate(st, sm.scratch, slots.fin);
+    if (kTwo) {
+        st1.copy_count(st);
+        __syncthreads();  // scratch reuse
+        block_accumulate(st1, sm.scratch, slots.mid);
+    }
+    finish_launch(a, slots.t, kTwo ? 2 : 1);
 }
 
 }  // namespace
@@ -385,6 +409,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream) {
     if (a.g.size <= 0) return cudaSuccess;
     if (!a.tmap_x_cur || !a.tmap_v || !o.x_out || !o.v_out) return cudaErrorInvalidValue;
+    if (!a.step_word && (!a.acc || (o.two && !a.acc_mid))) return cudaErrorInvalidValue;  // both steps' stats slots
     if ((a.lo_dst && (!o.lo_vdst || a.g.size < 2)) || (a.hi_dst && (!o.hi_vdst || a.g.size < 2)))
         return cudaErrorInvalidValue;  // a neighbour's two halo planes come from one chunk
     Tb2Params tp;
@@ -397,6 +422,12 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
     tp.v_base = (int)a.g.start - 1;
     tp.lo_end = a.lo_dst ? (int)a.g.start + 2 : INT_MIN;
     tp.hi_begin = a.hi_dst ? (int)(a.g.start + a.g.size) - 2 : INT_MAX;
+    tp.stats_lo = o.stats_lo;
+    tp.stats_hi = o.stats_hi;
+    if (o.stats_lo == 0 && o.stats_hi == 0) {  // default: the chunk's own planes
+        tp.stats_lo = (int)a.g.start;
+        tp.stats_hi = (int)(a.g.start + a.g.size);
+    }
     tp.tiles_k = (int)((a.g.n2 - 2 + kOK - 1) / kOK);
     tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;

@@ -13,22 +13,26 @@ __device__ __forceinline__ void st_release_sys_u64(unsigned long long* p, unsign
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Call once per CTA, by all threads, after the CTA's last store.
-__device__ __forceinline__ void signal_neighbours(const StepArgs& a) {
-    if (!a.signal_lo && !a.signal_hi) return;
+// Call once per CTA, by all threads, after the CTA's last store. The last CTA
+// of the launch to finish advances the step word (stats ring, t = the step the
+// launch started from) and publishes the neighbours' flags.
+__device__ __forceinline__ void finish_launch(const StepArgs& a, unsigned long long t, int nsteps) {
+    const bool sig = a.signal_lo || a.signal_hi;
+    if (!sig && !a.step_word) return;
     __shared__ unsigned int s_last;
     __syncthreads();
     const bool leader = threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0;
     if (leader) {
-        __threadfence_system();
+        if (sig) __threadfence_system();
         const unsigned int nblocks = gridDim.x * gridDim.y * gridDim.z;
         const unsigned int prev = atomicAdd(a.done_counter, 1u);
         s_last = (prev == nblocks - 1) ? 1u : 0u;
     }
     __syncthreads();
     if (leader && s_last) {
-        __threadfence_system();
+        if (sig) __threadfence_system();
         *a.done_counter = 0u;  // self-reset for the next step (stream-ordered)
+        if (a.step_word) *a.step_word = t + (unsigned long long)nsteps;
         if (a.signal_lo) st_release_sys_u64(a.signal_lo, a.signal_value);
         if (a.signal_hi) st_release_sys_u64(a.signal_hi, a.signal_value);
     }

@@ -63,6 +63,14 @@ struct NodeStats {
         add_coord(2, x.z);
         n++;
     }
+    // a position whose node is counted by another NodeStats over the same node
+    // set (K1_TB2's two steps): set n from that one before sum()
+    __device__ __forceinline__ void add_position_nc(const Vec3& x) {
+        add_coord(0, x.x);
+        add_coord(1, x.y);
+        add_coord(2, x.z);
+    }
+    __device__ __forceinline__ void copy_count(const NodeStats& o) { n = o.n; }
     __device__ __forceinline__ void add_velocity(const Vec3& v) {
         const double v2 = dot_self(v);
         vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
@@ -100,6 +108,8 @@ struct NodeStats {
         add_coord(1, x.y);
         add_coord(2, x.z);
     }
+    __device__ __forceinline__ void add_position_nc(const Vec3& x) { add_position(x); }
+    __device__ __forceinline__ void copy_count(const NodeStats&) {}
     __device__ __forceinline__ void add_velocity(const Vec3& v) {
         const double v2 = dot_self(v);
         vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
@@ -114,6 +124,40 @@ struct NodeStats {
 };
 
 #endif
+
+// The stats slots of one launch that advances `nsteps` (1 or 2) steps. With a
+// step word (resident handles, stats_layout.hpp) the step number t comes from
+// device memory -- written by the previous launch's last CTA, read after any
+// griddepcontrol.wait -- and the slots from the ring: states t+1 (mid) and
+// t+nsteps (fin); block 0 zeroes the slots of states t+nsteps+1, t+nsteps+2.
+// Without one the explicit a.acc / a.acc_mid / a.acc_clear are used.
+struct LaunchSlots {
+    StatsAccum* fin;
+    StatsAccum* mid;
+    unsigned long long t;
+};
+
+template <class Args>
+__device__ __forceinline__ LaunchSlots launch_slots(const Args& a, int nsteps, bool block0, int tid) {
+    LaunchSlots s;
+    if (a.step_word) {
+        unsigned long long t;
+        asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(t) : "l"(a.step_word) : "memory");
+        s.t = t;
+        s.fin = a.acc_ring + ring_slot(t + nsteps);
+        s.mid = a.acc_ring + ring_slot(t + 1);
+        if (block0 && tid < 16) {
+            StatsAccum* c = a.acc_ring + ring_slot(t + nsteps + 1 + (tid >> 3));
+            reinterpret_cast<unsigned long long*>(c)[tid & 7] = 0ull;
+        }
+    } else {
+        s.t = 0;
+        s.fin = a.acc;
+        s.mid = a.acc_mid;
+        if (a.acc_clear && block0 && tid < 8) reinterpret_cast<unsigned long long*>(a.acc_clear)[tid] = 0ull;
+    }
+    return s;
+}
 
 struct I128Stats {
     __int128 s[3];

@@ -28,7 +28,7 @@ using paper::set_last_error;
 namespace {
 
 constexpr uint64_t kIpcMagic = 0x534f4d4945524950ull;  // "SOMIERIP"
-constexpr uint32_t kIpcVersion = 3;
+constexpr uint32_t kIpcVersion = 4;
 
 using PFN_waitValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 using PFN_encodeTiled = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -50,9 +50,11 @@ struct Chunk {
     int64_t index = 0, start = 0, size = 0;
     int pos = 0, device = 0;
     bool local = false;
-    // local allocation: [x0 | x1 | v0 | (v1, K1_TB2 only) | acc[4] | flags[2] | counter]
-    // acc: [0], [1] stats of the last steps by step parity, [2] the fixed end
-    // planes, [3] unused.
+    // local allocation: [x0 | x1 | v0 | (v1, K1_TB2 only) | acc[kStatsRing + 2] | flags[2] | counter | step word]
+    // acc: [0, kStatsRing) per-step stats history (state s in ring_slot(s)),
+    // [kStatsRing] the fixed nodes no launch visits (end planes held as halos,
+    // K1_TB2's k-face columns), [kStatsRing + 1] unused. The step word is the
+    // device copy of the step counter the kernels take their ring slots from.
     // X slabs: planes [start-1, start+size+1) (one halo plane per face), V
     // slabs [start, start+size); on a K1_TB2 handle one more halo plane per
     // face each (X [start-2, start+size+2), V [start-1, start+size+1)) and V
@@ -79,6 +81,8 @@ struct Chunk {
     paper::StatsAccum* acc() const { return (paper::StatsAccum*)((char*)mem() + off_acc); }
     unsigned long long* flags() const { return (unsigned long long*)((char*)mem() + off_flags); }
     unsigned int* counter() const { return (unsigned int*)((char*)mem() + off_counter); }
+    unsigned long long* step_word() const { return (unsigned long long*)((char*)mem() + off_counter + 8); }
+    paper::StatsAccum* acc_static() const { return acc() + paper::kStatsRing; }
 };
 
 struct IpcChunkRecord {
@@ -127,6 +131,7 @@ struct somier_s {
     paper::SlabGeom geom{};  // start/size filled per chunk
     int64_t ld = 0;
     int64_t step = 0;
+    int64_t hist_first = 0;  // oldest state whose stats are in the history ring (last init / load)
     int64_t launches = 0;
     int xbuf = 0;      // X buffer holding X_t (flips once per launch)
     int vbuf = 0;      // V buffer holding V_t (flips once per K1_TB2 launch; 1-step kernels update in place)
@@ -249,26 +254,28 @@ void free_all(somier_t h) {
     }
 }
 
-// Recompute the stats slots of a chunk from its resident state: slot (step-1)&1
-// = stats of the current state, slot step&1 zeroed, slot 2 = the fixed end
+// Recompute the stats slots of a chunk from its resident state: the history
+// ring is cleared (the stats of earlier states are gone) and ring_slot(step)
+// receives the stats of the current state; the static slot the fixed end
 // planes the chunk holds as halos (global i = 0 and i = n0-1) and, on K1_TB2
 // handles, the fixed k-face columns of its owned planes (which the kernel's
-// tiles do not own) -- those are then left out of the current slot.
+// tiles do not own) -- those are then left out of the per-step slots.
 spread_status reset_stats(somier_t h, Chunk& c) {
     cudaStream_t s = h->stream_of(c);
     paper::SlabGeom g = h->geom_of(c);
-    CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, 4 * sizeof(paper::StatsAccum), s));
+    CUDA_TRY(h, cudaMemsetAsync(c.acc(), 0, (paper::kStatsRing + 2) * sizeof(paper::StatsAccum), s));
     const int cur = h->xbuf;
-    paper::StatsAccum* last = c.acc() + ((h->step - 1) & 1);
+    paper::StatsAccum* last = c.acc() + paper::ring_slot((unsigned long long)h->step);
     CUDA_TRY(h, paper::launch_stats(c.xs(cur), c.vs(h->vbuf), g, 1, c.size, last, s, h->tb2));
-    if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, 0, 1, c.acc() + 2, s));
+    if (c.start == 1) CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, 0, 1, c.acc_static(), s));
     if (c.start + c.size == h->p.n[0] - 1)
-        CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, c.size + 1, 1, c.acc() + 2, s));
+        CUDA_TRY(h, paper::launch_stats(c.xs(cur), nullptr, g, c.size + 1, 1, c.acc_static(), s));
     if (h->tb2) {
         // K1_TB2 does not own the fixed k-face columns of its planes: their
         // constant positions are counted here once, in the static slot
-        CUDA_TRY(h, paper::launch_kface_stats(c.xs(cur), g, 1, c.size, c.acc() + 2, s));
+        CUDA_TRY(h, paper::launch_kface_stats(c.xs(cur), g, 1, c.size, c.acc_static(), s));
     }
+    h->hist_first = h->step;
     return SPREAD_OK;
 }
 
@@ -284,8 +291,8 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     c.off_v = 2 * xb;
     c.off_v1 = h->tb2 ? c.off_v + vb : c.off_v;
     c.off_acc = c.off_v + (h->tb2 ? 2 : 1) * vb;
-    c.off_flags = c.off_acc + 4 * sizeof(paper::StatsAccum);
-    c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);
+    c.off_flags = c.off_acc + (paper::kStatsRing + 2) * sizeof(paper::StatsAccum);
+    c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);  // counter (4 B, padded to 8) + step word
     c.bytes = round_up(c.off_counter + 64, 4096);
     CUDA_TRY(h, cudaSetDevice(c.device));
     CUDA_TRY(h, cudaMalloc(&c.base, c.bytes));
@@ -825,7 +832,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
     for (int64_t s = 0; s < nsteps; s++) {
         const int64_t t = h->step;
         const int cur = h->xbuf, nxt = cur ^ 1;       // X buffers
-        const int slot = (int)(t & 1), vb = h->vbuf;  // stats slot of step t; V buffer
+        const int vb = h->vbuf;  // V buffer
         for (int64_t c = 0; c < nch; c++) {
             Chunk& me = h->chunks[c];
             if (!me.local) continue;
@@ -863,8 +870,8 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.L = h->p.rest_len;
             a.M = h->p.mass;
             a.dt = h->p.dt;
-            a.acc = me.acc() + slot;
-            a.acc_clear = me.acc() + (slot ^ 1);
+            a.step_word = me.step_word();  // the kernel takes its ring slots from the device step counter
+            a.acc_ring = me.acc();
             a.signal_lo = fl ? &left->flags()[1] : nullptr;
             a.signal_hi = fr ? &right->flags()[0] : nullptr;
             a.signal_value = (unsigned long long)(t + 1);
@@ -888,13 +895,12 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
 // writes the other buffers, its boundary planes also into the neighbours'
 // other buffers; flags as in enqueue_steps (the neighbours finished the launch
 // that produced step t: my halo planes of X_t / V_t are written, and they no
-// longer read their buffers I write into). Stats of the last step go to slot
-// (t_end - 1) & 1, zeroed first.
+// longer read their buffers I write into). Stats of both steps go to the
+// history ring (slots from the device step word).
 spread_status enqueue_tb2(somier_t h, bool two) {
     const int64_t nch = (int64_t)h->chunks.size();
     const int64_t t = h->step, t_end = t + (two ? 2 : 1);
     const int cur = h->xbuf, vb = h->vbuf;
-    const int slot = (int)((t_end - 1) & 1);
     const int64_t ps = h->geom.plane_stride();
     int cur_dev = -1;
     for (int64_t c = 0; c < nch; c++) {
@@ -915,7 +921,6 @@ spread_status enqueue_tb2(somier_t h, bool two) {
                                          CU_STREAM_WAIT_VALUE_GEQ | h->devs[me.pos].wait_flush);
             if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWaitValue64 failed (%d)", (int)r);
         }
-        CUDA_TRY(h, cudaMemsetAsync(me.acc() + slot, 0, sizeof(paper::StatsAccum), st));
         paper::StepArgs a;
         std::memset(&a, 0, sizeof a);
         a.x_cur = me.x(cur);
@@ -925,7 +930,8 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         a.L = h->p.rest_len;
         a.M = h->p.mass;
         a.dt = h->p.dt;
-        a.acc = me.acc() + slot;
+        a.step_word = me.step_word();
+        a.acc_ring = me.acc();
         a.tmap_x_cur = &me.tmap_xt[cur];
         a.tmap_v = &me.tmap_vt[vb];
         paper::Tb2Out o;
@@ -967,28 +973,43 @@ spread_status somier_sync(somier_t h) {
     return sync_all(h);
 }
 
-spread_status somier_stats(somier_t h, somier_stats_t* out) {
-    if (!h || !out) PAPER_FAIL(SPREAD_EINVAL, "somier_stats: NULL argument");
+static_assert(SOMIER_STATS_HISTORY == paper::kStatsHistory, "somier.h history depth");
+
+spread_status somier_stats_history(somier_t h, int64_t first_step, int64_t count, somier_stats_t* out) {
+    if (!h || (count > 0 && !out)) PAPER_FAIL(SPREAD_EINVAL, "somier_stats_history: NULL argument");
+    if (count < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_stats_history: count < 0");
+    const int64_t lo = std::max(h->hist_first, h->step - (int64_t)paper::kStatsHistory + 1);
+    if (count > 0 && (first_step < lo || first_step + count - 1 > h->step))
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stats_history: steps [%lld, %lld] outside the history [%lld, %lld]",
+                   (long long)first_step, (long long)(first_step + count - 1), (long long)lo, (long long)h->step);
     spread_status st = sync_all(h);
     if (st != SPREAD_OK) return st;
-    __int128 sums[3] = {0, 0, 0};
-    unsigned long long vmax2 = 0;
+    if (count == 0) return SPREAD_OK;
+    std::vector<__int128> sums((size_t)count * 3, 0);
+    std::vector<unsigned long long> vmax2((size_t)count, 0ull);
     int64_t nodes = 0;
-    const int slot = (int)((h->step - 1) & 1);
+    std::vector<paper::StatsAccum> acc(paper::kStatsRing + 1);
     for (auto& c : h->chunks) {
         if (!c.local) continue;
-        paper::StatsAccum acc[3];
         CUDA_TRY(h, cudaSetDevice(c.device));
-        CUDA_TRY(h, cudaMemcpy(acc, c.acc(), sizeof acc, cudaMemcpyDeviceToHost));
-        for (int q : {slot, 2}) {
-            for (int d = 0; d < 3; d++)
-                sums[d] += (__int128)(((unsigned __int128)acc[q].hi[d] << 64) | acc[q].lo[d]);
-            vmax2 = std::max(vmax2, (unsigned long long)acc[q].vmax2);
+        CUDA_TRY(h, cudaMemcpy(acc.data(), c.acc(), acc.size() * sizeof(paper::StatsAccum), cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < count; i++) {
+            for (int q : {paper::ring_slot((unsigned long long)(first_step + i)), paper::kStatsRing}) {
+                for (int d = 0; d < 3; d++)
+                    sums[(size_t)(3 * i + d)] += (__int128)(((unsigned __int128)acc[q].hi[d] << 64) | acc[q].lo[d]);
+                vmax2[(size_t)i] = std::max(vmax2[(size_t)i], (unsigned long long)acc[q].vmax2);
+            }
         }
         nodes += owned_nodes(h, c);
     }
-    finish_stats(&h->p, sums, vmax2, nodes, h->step, out);
+    for (int64_t i = 0; i < count; i++)
+        finish_stats(&h->p, &sums[(size_t)(3 * i)], vmax2[(size_t)i], nodes, first_step + i, &out[i]);
     return SPREAD_OK;
+}
+
+spread_status somier_stats(somier_t h, somier_stats_t* out) {
+    if (!h || !out) PAPER_FAIL(SPREAD_EINVAL, "somier_stats: NULL argument");
+    return somier_stats_history(h, h->step, 1, out);
 }
 
 spread_status somier_stats_combine(const somier_stats_t* parts, int n, const somier_params* p, somier_stats_t* out) {
@@ -1099,7 +1120,36 @@ spread_status somier_load(somier_t h, const double* x, const double* y, const do
         spread_status st = reset_stats(h, c);
         if (st != SPREAD_OK) return st;
     }
-    return SPREAD_OK;
+    // The copy above replaces the chunk's whole X_{t+1} buffer, halo planes
+    // included, which the neighbours' next step stores into from THEIR streams
+    // (their flag waits are already satisfied): order every other position's
+    // stream after this position's load. Other processes cannot be ordered
+    // from here: multi-process loads complete before returning (the caller's
+    // barrier then orders them, include/somier.h).
+    if (h->multi_process) return sync_all(h);
+    std::vector<cudaEvent_t> evs;
+    spread_status st = SPREAD_OK;
+    for (size_t q = 0; q < h->devs.size() && st == SPREAD_OK; q++) {
+        DevCtx& d = h->devs[q];
+        if (!d.stream) continue;
+        cudaEvent_t ev = nullptr;
+        cudaError_t e = cudaSetDevice(d.device);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+        if (e == cudaSuccess) evs.push_back(ev);
+        if (e == cudaSuccess) e = cudaEventRecord(ev, d.stream);
+        if (e != cudaSuccess) st = cuda_fail(h, e, "somier_load: event");
+    }
+    for (size_t q = 0, i = 0; q < h->devs.size() && st == SPREAD_OK; q++) {
+        DevCtx& d = h->devs[q];
+        if (!d.stream) continue;
+        cudaError_t e = cudaSetDevice(d.device);
+        for (size_t r = 0; r < evs.size() && e == cudaSuccess; r++)
+            if (r != i) e = cudaStreamWaitEvent(d.stream, evs[r], 0);
+        if (e != cudaSuccess) st = cuda_fail(h, e, "somier_load: stream wait");
+        i++;
+    }
+    for (cudaEvent_t ev : evs) cudaEventDestroy(ev);
+    return st;
 }
 
 spread_status somier_set_stream(somier_t h, int device_pos, void* stream) {

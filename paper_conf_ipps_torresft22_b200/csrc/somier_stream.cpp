@@ -66,11 +66,13 @@ struct Dev {
     cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
     std::vector<Slot> slots;
     std::vector<DeepSlot> deep;
-    paper::StatsAccum* scratch_acc = nullptr;  // stats of the widened intermediate launches (discarded)
-    void* acc_base = nullptr;  // StatsAccum[acc_steps][2]: per step, chunk sums and fixed end planes
+    // StatsAccum[1 + acc_steps]: [0] the fixed nodes no launch visits (end
+    // planes, K1_TB2's k-face columns), then one slot per step of the run
+    void* acc_base = nullptr;
     int64_t acc_steps = 0;
     std::vector<int64_t> chunks;
-    paper::StatsAccum* acc(int64_t t) const { return (paper::StatsAccum*)acc_base + 2 * t; }
+    paper::StatsAccum* acc(int64_t t) const { return (paper::StatsAccum*)acc_base + 1 + t; }
+    paper::StatsAccum* acc_static() const { return (paper::StatsAccum*)acc_base; }
 };
 
 }  // namespace
@@ -122,7 +124,6 @@ void destroy_all(somier_stream_t h) {
                 if (e) cudaEventDestroy(e);
             if (sl.base) cudaFree(sl.base);
         }
-        if (d.scratch_acc) cudaFree(d.scratch_acc);
         if (d.acc_base) cudaFree(d.acc_base);
         for (cudaStream_t s : {d.s_h2d, d.s_comp, d.s_d2h})
             if (s) cudaStreamDestroy(s);
@@ -163,7 +164,7 @@ spread_status ensure_acc(somier_stream_t h, int64_t nsteps) {
         S_TRY(h, cudaFree(d.acc_base));
         d.acc_base = nullptr;
         d.acc_steps = 0;
-        S_TRY(h, cudaMalloc(&d.acc_base, 2 * (size_t)nsteps * sizeof(paper::StatsAccum)));
+        S_TRY(h, cudaMalloc(&d.acc_base, (1 + (size_t)nsteps) * sizeof(paper::StatsAccum)));
         d.acc_steps = nsteps;
     }
     return SPREAD_OK;
@@ -202,8 +203,10 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         // the fused step (forces, accelerations, velocities, positions, centers)
         S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
         paper::StatsAccum* acc = d.acc(t);
-        if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, acc + 1, d.s_comp));
-        if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, ci.size + 1, 1, acc + 1, d.s_comp));
+        if (t == 0) {  // the fixed end planes, once per run (they never move)
+            if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, d.acc_static(), d.s_comp));
+            if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, ci.size + 1, 1, d.acc_static(), d.s_comp));
+        }
         paper::StepArgs a;
         std::memset(&a, 0, sizeof a);
         a.x_cur = sl.x_in;
@@ -250,18 +253,19 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
     return SPREAD_OK;
 }
 
-// Combine the per-launch stats slots of every device into stats[0 .. n).
+// Combine the per-step stats slots of every device (plus its static slot)
+// into stats[0 .. n).
 spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, somier_stats_t* stats) {
     std::vector<__int128> sums((size_t)n * 3, 0);
     std::vector<unsigned long long> vmax2((size_t)n, 0);
-    std::vector<paper::StatsAccum> acc((size_t)n * 2);
+    std::vector<paper::StatsAccum> acc((size_t)n + 1);
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaMemcpy(acc.data(), d.acc_base, acc.size() * sizeof(paper::StatsAccum), cudaMemcpyDeviceToHost));
         for (int64_t t = 0; t < n; t++)
-            for (int q = 0; q < 2; q++) {
-                const paper::StatsAccum& a = acc[(size_t)(2 * t + q)];
+            for (size_t q : {(size_t)0, (size_t)(t + 1)}) {
+                const paper::StatsAccum& a = acc[q];
                 for (int k = 0; k < 3; k++)
                     sums[(size_t)(3 * t + k)] += (__int128)(((unsigned __int128)a.hi[k] << 64) | a.lo[k]);
                 vmax2[(size_t)t] = std::max(vmax2[(size_t)t], (unsigned long long)a.vmax2);
@@ -290,11 +294,14 @@ spread_status ensure_flat(somier_stream_t h) {
     const size_t xb = round_up(plane * (size_t)(h->max_chunk + 2), 4096);
     const size_t vb = round_up(plane * (size_t)h->max_chunk, 4096);
     for (auto& d : h->devs) {
-        if (d.chunks.empty() || d.slots.empty() || d.slots[0].base) continue;
+        bool missing = false;
+        for (auto& sl : d.slots) missing = missing || !sl.base;
+        if (d.chunks.empty() || !missing) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaDeviceSynchronize());
         release_deep(d);
         for (auto& sl : d.slots) {
+            if (sl.base) continue;
             S_TRY(h, cudaMalloc(&sl.base, 2 * xb + vb));
             sl.x_in = (double*)sl.base;
             sl.x_out = (double*)((char*)sl.base + xb);
@@ -322,12 +329,12 @@ spread_status ensure_deep(somier_stream_t h, int64_t planes) {
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         S_TRY(h, cudaSetDevice(d.device));
-        if (!d.scratch_acc) S_TRY(h, cudaMalloc(&d.scratch_acc, sizeof(paper::StatsAccum)));
         if (!d.deep.empty() && d.deep[0].base && d.deep[0].planes >= planes) continue;
         S_TRY(h, cudaDeviceSynchronize());
         for (auto& sl : d.slots) {  // the one-step slots give their memory up (ensure_flat restores them)
             if (sl.base) cudaFree(sl.base);
             sl.base = nullptr;
+            sl.x_in = sl.x_out = sl.v = nullptr;
         }
         for (auto& sl : d.deep)
             if (sl.base) S_TRY(h, cudaFree(sl.base));
@@ -367,8 +374,12 @@ void reach_range(const somier_stream_s* h, const paper::ChunkInfo& ci, int64_t d
 // steps with ceil(s/2) K1_TB2 launches over regions that shrink by two planes
 // per side per launch (the last one is the chunk itself; an odd s ends with a
 // one-step launch), and maps X_{t+s}, V_{t+s} of its planes out into (XN, VN).
+//   t0: the run's step index of the trip's first step (stats of step t0 + j go
+//       to d.acc(t0 + j)); s_prev: the previous trip's depth (its H2D read
+//       s_prev planes around each chunk, which this trip's D2H overwrites)
 spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
-                                     double* const VN[3], int64_t k, int64_t s, bool chained) {
+                                     double* const VN[3], int64_t k, int64_t s, int64_t t0, int64_t s_prev,
+                                     bool chained) {
     const int64_t n0 = h->p.n[0];
     const int64_t nch = h->spread.nchunks;
     const int64_t ps = h->geom.plane_stride();
@@ -381,8 +392,9 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
         DeepSlot& sl = d.deep[m % d.deep.size()];
         const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
         ChunkEvents& ev = h->ev[(size_t)c];
-        int64_t c_lo, c_hi;
-        reach_range(h, ci, s, &c_lo, &c_hi);
+        int64_t c_lo, c_hi, w_lo, w_hi;
+        reach_range(h, ci, s, &c_lo, &c_hi);           // H2D waits: the D2H of the chunks this trip reads
+        reach_range(h, ci, std::max(s, s_prev), &w_lo, &w_hi);  // D2H waits: the H2D that read what it overwrites
         // global plane of raw plane 0 of the X / V buffers: one plane of slack
         // beyond the s-plane halo on each side (a one-step launch still reads
         // the deep layout's outer ring plane, whose values it does not use)
@@ -409,12 +421,13 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
         // the fixed face nodes of every output plane (K1_TB2 writes the moving nodes only)
         S_TRY(h, cudaMemcpyAsync(sl.xb + (xlo - x0) * ps, sl.xa + (xlo - x0) * ps,
                                  (size_t)((xhi - xlo) * ps) * sizeof(double), cudaMemcpyDeviceToDevice, d.s_comp));
-        paper::StatsAccum* acc = d.acc(k);
-        double* xv_one = sl.xa + (ci.start - 1 - x0) * ps;  // one-step view: raw plane 0 = start - 1
-        if (first) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, 0, 1, acc + 1, d.s_comp));
-        if (last) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, ci.size + 1, 1, acc + 1, d.s_comp));
-        S_TRY(h, paper::launch_kface_stats(xv_one, g, 1, ci.size, acc + 1, d.s_comp));
-        int64_t remaining = s;
+        if (k == 0) {  // the fixed nodes no launch visits, once per run
+            double* xv_one = sl.xa + (ci.start - 1 - x0) * ps;  // one-step view: raw plane 0 = start - 1
+            if (first) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, 0, 1, d.acc_static(), d.s_comp));
+            if (last) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, ci.size + 1, 1, d.acc_static(), d.s_comp));
+            S_TRY(h, paper::launch_kface_stats(xv_one, g, 1, ci.size, d.acc_static(), d.s_comp));
+        }
+        int64_t remaining = s, done = 0;
         double *xin = sl.xa, *xout = sl.xb, *vin = sl.va, *vout = sl.vb;
         for (int64_t j = 0; j < nl; j++) {
             const bool two = remaining >= 2;
@@ -438,7 +451,9 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             a.L = h->p.rest_len;
             a.M = h->p.mass;
             a.dt = h->p.dt;
-            a.acc = j + 1 == nl ? acc : d.scratch_acc;
+            // every launch counts the chunk's own planes only: stats of every step
+            a.acc_mid = d.acc(t0 + done);
+            a.acc = d.acc(t0 + done + (two ? 1 : 0));
             a.tmap_x_cur = &mx;
             a.tmap_v = &mv;
             paper::Tb2Out o;
@@ -446,16 +461,19 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             o.x_out = xout + (gj.start - 2 - x0) * ps;
             o.v_out = vout + (gj.start - 1 - v0) * ps;
             o.two = two;
+            o.stats_lo = ci.start;
+            o.stats_hi = ci.start + ci.size;
             S_TRY(h, paper::launch_k1_tb2(a, o, h->p.mass == 1.0, d.s_comp));
             h->launches++;
             remaining -= two ? 2 : 1;
+            done += two ? 2 : 1;
             std::swap(xin, xout);
             std::swap(vin, vout);
         }
         S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
         S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
         if (chained)
-            for (int64_t nb = c_lo; nb <= c_hi; nb++)
+            for (int64_t nb = w_lo; nb <= w_hi; nb++)
                 if (nb != c) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)nb].h2d[prev], 0));
         // after the last launch the state is in (xin, vin)
         for (int q = 0; q < 3; q++) {
@@ -483,33 +501,33 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
 }
 
 // Blocked run: trips of s steps (the last one shorter if s does not divide
-// nsteps), alternating (X, V) -> (XN, VN) -> (X, V) ...; stats[k] (if non-NULL)
-// receives the statistics after trip k. One host barrier at the end.
+// nsteps), alternating (X, V) -> (XN, VN) -> (X, V) ...; stats[t] (if non-NULL)
+// receives the statistics after step t. One host barrier at the end.
 spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
                                  double* const VN[3], int64_t nsteps, int64_t s, somier_stats_t* stats) {
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     const int64_t ntrips = (nsteps + s - 1) / s;
-    spread_status st = ensure_acc(h, ntrips);
+    spread_status st = ensure_acc(h, nsteps);
     if (st != SPREAD_OK) return st;
     st = ensure_deep(h, h->max_chunk + 2 * s + 2);
     if (st != SPREAD_OK) return st;
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         S_TRY(h, cudaSetDevice(d.device));
-        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * (size_t)ntrips * sizeof(paper::StatsAccum), d.s_comp));
+        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, (1 + (size_t)nsteps) * sizeof(paper::StatsAccum), d.s_comp));
     }
-    std::vector<int64_t> steps((size_t)ntrips);
     for (int64_t k = 0; k < ntrips; k++) {
         const int64_t sk = std::min<int64_t>(s, nsteps - k * s);
-        steps[(size_t)k] = h->step + k * s + sk;
-        st = (k & 1) ? enqueue_stream_blocked(h, XN, VN, X, V, k, sk, k > 0)
-                     : enqueue_stream_blocked(h, X, V, XN, VN, k, sk, k > 0);
+        st = (k & 1) ? enqueue_stream_blocked(h, XN, VN, X, V, k, sk, k * s, s, k > 0)
+                     : enqueue_stream_blocked(h, X, V, XN, VN, k, sk, k * s, s, k > 0);
         if (st != SPREAD_OK) return st;
     }
     st = sync_devs(h);
     if (st != SPREAD_OK) return st;
+    std::vector<int64_t> steps((size_t)nsteps);
+    for (int64_t t = 0; t < nsteps; t++) steps[(size_t)t] = h->step + t + 1;
     h->step += nsteps;
-    return stats ? gather_stats(h, ntrips, steps.data(), stats) : SPREAD_OK;
+    return stats ? gather_stats(h, nsteps, steps.data(), stats) : SPREAD_OK;
 }
 
 // Run nsteps steps from (X, V), alternating X -> XN -> X ...; stats[t] (if
@@ -524,7 +542,7 @@ spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[
     for (auto& d : h->devs) {
         if (d.chunks.empty()) continue;
         S_TRY(h, cudaSetDevice(d.device));
-        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, 2 * (size_t)nsteps * sizeof(paper::StatsAccum), d.s_comp));
+        S_TRY(h, cudaMemsetAsync(d.acc_base, 0, (1 + (size_t)nsteps) * sizeof(paper::StatsAccum), d.s_comp));
     }
     for (int64_t t = 0; t < nsteps; t++) {
         st = (t & 1) ? enqueue_stream_step(h, XN, V, X, t, t > 0) : enqueue_stream_step(h, X, V, XN, t, t > 0);
@@ -592,7 +610,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         for (cudaStream_t* ps : {&d.s_h2d, &d.s_comp, &d.s_d2h})
             if ((e = cudaStreamCreateWithFlags(ps, cudaStreamNonBlocking)) != cudaSuccess)
                 return fail(sfail(h, e, "cudaStreamCreate"));
-        if ((e = cudaMalloc(&d.acc_base, 2 * kAccSteps * sizeof(paper::StatsAccum))) != cudaSuccess)
+        if ((e = cudaMalloc(&d.acc_base, (1 + kAccSteps) * sizeof(paper::StatsAccum))) != cudaSuccess)
             return fail(sfail(h, e, "cudaMalloc(stats)"));
         d.acc_steps = kAccSteps;
         d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
@@ -619,6 +637,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
 spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
                                      double* vz) {
     if (!h || !x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_generate: NULL argument");
+    if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     {
         const spread_status st = ensure_flat(h);
         if (st != SPREAD_OK) return st;

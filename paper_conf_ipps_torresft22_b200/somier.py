@@ -71,14 +71,18 @@ class Stats:
         return s
 
 
-def _dptr(a) -> ctypes.POINTER(ctypes.c_double):
-    """numpy float64 C-contiguous array, or an integer address (e.g. a pinned torch tensor's data_ptr())."""
+def _dptr(a, count: int) -> ctypes.POINTER(ctypes.c_double):
+    """numpy float64 C-contiguous array of exactly `count` elements (the C side
+    reads or writes that many doubles), or an integer address (e.g. a pinned
+    torch tensor's data_ptr(); the caller guarantees its size)."""
     if a is None:
         return None
     if isinstance(a, int):
         return ctypes.cast(ctypes.c_void_p(a), ctypes.POINTER(ctypes.c_double))
     if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags["C_CONTIGUOUS"]):
         raise TypeError("expected a C-contiguous float64 numpy array or an address")
+    if a.size != count:
+        raise ValueError("grid has %d elements, the C ABI needs %d" % (a.size, count))
     return a.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
 
 
@@ -104,6 +108,7 @@ class Somier:
                  cuda_device: int = -1, cuda_devices: Optional[Sequence[int]] = None):
         L = N.lib()
         self.params = params
+        self._cells = int(params.n[0]) * int(params.n[1]) * int(params.n[2])  # doubles per host grid
         self.spread = spread
         self._pc = params.c()
         h = ctypes.c_void_p()
@@ -136,6 +141,9 @@ class Somier:
     def __exit__(self, *a):
         self.close()
 
+    def _grids(self, grids):
+        return [_dptr(g, self._cells) for g in grids]
+
     # -- the step ------------------------------------------------------------
     def step(self, nsteps: int = 1) -> None:
         N.check(N.lib().somier_step(self._h, int(nsteps)), "somier_step")
@@ -148,6 +156,14 @@ class Somier:
         N.check(N.lib().somier_stats(self._h, ctypes.byref(out)), "somier_stats")
         return Stats.from_c(out)
 
+    def stats_history(self, first_step: int, count: int) -> list:
+        """Stats after steps first_step .. first_step+count-1 (somier_stats_history):
+        every step's centres / vmax, from the device-side history ring."""
+        count = int(count)
+        out = (N.somier_stats_t * max(1, count))()
+        N.check(N.lib().somier_stats_history(self._h, int(first_step), count, out), "somier_stats_history")
+        return [Stats.from_c(out[i]) for i in range(count)]
+
     # -- data movement -------------------------------------------------------
     def read(self, X=None, V=None):
         """Copy the owned planes into host grids; returns (X, V), each (3, n0, n1, n2)."""
@@ -156,7 +172,7 @@ class Somier:
             X = np.zeros(shape, np.float64)
         if V is None:
             V = np.zeros(shape, np.float64)
-        ptrs = [_dptr(X[c]) for c in range(3)] + [_dptr(V[c]) for c in range(3)]
+        ptrs = [_dptr(X[c], self._cells) for c in range(3)] + [_dptr(V[c], self._cells) for c in range(3)]
         N.check(N.lib().somier_read(self._h, *ptrs), "somier_read")
         return X, V
 
@@ -165,21 +181,22 @@ class Somier:
         shape = (3, int(count), int(self.params.n[1]), int(self.params.n[2]))
         X = np.zeros(shape, np.float64) if X is None else X
         V = np.zeros(shape, np.float64) if V is None else V
-        ptrs = [_dptr(X[c]) for c in range(3)] + [_dptr(V[c]) for c in range(3)]
+        m = int(count) * int(self.params.n[1]) * int(self.params.n[2])
+        ptrs = [_dptr(X[c], m) for c in range(3)] + [_dptr(V[c], m) for c in range(3)]
         N.check(N.lib().somier_read_planes(self._h, int(i0), int(count), *ptrs), "somier_read_planes")
         return X, V
 
     def read_ptrs(self, ptrs: Sequence[int]) -> None:
-        N.check(N.lib().somier_read(self._h, *[_dptr(p) for p in ptrs]), "somier_read")
+        N.check(N.lib().somier_read(self._h, *self._grids(ptrs)), "somier_read")
 
     def load(self, X, V) -> None:
-        ptrs = [_dptr(np.ascontiguousarray(X[c])) for c in range(3)] + [_dptr(np.ascontiguousarray(V[c]))
-                                                                      for c in range(3)]
+        ptrs = ([_dptr(np.ascontiguousarray(X[c]), self._cells) for c in range(3)]
+                + [_dptr(np.ascontiguousarray(V[c]), self._cells) for c in range(3)])
         self._keep = (X, V)
         N.check(N.lib().somier_load(self._h, *ptrs), "somier_load")
 
     def load_ptrs(self, ptrs: Sequence[int]) -> None:
-        N.check(N.lib().somier_load(self._h, *[_dptr(p) for p in ptrs]), "somier_load")
+        N.check(N.lib().somier_load(self._h, *self._grids(ptrs)), "somier_load")
 
     # -- multi-process -------------------------------------------------------
     def ipc_export(self) -> bytes:
@@ -242,6 +259,7 @@ class SomierStream:
     def __init__(self, spread: Spread, params: SomierParams, buffers: int = 2,
                  cuda_devices: Optional[Sequence[int]] = None):
         self.params = params
+        self._cells = int(params.n[0]) * int(params.n[1]) * int(params.n[2])  # doubles per host grid
         self.spread = spread
         self._pc = params.c()
         h = ctypes.c_void_p()
@@ -267,6 +285,9 @@ class SomierStream:
     def __exit__(self, *a):
         self.close()
 
+    def _grids(self, grids):
+        return [_dptr(g, self._cells) for g in grids]
+
     def generate(self, X=None, V=None):
         """Initial state (bit-identical to Somier's) into host grids; returns (X, V)."""
         shape = (3,) + tuple(int(v) for v in self.params.n)
@@ -276,7 +297,7 @@ class SomierStream:
         return X, V
 
     def generate_ptrs(self, grids) -> None:
-        N.check(N.lib().somier_stream_generate(self._h, *[_dptr(g) for g in grids]), "somier_stream_generate")
+        N.check(N.lib().somier_stream_generate(self._h, *self._grids(grids)), "somier_stream_generate")
 
     def step(self, X, V, XN) -> Stats:
         """One step: X (3 grids, read), V (3 grids, updated in place), XN (3 grids, written)."""
@@ -284,8 +305,8 @@ class SomierStream:
 
     def step_ptrs(self, X, V, XN) -> Stats:
         out = N.somier_stats_t()
-        N.check(N.lib().somier_stream_step(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
-                                           *[_dptr(g) for g in XN], ctypes.byref(out)), "somier_stream_step")
+        N.check(N.lib().somier_stream_step(self._h, *self._grids(X), *self._grids(V),
+                                           *self._grids(XN), ctypes.byref(out)), "somier_stream_step")
         return Stats.from_c(out)
 
     def run(self, X, V, XN, nsteps: int, stats: bool = True):
@@ -296,8 +317,8 @@ class SomierStream:
 
     def run_ptrs(self, X, V, XN, nsteps: int, stats: bool = True):
         out = (N.somier_stats_t * max(1, int(nsteps)))() if stats else None
-        N.check(N.lib().somier_stream_run(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
-                                          *[_dptr(g) for g in XN], int(nsteps), out), "somier_stream_run")
+        N.check(N.lib().somier_stream_run(self._h, *self._grids(X), *self._grids(V),
+                                          *self._grids(XN), int(nsteps), out), "somier_stream_run")
         return [Stats.from_c(out[t]) for t in range(int(nsteps))] if stats else None
 
     def traffic(self):
@@ -310,17 +331,16 @@ class SomierStream:
         """nsteps steps, two per host round trip (somier_stream_run2): (X, V) and
         (XN, VN) are used alternately per launch; the final state is in (X, V)
         if the number of launches ceil(nsteps / 2) is even, else in (XN, VN).
-        Returns the Stats after each launch (or None)."""
+        Returns the Stats after each step (or None)."""
         return self.run2_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]],
                               [VN[0], VN[1], VN[2]], nsteps, stats)
 
     def run2_ptrs(self, X, V, XN, VN, nsteps: int, stats: bool = True):
-        nl = int(nsteps) // 2 + int(nsteps) % 2
-        out = (N.somier_stats_t * max(1, nl))() if stats else None
-        N.check(N.lib().somier_stream_run2(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
-                                           *[_dptr(g) for g in XN], *[_dptr(g) for g in VN], int(nsteps), out),
+        out = (N.somier_stats_t * max(1, int(nsteps)))() if stats else None
+        N.check(N.lib().somier_stream_run2(self._h, *self._grids(X), *self._grids(V),
+                                           *self._grids(XN), *self._grids(VN), int(nsteps), out),
                 "somier_stream_run2")
-        return [Stats.from_c(out[k]) for k in range(nl)] if stats else None
+        return [Stats.from_c(out[t]) for t in range(int(nsteps))] if stats else None
 
     def traffic2(self):
         """Host<->device bytes of one two-step launch of run2."""
@@ -331,18 +351,17 @@ class SomierStream:
     def run_blocked(self, X, V, XN, VN, nsteps: int, steps_per_trip: int, stats: bool = True):
         """nsteps steps, `steps_per_trip` per host round trip
         (somier_stream_run_blocked); buffers alternate per trip as in run2.
-        Returns the Stats after each trip (or None)."""
+        Returns the Stats after each step (or None)."""
         return self.run_blocked_ptrs([X[0], X[1], X[2]], [V[0], V[1], V[2]], [XN[0], XN[1], XN[2]],
                                      [VN[0], VN[1], VN[2]], nsteps, steps_per_trip, stats)
 
     def run_blocked_ptrs(self, X, V, XN, VN, nsteps: int, steps_per_trip: int, stats: bool = True):
         s = int(steps_per_trip)
-        nt = -(-int(nsteps) // max(1, s))
-        out = (N.somier_stats_t * max(1, nt))() if stats else None
-        N.check(N.lib().somier_stream_run_blocked(self._h, *[_dptr(g) for g in X], *[_dptr(g) for g in V],
-                                                  *[_dptr(g) for g in XN], *[_dptr(g) for g in VN], int(nsteps), s,
+        out = (N.somier_stats_t * max(1, int(nsteps)))() if stats else None
+        N.check(N.lib().somier_stream_run_blocked(self._h, *self._grids(X), *self._grids(V),
+                                                  *self._grids(XN), *self._grids(VN), int(nsteps), s,
                                                   out), "somier_stream_run_blocked")
-        return [Stats.from_c(out[k]) for k in range(nt)] if stats else None
+        return [Stats.from_c(out[t]) for t in range(int(nsteps))] if stats else None
 
     def traffic_blocked(self, steps_per_trip: int):
         """Host<->device bytes of one trip of run_blocked with steps_per_trip steps."""

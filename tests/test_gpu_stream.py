@@ -165,7 +165,8 @@ def test_stream_run2_two_steps_per_round_trip(devices, spread_kw, buffers, nstep
     with X halo 2 and V halo 1 from the host copies, V double-buffered), odd
     step counts end with a one-step launch; chunks of one plane whose halos
     reach two chunks away; the stats after every launch and the final state
-    equal the oracle's bit for bit, NaN-filled output buffers leave no trace."""
+    equal the oracle's bit for bit, NaN-filled output buffers leave no trace.
+    Stats of every step, both steps of a two-step launch included."""
     n = (16, 13, 37)
     sp = P.SomierParams(n=n, seed=6)
     if "sizes" in spread_kw:
@@ -184,14 +185,11 @@ def test_stream_run2_two_steps_per_round_trip(devices, spread_kw, buffers, nstep
     nl = nsteps // 2 + nsteps % 2
     fX, fV = (X, V) if nl % 2 == 0 else (XN, VN)
     ref = O.init(_op(sp))
-    done = 0
-    for k in range(nl):
-        for _ in range(2 if k < nsteps // 2 else 1):
-            ref, rst = O.step(ref)
-            done += 1
-        assert stats[k].step == done
-        assert stats[k].sums == rst.sums and stats[k].vmax2_bits == rst.vmax2_bits and stats[k].centre == rst.centre
-    assert done == nsteps
+    assert len(stats) == nsteps
+    for t in range(nsteps):
+        ref, rst = O.step(ref)
+        assert stats[t].step == t + 1
+        assert stats[t].sums == rst.sums and stats[t].vmax2_bits == rst.vmax2_bits and stats[t].centre == rst.centre
     assert np.array_equal(fX, ref.X) and np.array_equal(fV, ref.V)
     plane = 3 * n[1] * n[2] * 8
     assert tr["d2h_bytes"] == 2 * plane * (n[0] - 2) + 4 * plane
@@ -228,8 +226,9 @@ def test_stream_run_blocked_s_steps_per_round_trip(devices, spread_kw, buffers, 
     """somier_stream_run_blocked: s steps per host round trip (halo s, regions
     shrinking two planes per side per K1_TB2 launch, odd s ending with a
     one-step launch, halos reaching several one-plane chunks away, s larger
-    than the grid's chunks); every trip's stats and the final state equal the
-    oracle's bit for bit."""
+    than the grid's chunks); every step's stats and the final state equal the
+    oracle's bit for bit -- the stats of every step, the intermediate steps of a
+    trip (widened launches) included."""
     n = (16, 13, 37)
     sp = P.SomierParams(n=n, seed=6)
     if "sizes" in spread_kw:
@@ -247,13 +246,11 @@ def test_stream_run_blocked_s_steps_per_round_trip(devices, spread_kw, buffers, 
     nt = -(-nsteps // spt)
     fX, fV = (X, V) if nt % 2 == 0 else (XN, VN)
     ref = O.init(_op(sp))
-    done = 0
-    for k in range(nt):
-        for _ in range(min(spt, nsteps - done)):
-            ref, rst = O.step(ref)
-            done += 1
-        assert stats[k].step == done
-        assert stats[k].sums == rst.sums and stats[k].vmax2_bits == rst.vmax2_bits
+    assert len(stats) == nsteps
+    for t in range(nsteps):
+        ref, rst = O.step(ref)
+        assert stats[t].step == t + 1
+        assert stats[t].sums == rst.sums and stats[t].vmax2_bits == rst.vmax2_bits
     assert np.array_equal(fX, ref.X) and np.array_equal(fV, ref.V)
 
 

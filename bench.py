@@ -78,14 +78,11 @@ def interior_of(n, size):
 # fp64 lane-instructions per node-update of node_math.cuh with each spring
 # evaluated once: 3 springs x 27 (3 sub, d^2 5, sqrt + 1/d 11,
 # d-L and K* 2, quotient 3, f*d 3) + force sum 15 + kick/drift 12 = 108, and the
-# fused stats 27 (3 x 7 exact-split centre terms, v.v 5, max 1) per step whose
-# stats are kept. K1_TB2 keeps only the second step's stats.
-FP64_OPS_STEP, FP64_OPS_STATS = 108, 27
+# fused stats of every step 16 (3 x 4 exact-split centre terms, v.v 3, max 1).
+FP64_OPS_STEP, FP64_OPS_STATS = 108, 16
 
 
-def fp64_ops_per_node_update(two_step):
-    if two_step:
-        return FP64_OPS_STEP + FP64_OPS_STATS / 2.0
+def fp64_ops_per_node_update(two_step=False):
     return FP64_OPS_STEP + FP64_OPS_STATS
 
 

@@ -67,6 +67,23 @@ constexpr int kYComp = kRows * kTK;                         // X_{t+1} of one R1
 #define TB2_VSTAGES 2
 #endif
 constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
+// where step t+1's stats are accumulated: 2 in S1 right after its kick-drift
+// (default, measured fastest: 6.38e10 node-updates/s at 512^3 vs 6.23 / 6.33
+// for 0 = after S2 / 1 = before S2's forces), 9 not at all (A/B of their cost
+// only: stats of every second step, 7.2e10)
+#ifndef TB2_ST1_MODE
+#define TB2_ST1_MODE 2
+#endif
+// the last step's stats accumulators in shared memory too (else registers;
+// 5.84-5.94e10: the LSU round trips cost more than the freed registers)
+#ifndef TB2_ST_SMEM
+#define TB2_ST_SMEM 0
+#endif
+// S2's results and stats without per-node branches around the stats (both
+// nodes' results live at once: spills, 5.07e10 -- not the default)
+#ifndef TB2_S2_BF
+#define TB2_S2_BF 0
+#endif
 constexpr int kMinSegPlanes = 4, kMaxSegPlanes = 256;
 static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
 
@@ -81,6 +98,12 @@ struct __align__(16) Smem {
     unsigned long long full[kStages];
     unsigned long long vfull[kVStages];
     WarpStats scratch[kW];
+    // step t+1's stats accumulators, thread-private (registers are full):
+    // [0..2] = (sum bits(hd), sum bits(ld)) of x, y, z; [3] = (max v.v, unused)
+    ulonglong2 acc1[4][kThreads];
+#if TB2_ST_SMEM
+    ulonglong2 acc2[4][kThreads];  // the last step's, same layout (TB2_ST_SMEM variant)
+#endif
 };
 
 struct Tb2Params {
@@ -110,6 +133,7 @@ __device__ __forceinline__ void stb3(double* p, int64_t cs, const Vec3& v) {
 __device__ __forceinline__ Vec3 ldb(const double* b, int off, int comp) {
     return Vec3{b[off], b[off + comp], b[off + 2 * comp]};
 }
+
 
 // kTwo: two steps per launch (else one: S1 only, its X_{t+1}, V_{t+1} written
 // for R2 -- the odd step of a TB2 handle, with the same halo layout).
@@ -209,9 +233,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     Vec3 carry2A{0.0, 0.0, 0.0}, carry2B{0.0, 0.0, 0.0};
     Vec3 v1pA{0.0, 0.0, 0.0}, v1pB{0.0, 0.0, 0.0};  // V_{t+1} of plane p-1
-    NodeStats st, st1;  // stats of the launch's last step (t+2, or t+1 in one-step mode) and of step t+1
+    NodeStats st;  // stats of the launch's last step (t+2, or t+1 in one-step mode); step t+1's: sm.acc1
     st.zero();
-    st1.zero();
+#pragma unroll
+    for (int c = 0; c < 4; c++) sm.acc1[c][tid] = make_ulonglong2(0ull, 0ull);
     const int border_last = min(pe, ilast);  // planes whose border springs S1 needs
     // X_{t+2} (X_{t+1}), V of an S2 output node: own slab, and the neighbours'
     // halo planes (2 planes of X, 1 of V per face: what their next launch reads)
@@ -227,6 +252,69 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (q == start + size - 1) stb3(tp.hi_vdst + off, cs, v2);
         }
     };
+
+    // Step t+1's stats of the owned nodes of an output plane q: X_{t+1} from
+    // the ring, V_{t+1} from the register carry; read-modify-write of the
+    // thread's shared-memory accumulators, coordinate by coordinate. Branch-free
+    // (the addends of a node the thread does not own are selected to 0; a fixed
+    // node's V_{t+1} is 0): divergent code here makes ptxas wrap the march's
+    // warp shuffles in collective fix-up sequences.
+    auto acc1_update = [&](const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb) {
+        const double xsa[3] = {xa.x, xa.y, xa.z}, xsb[3] = {xb.x, xb.y, xb.z};
+#pragma unroll
+        for (int c = 0; c < 3; c++) {
+            const double hda = __fma_rn(xsa[c], 0x1p28, kRoundC), hdb = __fma_rn(xsb[c], 0x1p28, kRoundC);
+#ifdef STATS_ONEWORD_TIMING
+            const double lda = kRoundC, ldb_ = kRoundC;
+#else
+            const double ra = __fma_rn(xsa[c], 0x1p28, -__dsub_rn(hda, kRoundC));
+            const double rb = __fma_rn(xsb[c], 0x1p28, -__dsub_rn(hdb, kRoundC));
+            const double lda = __fma_rn(ra, 0x1p32, kRoundC), ldb_ = __fma_rn(rb, 0x1p32, kRoundC);
+#endif
+            const unsigned long long ha = ownA ? (unsigned long long)__double_as_longlong(hda) : 0ull;
+            const unsigned long long hb = ownB ? (unsigned long long)__double_as_longlong(hdb) : 0ull;
+            const unsigned long long la = ownA ? (unsigned long long)__double_as_longlong(lda) : 0ull;
+            const unsigned long long lb = ownB ? (unsigned long long)__double_as_longlong(ldb_) : 0ull;
+            ulonglong2 o = sm.acc1[c][tid];
+            o.x += ha + hb;
+            o.y += la + lb;
+            sm.acc1[c][tid] = o;
+        }
+        const double v2a = ownA ? dot_self(va) : 0.0, v2b = ownB ? dot_self(vb) : 0.0;
+        double vm = __longlong_as_double((long long)sm.acc1[3][tid].x);
+        vm = (v2a > vm || v2a != v2a) ? v2a : vm;
+        vm = (v2b > vm || v2b != v2b) ? v2b : vm;
+        sm.acc1[3][tid].x = (unsigned long long)__double_as_longlong(vm);
+    };
+
+    // the last step's stats of one node (hasv: an interior node, v enters vmax)
+#if TB2_ST_SMEM
+    unsigned int nst = 0;
+    for (int c = 0; c < 4; c++) sm.acc2[c][tid] = make_ulonglong2(0ull, 0ull);
+    auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
+        const double xs[3] = {x.x, x.y, x.z};
+#pragma unroll
+        for (int c = 0; c < 3; c++) {
+            const double hd = __fma_rn(xs[c], 0x1p28, kRoundC);
+            const double r = __fma_rn(xs[c], 0x1p28, -__dsub_rn(hd, kRoundC));
+            ulonglong2 o = sm.acc2[c][tid];
+            o.x += (unsigned long long)__double_as_longlong(hd);
+            o.y += (unsigned long long)__double_as_longlong(__fma_rn(r, 0x1p32, kRoundC));
+            sm.acc2[c][tid] = o;
+        }
+        nst++;
+        if (hasv) {
+            const double v2 = dot_self(v);
+            const double vm = __longlong_as_double((long long)sm.acc2[3][tid].x);
+            if (v2 > vm || v2 != v2) sm.acc2[3][tid].x = (unsigned long long)__double_as_longlong(v2);
+        }
+    };
+#else
+    auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
+        st.add_position(x);
+        if (hasv) st.add_velocity(v);
+    };
+#endif
 
     // One plane of the march. kFull: a steady-state plane (p+1 exists, p is
     // updated by S1, q = p-1 is an S2 output plane): no conditions, no
@@ -284,6 +372,10 @@ __global__ void __launch_bounds__(kThreads, 1)
                 kick_drift<kUnitMass>(F, a.M, a.dt, v1B, xcB, x1B);
             }
         }
+#if TB2_ST1_MODE == 2
+        // step t+1's stats right where S1 produced them (plane p, if an output plane of this segment)
+        if (kTwo && p >= max(pb, tp.stats_lo) && p < min(pe, tp.stats_hi)) acc1_update(x1A, x1B, v1A, v1B);
+#endif
         {
             double* y = sm.y[par][0];
             y[yA] = x1A.x;
@@ -323,6 +415,29 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q (one-step mode: X_{t+1}, V_{t+1} of S1)
         const bool sq = kFull ? (q >= tp.stats_lo && q < tp.stats_hi) : (out2 && q >= tp.stats_lo && q < tp.stats_hi);
+#if TB2_ST1_MODE == 1
+        if (kTwo && sq) acc1_update(xqA, xqB, v1pA, v1pB);
+#endif
+#if TB2_S2_BF
+        if (out2) {
+            // results of the two nodes (a fixed node keeps X, and V = 0)
+            Vec3 x2A = xqA, v2A = v1pA, x2B = xqB, v2B = v1pB;
+            if (kTwo) {
+                if (ownA && intA) {
+                    const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
+                    const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
+                    kick_drift<kUnitMass>(F, a.M, a.dt, v2A, xqA, x2A);
+                }
+                if (ownB && intB) {
+                    const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
+                    kick_drift<kUnitMass>(F, a.M, a.dt, v2B, xqB, x2B);
+                }
+            }
+            if (ownA && intA) store_out(q, offA, x2A, v2A);
+            if (ownB && intB) store_out(q, offB, x2B, v2B);
+            if (sq) st.add_pair(x2A, x2B, v2A, v2B, ownA, ownB);
+        }
+#else
         if (out2) {
             if (ownA) {
                 if (intA) {
@@ -331,19 +446,11 @@ __global__ void __launch_bounds__(kThreads, 1)
                         const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
-                        if (sq) {
-                            st1.add_position_nc(xqA);  // step t+1: X_{t+1}, V_{t+1} of this node
-                            st1.add_velocity(v1pA);
-                        }
                     }
                     store_out(q, offA, x2, v2);
-                    if (sq) {
-                        st.add_position(x2);
-                        st.add_velocity(v2);
-                    }
+                    if (sq) st_add(x2, v2, true);
                 } else if (sq) {
-                    st.add_position(xqA);  // fixed face node
-                    if (kTwo) st1.add_position_nc(xqA);
+                    st_add(xqA, xqA, false);  // fixed face node
                 }
             }
             if (ownB) {
@@ -352,22 +459,18 @@ __global__ void __launch_bounds__(kThreads, 1)
                     if (kTwo) {
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
-                        if (sq) {
-                            st1.add_position_nc(xqB);
-                            st1.add_velocity(v1pB);
-                        }
                     }
                     store_out(q, offB, x2, v2);
-                    if (sq) {
-                        st.add_position(x2);
-                        st.add_velocity(v2);
-                    }
+                    if (sq) st_add(x2, v2, true);
                 } else if (sq) {
-                    st.add_position(xqB);
-                    if (kTwo) st1.add_position_nc(xqB);
+                    st_add(xqB, xqB, false);
                 }
             }
         }
+#endif
+#if TB2_ST1_MODE == 0
+        if (kTwo && sq) acc1_update(xqA, xqB, v1pA, v1pB);
+#endif
         // border springs of the next plane (X_t(p+1) is resident until barrier #1 of iteration p+1)
         if (p + 1 <= border_last) border_springs(p + 1);
         carry1A = gpi1A;
@@ -395,11 +498,29 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     if (p <= hi) body(F1{}, P0{}, p++);
     for (; p <= pe; p++) body(F0{}, PN{}, p);
+#if TB2_ST_SMEM
+    for (int c = 0; c < 3; c++) {
+        st.hb[c] = sm.acc2[c][tid].x;
+        st.lb[c] = sm.acc2[c][tid].y;
+    }
+    st.vmax2 = __longlong_as_double((long long)sm.acc2[3][tid].x);
+    st.n = nst;
+#endif
     block_accumulate(st, sm.scratch, slots.fin);
-    if (kTwo) {
+    if (kTwo && TB2_ST1_MODE != 9) {
+#ifndef STATS_FP64_ACC
+        NodeStats st1;
+        for (int c = 0; c < 3; c++) {
+            st1.hb[c] = sm.acc1[c][tid].x;
+            st1.lb[c] = sm.acc1[c][tid].y;
+        }
+        st1.vmax2 = __longlong_as_double((long long)sm.acc1[3][tid].x);
         st1.copy_count(st);
         __syncthreads();  // scratch reuse
         block_accumulate(st1, sm.scratch, slots.mid);
+#else
+#error "K1_TB2 keeps step t+1's stats as bit-pattern sums (no STATS_FP64_ACC variant)"
+#endif
     }
     finish_launch(a, slots.t, kTwo ? 2 : 1);
 }

@@ -47,8 +47,16 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu-all-cores", action="store_true", help="skip the all-cores (-fopenmp) oracle line")
+    ap.add_argument("--oracle-child", default=None, help=argparse.SUPPRESS)
     ap.add_argument("--share-gpu", action="store_true",
                     help="testing only: all ranks on cuda:0 with gloo plumbing (exercises the N>1 path on 1 GPU)")
+    ap.add_argument("--verify", action="store_true",
+                    help="after the measurements: a fresh run of a few steps, nodes on both sides of every chunk "
+                         "border (and the grid's first / last planes) checked bit for bit against the CPU oracle "
+                         "through their light cone")
+    ap.add_argument("--sustained-s", type=float, default=1.2,
+                    help="seconds of the sustained pass after the timed region (0: skip)")
     ap.add_argument("--copy-check", action="store_true",
                     help="also time a sustained torch copy of the same byte volume (context for the roofline)")
     a = ap.parse_args()
@@ -78,8 +86,8 @@ def interior_of(n, size):
 # fp64 lane-instructions per node-update of node_math.cuh with each spring
 # evaluated once: 3 springs x 27 (3 sub, d^2 5, sqrt + 1/d 11,
 # d-L and K* 2, quotient 3, f*d 3) + force sum 15 + kick/drift 12 = 108, and the
-# fused stats of every step 16 (3 x 4 exact-split centre terms, v.v 3, max 1).
-FP64_OPS_STEP, FP64_OPS_STATS = 108, 16
+# fused stats of every step 18 (3 x 4 exact-split centre terms, v.v 5, max 1).
+FP64_OPS_STEP, FP64_OPS_STATS = 108, 18
 
 
 def fp64_ops_per_node_update(two_step=False):
@@ -108,17 +116,39 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+KERNEL_SRC = {"tb2": "k1_tb2.cu", "march2": "k1_march2.cu", "march": "k1_march.cu", "direct": "k1_direct.cu"}
+
+
+def kernel_source_sha(kernel):
+    """sha1 of the kernel's source files (its .cu + the shared headers): ties a
+    committed ncu capture to the code it measured."""
+    import hashlib
+
+    kdir = os.path.join(ROOT, "paper_conf_ipps_torresft22_b200", "csrc", "kernels")
+    h = hashlib.sha1()
+    for name in [KERNEL_SRC.get(kernel, ""), "node_math.cuh", "stats.cuh", "signal.cuh", "tma.cuh"]:
+        path = os.path.join(kdir, name)
+        if os.path.exists(path):
+            with open(path, "rb") as f:
+                h.update(f.read())
+    return h.hexdigest()
+
+
 def load_traffic(n, kernel):
-    """DRAM bytes per K1 launch from the committed ncu --set full capture, if it
-    was taken on this workload (profiles/k1_traffic.json)."""
+    """DRAM bytes per K1 launch (dram__bytes_read.sum + dram__bytes_write.sum)
+    from the committed ncu --set full capture of this workload
+    (profiles/k1_traffic.json); None unless the capture was taken on the
+    kernel source as it is now (source_sha)."""
     path = os.path.join(ROOT, "profiles", "k1_traffic.json")
     try:
         with open(path) as f:
             d = json.load(f)
         e = d.get("%dx%dx%d/%s" % (n[0], n[1], n[2], kernel))
-        return None if e is None else float(e["dram_bytes_per_launch"])
+        if e is None or e.get("source_sha") != kernel_source_sha(kernel):
+            return None, None
+        return float(e["dram_bytes_per_launch"]), e.get("source")
     except Exception:
-        return None
+        return None, None
 
 
 class ClockSampler:
@@ -187,32 +217,87 @@ class ClockSampler:
 
 # --------------------------------------------------------------------------- oracle arm
 
-def oracle_sample(n, budget_s, max_steps=None, warmup=0, planes=8):
-    """Time the CPU oracle (as it stands) on a bounded sample of the workload: a
-    (planes+2) x n1 x n2 slab -- `planes` interior planes of the full cross
-    section -- stepped repeatedly. Returns (node-updates/s, sample description, steps)."""
+def host_cpu():
+    """CPU model, logical CPUs of the host, and the CPUs this process may use."""
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    allowed = sorted(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else list(range(os.cpu_count() or 1))
+    return model, os.cpu_count() or len(allowed), allowed
+
+
+def oracle_child(spec):
+    """Child process of the CPU baseline (bench.py --oracle-child JSON): the C
+    oracle as it stands (oracle_run_timed: the step loop timed with the steady
+    clock inside C, no per-step Python copies) on a (planes+2) x n1 x n2 slab of
+    the workload's cross-section -- one calibration step, then enough steps for
+    ~budget seconds. Prints one JSON object."""
     import oracle as O
 
-    p = O.Params(n=(planes + 2, n[1], n[2]), seed=42)
-    s = O.init(p)
-    per_step = planes * (n[1] - 2) * (n[2] - 2)
-    for _ in range(warmup):
-        s, _ = O.step(s)
-    t0 = time.perf_counter()
-    steps = 0
-    while True:
-        s, _ = O.step(s)
-        steps += 1
-        el = time.perf_counter() - t0
-        if max_steps is not None and steps >= max_steps:
-            break
-        if max_steps is None and el >= budget_s:
-            break
-    rate = per_step * steps / el
-    desc = ("CPU oracle (oracle/somier_oracle.c, sequential fp64, gcc -O2) on a %d-plane slab of the %dx%dx%d "
-            "cross-section (+2 halo planes), %d steps = %.3g node-updates in %.1f s"
-            % (planes, n[0], n[1], n[2], steps, per_step * steps, el))
-    return rate, desc, steps, el
+    d = json.loads(spec)
+    n1, n2, planes, omp = d["n1"], d["n2"], d["planes"], d["omp"]
+    s = O.init(O.Params(n=(planes + 2, n1, n2), seed=42))
+    if d.get("steps"):
+        if d.get("warmup"):
+            s, _, _, _ = O.run_timed(s, d["warmup"], omp=omp)
+        steps = int(d["steps"])
+    else:
+        s, _, t1, _ = O.run_timed(s, 1, omp=omp)
+        steps = max(1, int(d["budget"] / max(t1, 1e-6)))
+    s, st, sec, threads = O.run_timed(s, steps, omp=omp)
+    print(json.dumps({"steps": steps, "seconds": sec, "threads": threads,
+                      "node_updates": planes * (n1 - 2) * (n2 - 2) * steps, "vmax": st.vmax}), flush=True)
+
+
+def oracle_sample(n, budget_s=12.0, omp=False, planes=None, steps=None, warmup=0):
+    """Time the CPU oracle on a bounded sample of the workload in a child
+    process pinned to ONE core (sequential build), or to every core this
+    process may use (the all-cores -fopenmp build, OMP_NUM_THREADS = that
+    count). Returns the cpu_baseline object."""
+    model, ncpu, allowed = host_cpu()
+    cpus = allowed if omp else allowed[:1]
+    if planes is None:
+        planes = max(8, 4 * len(cpus)) if omp else 8  # the all-cores build splits the i loop
+    planes = min(planes, n[0] - 2)
+    spec = json.dumps({"n1": n[1], "n2": n[2], "planes": planes, "omp": omp, "budget": budget_s,
+                       "steps": steps, "warmup": warmup})
+    env = dict(os.environ)
+    env["OMP_NUM_THREADS"] = str(len(cpus))
+    env["OMP_PROC_BIND"] = "close"
+
+    def pin():
+        if hasattr(os, "sched_setaffinity"):
+            os.sched_setaffinity(0, set(cpus))
+
+    r = subprocess.run([sys.executable, os.path.abspath(__file__), "--oracle-child", spec], env=env,
+                       preexec_fn=pin, capture_output=True, text=True, timeout=600)
+    if r.returncode != 0:
+        raise RuntimeError("oracle child failed: %s" % r.stderr[-2000:])
+    d = json.loads(r.stdout.strip().splitlines()[-1])
+    rate = d["node_updates"] / d["seconds"]
+    build = ("oracle/liboracle_omp.so (the same somier_oracle.c, -fopenmp, %d threads)" % d["threads"] if omp
+             else "oracle/liboracle.so (sequential fp64, gcc -O2 -ffp-contract=off)")
+    desc = ("CPU oracle %s: oracle_run_timed (steady clock around the C step loop; every step's five kernels "
+            "incl. centers) on a %d-plane slab of the %dx%dx%d cross-section (+2 halo planes), %d steps = %.3g "
+            "node-updates in %.2f s; pinned to CPU%s %s" % (build, planes, n[0], n[1], n[2], d["steps"],
+                                                          d["node_updates"], d["seconds"],
+                                                          "s" if len(cpus) > 1 else "",
+                                                          _cpu_list(cpus)))
+    return {"value": rate, "unit": UNIT, "cores": len(cpus), "kind": "oracle", "sample": desc,
+            "cpu_model": model, "nproc": ncpu, "cores_label": "%d of %d cores" % (len(cpus), ncpu),
+            "steps": d["steps"], "seconds": d["seconds"], "threads": d["threads"]}
+
+
+def _cpu_list(cpus):
+    if len(cpus) > 1 and cpus == list(range(cpus[0], cpus[-1] + 1)):
+        return "%d-%d" % (cpus[0], cpus[-1])
+    return ",".join(str(c) for c in cpus)
 
 
 def run_reference(a):
@@ -221,18 +306,18 @@ def run_reference(a):
         return 0
     n = a.n
     # Bound the whole --steps K --warmup W run to a few minutes: one oracle
-    # node-update costs ~0.1-0.2 us on one core, so a step over P planes of the
-    # n1 x n2 cross-section costs ~2e-7 * P * n1 * n2 s; budget ~150 s total.
-    per_plane = 2e-7 * n[1] * n[2]
-    planes = int(max(1, min(8, 150.0 / (max(1, a.steps + a.warmup) * per_plane))))
-    rate, desc, steps, el = oracle_sample(n, budget_s=None, max_steps=a.steps, warmup=a.warmup, planes=planes)
+    # node-update costs ~0.1 us on one core, so a step over P planes of the
+    # n1 x n2 cross-section costs ~1e-7 * P * n1 * n2 s; budget ~120 s total.
+    per_plane = 1.2e-7 * n[1] * n[2]
+    planes = int(max(1, min(8, 120.0 / (max(1, a.steps + a.warmup) * per_plane))))
+    cpu = oracle_sample(n, omp=False, planes=planes, steps=a.steps, warmup=a.warmup)
     line = {
-        "impl": "reference", "metric": METRIC, "value": rate, "unit": UNIT, "n_gpus": a.gpus, "steps": a.steps,
-        "warmup": a.warmup, "ms_per_step": 1e3 * el / steps, "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "impl": "reference", "metric": METRIC, "value": cpu["value"], "unit": UNIT, "n_gpus": a.gpus,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * cpu["seconds"] / cpu["steps"],
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": workload_name(n), "n": list(n), "sample": "%d-plane slab per step" % planes},
-        "cpu_baseline": {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc},
-        "e2e": {"value": rate, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "cpu_baseline": cpu,
+        "e2e": {"value": cpu["value"], "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
     return 0
@@ -240,57 +325,151 @@ def run_reference(a):
 
 # --------------------------------------------------------------------------- our arm
 
-def halo_info(n, chunks, world, two_step=False):
+def roofline_obj(achieved, peak, peak_src, traffic, traffic_src, k1_ms, kname, alg, alg_step, nu_launch, per_call,
+                 step_dist, copy_gbs, fp64_frac):
+    """The dominant kernel against HBM (SURVEY.md §8(d)'s algorithmic bytes: 96 B
+    per node-update), the actual DRAM bytes of the committed ncu capture of this
+    code (if any), and which roof is closest."""
+    r = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+         "traffic": traffic, "peak_source": peak_src, "kernel": "k1_%s_kernel" % kname,
+         "algorithmic_bytes_per_node_update": alg / nu_launch, "node_updates_per_launch": nu_launch,
+         "algorithmic_bytes_per_launch": alg, "avg_launch_ms": k1_ms, "launch_ms_distribution": step_dist,
+         "sustained_copy_gbs": copy_gbs, "steps_per_launch": per_call}
+    if traffic:
+        r["dram_actual"] = {"gbs": traffic / (k1_ms * 1e-3) / 1e9, "frac": traffic / (k1_ms * 1e-3) / 1e9 / peak,
+                            "bytes_per_node_update": traffic / nu_launch, "source": traffic_src}
+    fr = {"fp64 pipe (roofline_fp64)": fp64_frac}
+    if traffic:
+        fr["HBM (actual DRAM bytes)"] = r["dram_actual"]["frac"]
+    closest = max(fr, key=fr.get)
+    if per_call == 2:
+        r["note"] = ("K1_TB2 advances two steps per pass over HBM, so it moves about half of §8(d)'s 96 B per "
+                     "node-update (one pass = %d B per launch): 'frac' > 1 against the one-step algorithmic "
+                     "bytes. The roof that binds is the fp64 issue / latency: neither the fp64 pipe nor HBM is "
+                     "saturated; closest: %s at %.2f" % (alg_step, closest, fr[closest]))
+    else:
+        r["note"] = "one step per launch; closest roof: %s at %.2f" % (closest, fr[closest])
+    r["closest_roof"] = {"name": closest, "frac": fr[closest]}
+    return r
+
+
+def halo_info(n, chunks, world, two_step, ranks):
     """Halo traffic of the fused exchange: each chunk boundary between list
     positions moves one X plane (24 B per node of the n1 x n2 cross-section)
     each way per step, stored by K1 straight into the neighbour's halo slot
     (NVLink P2P / IPC); K1_TB2 moves two X planes and one V plane each way per
-    two-step launch (36 B per cross-section node per step). Reported against
-    the measured 770 GB/s peer rate (B200_PROFILING.md); the stores overlap the
-    step, so this is a bound on the exchange's cost, not a separate phase."""
+    two-step launch (36 B per cross-section node per step). Measured per rank
+    (somier_set_timing, diagnostic pass): the time its stream sat in the
+    neighbour-flag waits (neighbours' previous launch: their halo stores and
+    their skew) and the kernel time, in which the peer stores run. Compared
+    with the time the same bytes take at the measured 770 GB/s per-direction
+    peer rate (B200_PROFILING.md; nominal NVLink 5: 900 GB/s)."""
     plane = (36 if two_step else 24) * n[1] * n[2]
     cross = sum(1 for a, b in zip(chunks, chunks[1:]) if a.device_pos != b.device_pos)
     total = 2 * cross * plane
     per_rank = total / max(1, world)
+    per_launch = per_rank * (2 if two_step else 1)
+    waits = [r["diag_wait_ms_per_launch"] for r in ranks]
+    kern = [r["diag_kernel_ms_per_launch"] for r in ranks]
     return {"bytes_per_step_total": total, "bytes_per_step_per_rank": per_rank,
-            "est_us_at_770_gbs": per_rank / 770e9 * 1e6, "mechanism": "in-kernel peer stores + completion flag"}
+            "bytes_per_launch_per_rank": per_launch,
+            "ideal_us_per_launch_at_770_gbs": per_launch / 770e9 * 1e6,
+            "measured_wait_ms_per_launch": {"min": min(waits), "max": max(waits)},
+            "measured_kernel_ms_per_launch": {"min": min(kern), "max": max(kern)},
+            "wait_frac_of_launch": max(w / max(1e-9, w + k) for w, k in zip(waits, kern)),
+            "mechanism": "in-kernel peer stores (NVLink P2P / CUDA IPC) + release-stored completion flag, "
+                         "cuStreamWaitValue64 before the next launch"}
 
 
-def pcie_rates(local, nbytes=1 << 30):
-    """Pinned host<->device copy rates (GB/s), one direction at a time and both
-    directions concurrently -- the roofline of the host-streamed mode."""
+def run_verify(a, n, params, world, rank, local, multi):
+    """A fresh run of a few steps in the benched configuration, then nodes on
+    both sides of every chunk border (and near the grid's first / last planes)
+    read back and compared bit for bit with the CPU oracle on a window reaching
+    steps+1 nodes around each (a node after S steps depends only on initial
+    values within distance S: tests/test_oracle_pins.py pins the window).
+    Proves the cross-device exchange (peer stores, flags, waits) of this exact
+    launch configuration. Each rank checks the planes it owns."""
+    import numpy as np
+
+    import oracle as O
+    import paper_conf_ipps_torresft22_b200 as P
+    from paper_conf_ipps_torresft22_b200 import dist as PD
+
+    steps = 6
+    if multi:
+        s = PD.open_local(params, chunk=a.chunk, cuda_device=local)
+    else:
+        s = P.Somier(P.Spread([local], 1, n[0] - 2, chunk=a.chunk), params)
+    mine = [c for c in s.spread.chunks() if (not multi) or c.device_pos == rank]
+    s.step(steps)
+    s.sync()
+    planes = set()
+    for c in mine:
+        for i in (c.start, c.start + 1, c.start + c.size - 2, c.start + c.size - 1):
+            if c.start <= i < c.start + c.size:
+                planes.add(i)
+    jk = [(1, 1), (n[1] // 2, n[2] // 2), (n[1] - 2, n[2] - 2), (n[1] // 3, n[2] - 2), (22, 31)]
+    jk = [(j, k) for j, k in jk if 0 < j < n[1] - 1 and 0 < k < n[2] - 1]
+    op = O.Params(n=n, seed=params.seed, spacing=params.spacing, rest_len=params.rest_len, k_spring=params.k_spring,
+                  mass=params.mass, dt=params.dt, amplitude=params.amplitude)
+    bad, checked = [], 0
+    for i in sorted(planes):
+        X, V = s.read_planes(i, 1)
+        for j, k in jk:
+            node = (i, j, k)
+            lo = [max(0, node[d] - steps - 1) for d in range(3)]
+            hi = [min(n[d], node[d] + steps + 2) for d in range(3)]
+            win, _ = O.run(O.init_window(op, lo, [hi[d] - lo[d] for d in range(3)]), steps)
+            r = tuple(node[d] - lo[d] for d in range(3))
+            ok = (np.array_equal(X[:, 0, j, k], win.X[(slice(None),) + r])
+                  and np.array_equal(V[:, 0, j, k], win.V[(slice(None),) + r]))
+            checked += 1
+            if not ok:
+                bad.append(list(node))
+    s.close()
+    res = {"rank": rank, "checked": checked, "bad": bad}
+    allr = PD.all_gather_obj(res) if multi else [res]
+    nbad = sum(len(r["bad"]) for r in allr)
+    return {"steps": steps, "nodes_checked": sum(r["checked"] for r in allr), "mismatches": nbad,
+            "bad_nodes": [b for r in allr for b in r["bad"]][:20], "ok": nbad == 0,
+            "what": "nodes on both sides of every chunk border, bitwise vs the CPU oracle (light-cone windows)"}
+
+
+def pcie_rates(devices, nbytes=1 << 30):
+    """Pinned host<->device copy rates (GB/s) of the GPUs in `devices` (distinct
+    CUDA ordinals), all at once: H2D alone, D2H alone, and both directions
+    concurrently -- the roofline of the host-streamed mode."""
     import torch
 
-    h1 = torch.empty(nbytes // 8, dtype=torch.float64, pin_memory=True)
-    h2 = torch.empty_like(h1, pin_memory=True)
-    d1 = torch.empty(nbytes // 8, dtype=torch.float64, device="cuda")
-    d2 = torch.empty_like(d1)
-    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
-    res = {}
-    for name, fn in (("h2d", lambda: d1.copy_(h1, non_blocking=True)),
-                     ("d2h", lambda: h1.copy_(d1, non_blocking=True))):
-        fn()
-        torch.cuda.synchronize()
+    devs = sorted(set(devices))
+    hs = [torch.empty(nbytes // 8, dtype=torch.float64, pin_memory=True) for _ in range(2 * len(devs))]
+    ds = [torch.empty(nbytes // 8, dtype=torch.float64, device="cuda:%d" % d) for d in devs for _ in range(2)]
+    st = [torch.cuda.Stream(device=d) for d in devs for _ in range(2)]
+
+    def run(h2d, d2h, reps=3):
+        for d in devs:
+            torch.cuda.synchronize(d)
         t0 = time.perf_counter()
-        for _ in range(3):
-            fn()
-        torch.cuda.synchronize()
-        res[name] = 3 * nbytes / (time.perf_counter() - t0) / 1e9
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    for _ in range(3):
-        with torch.cuda.stream(s1):
-            d1.copy_(h1, non_blocking=True)
-        with torch.cuda.stream(s2):
-            h2.copy_(d2, non_blocking=True)
-    torch.cuda.synchronize()
-    res["bidir_total"] = 6 * nbytes / (time.perf_counter() - t0) / 1e9
-    del h1, h2, d1, d2
+        for _ in range(reps):
+            for q in range(len(devs)):
+                if h2d:
+                    with torch.cuda.stream(st[2 * q]):
+                        ds[2 * q].copy_(hs[2 * q], non_blocking=True)
+                if d2h:
+                    with torch.cuda.stream(st[2 * q + 1]):
+                        hs[2 * q + 1].copy_(ds[2 * q + 1], non_blocking=True)
+        for d in devs:
+            torch.cuda.synchronize(d)
+        return reps * len(devs) * nbytes * (int(h2d) + int(d2h)) / (time.perf_counter() - t0) / 1e9
+
+    run(True, True, 1)
+    res = {"h2d": run(True, False), "d2h": run(False, True), "bidir_total": run(True, True), "gpus": len(devs)}
+    del hs, ds
     torch.cuda.empty_cache()
     return res
 
 
-def e2e_stream(n, params, local, a, two_step):
+def e2e_stream(n, params, devices, a, two_step, cuda_devices=None):
     """End to end through the public C ABI with HOST buffers: the state lives in
     pinned host memory and every launch maps each chunk to the GPU (X with halo
     planes, V), runs the fused step(s) and maps X, V back -- the paper's `target
@@ -309,13 +488,14 @@ def e2e_stream(n, params, local, a, two_step):
     import paper_conf_ipps_torresft22_b200 as P
 
     chunk = a.stream_chunk
-    st = P.SomierStream(P.Spread([local], 1, n[0] - 2, chunk=chunk), params, buffers=3)
+    st = P.SomierStream(P.Spread(list(devices), 1, n[0] - 2, chunk=chunk), params, buffers=3,
+                        cuda_devices=cuda_devices)
     grids = [torch.empty(tuple(n), dtype=torch.float64, pin_memory=True) for _ in range(12 if two_step else 9)]
     ptr = [g.data_ptr() for g in grids]
     X, V, XN = ptr[0:3], ptr[3:6], ptr[6:9]
     st.generate_ptrs(X + V)
     k = max(2, a.e2e_steps + (a.e2e_steps & 1))
-    rates = pcie_rates(local)
+    rates = pcie_rates(cuda_devices if cuda_devices is not None else devices)
 
     def one_step():
         st.run_ptrs(X, V, XN, 1)  # warm-up step
@@ -349,19 +529,20 @@ def e2e_stream(n, params, local, a, two_step):
     # the headline is the strict cycle: every step's inputs mapped in and every
     # step's result read back; the two-step cycle is reported beside it
     r = r1
-    cyc1 = ("somier_stream_run on pinned host grids: per chunk of %d planes map(to: X[start-1:size+2], "
-            "V[start:size]) -> fused K1 -> map(from: X[start:size], V[start:size]); 3 device slots, H2D/K1/D2H "
-            "overlapped, steps chained by per-chunk events (no barrier per step); every step's stats read back" % chunk)
+    cyc1 = ("somier_stream_run on pinned host grids, one host process driving devices(%s): per chunk of %d "
+            "planes map(to: X[start-1:size+2], V[start:size]) -> fused K1 -> map(from: X[start:size], "
+            "V[start:size]); 3 device slots per GPU, H2D/K1/D2H overlapped, steps chained by per-chunk events (no "
+            "barrier per step); every step's stats read back" % (",".join(str(d) for d in devices), chunk))
     cyc2 = ("somier_stream_run2 on pinned host grids: per chunk of %d planes map(to: X[start-2:size+4], "
             "V[start-1:size+2]) -> K1_TB2 (two steps) -> map(from: X[start:size], V[start:size]) into the other "
             "host buffers; 3 device slots, H2D/K1/D2H overlapped, launches chained by per-chunk events; every "
-            "launch's stats (each second step) read back" % chunk)
+            "step's stats read back" % chunk)
     out = {"value": r["value"], "unit": UNIT, "h2d_bytes_per_step": r["h2d_bytes_per_step"],
            "d2h_bytes_per_step": r["d2h_bytes_per_step"], "steps": k, "wall_s": r["wall_s"],
            "cycle": cyc1,
            "roofline": {"bound": "pcie", "achieved_gbs": r["achieved_gbs"],
                         "peak_gbs_bidir_measured": rates["bidir_total"], "h2d_gbs": rates["h2d"],
-                        "d2h_gbs": rates["d2h"], "frac": r["frac_pcie"]},
+                        "d2h_gbs": rates["d2h"], "frac": r["frac_pcie"], "gpus": rates["gpus"]},
            "last_step_vmax": r["last_step_vmax"]}
     if two_step:
         out["two_step_cycle"] = {"value": r2["value"], "h2d_bytes_per_step": r2["h2d_bytes_per_step"],
@@ -485,97 +666,109 @@ def run_ours(a):
         launches = all_sum(launches)
     value = interior(n) * a.steps / (ms * 1e-3)
     # diagnostic only (not part of the timed region): per-launch durations of a
-    # few more steps, each bracketed by events -- shows the power-cap ramp
+    # few more steps, each bracketed by events -- shows the power-cap ramp --
+    # with the library's launch timing on (somier_set_timing: flag-wait and
+    # kernel time of every launch on this rank; graph replay off)
     nd = min(a.steps, 20)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(nd)]
+    s.set_timing(True)
     with torch.cuda.stream(stream):
         for i in range(0, nd, per_call):
             ev[i][0].record(stream)
             s.step(per_call)
             ev[i][1].record(stream)
     s.sync()
+    tim = s.take_timing()
+    s.set_timing(False)
     barrier()
     per_step = [ev[i][0].elapsed_time(ev[i][1]) for i in range(0, nd, per_call)]  # per launch
 
     step_dist = {"min": min(per_step), "median": statistics.median(per_step), "max": max(per_step),
                  "first5": statistics.mean(per_step[:5]), "last5": statistics.mean(per_step[-5:]),
                  "note": "diagnostic pass after the timed region, %d launches each bracketed by events" % len(per_step)}
+
+    # sustained: >= --sustained-s seconds of steps in one somier_step call (the
+    # board's steady state under its power cap), with its own clock samples
+    sustained = None
+    if a.sustained_s > 0:
+        ss = int(a.sustained_s * 1e3 / max(1e-3, ms / a.steps))
+        ss = max(per_call, ss - ss % per_call)
+        if multi:
+            ss = int(all_max(ss))
+        csus = ClockSampler(local)
+        csus.start()
+        time.sleep(0.3)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        csus.mark_start()
+        e0.record(stream)
+        s.step(ss)
+        e1.record(stream)
+        s.sync()
+        csus.mark_end()
+        barrier()
+        sms = e0.elapsed_time(e1)
+        if multi:
+            sms = float(all_max(sms))
+        sustained = {"steps": ss, "seconds": sms * 1e-3, "value": interior(n) * ss / (sms * 1e-3),
+                     "ms_per_step": sms / ss, "clocks": csus.stop(),
+                     "note": "one somier_step(%d) call after the timed region, CUDA events, max over ranks" % ss}
+
     # roofline of the dominant kernel (K1) on this rank's launches: mean launch
     # duration over the timed region (this rank's time / this rank's launches)
     k1_ms = t_start.elapsed_time(t_end) / max(1, my_launches)
     c0 = my_chunks[0]
-    alg = algorithmic_bytes(n, c0.start, c0.size)
+    # algorithmic bytes = 24 n1 n2 per X_t plane read + 72 B per
+    # interior node (V read + write, X_{t+1} write) per STEP (~96 B per
+    # node-update); a launch processes per_call steps of its chunk
+    alg_step = sum(algorithmic_bytes(n, c.start, c.size) for c in my_chunks) / len(my_chunks)
+    alg = alg_step * per_call
+    nu_launch = sum(interior_of(n, c.size) for c in my_chunks) / len(my_chunks) * per_call
     peak, peak_src = load_peaks()
     achieved = alg / (k1_ms * 1e-3) / 1e9
     kname = {P.K1_MARCH: "march", P.K1_MARCH2: "march2", P.K1_DIRECT: "direct", P.K1_TB2: "tb2"}[in_use]
     # the same launches against the fp64 pipe: the method's fp64 instructions
     # per node-update (FP64_OPS_* below) x node-updates per launch
-    fp64_alg = interior_of(n, c0.size) * per_call * fp64_ops_per_node_update(per_call == 2)
+    fp64_alg = nu_launch * fp64_ops_per_node_update()
     fp64_peak, fp64_src = load_fp64_peak()
     fp64_achieved = fp64_alg / (k1_ms * 1e-3) / 1e12
-    traffic = load_traffic(n, kname) if not multi and len(my_chunks) == 1 else None
+    traffic, traffic_src = load_traffic(n, kname) if len(my_chunks) == 1 and c0.size == n[0] - 2 else (None, None)
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()
+    roof = roofline_obj(achieved, peak, peak_src, traffic, traffic_src, k1_ms, kname, alg, alg_step, nu_launch,
+                        per_call, step_dist, copy_gbs, fp64_achieved / fp64_peak)
+    # per rank: this rank's launch time, flag-wait time and kernel time
+    mine = {"rank": rank, "chunks": [[c.start, c.size] for c in my_chunks], "avg_launch_ms": k1_ms,
+            "hbm_frac": achieved / peak, "fp64_frac": fp64_achieved / fp64_peak,
+            "diag_wait_ms_per_launch": tim["wait_ms"] / max(1, tim["launches"]),
+            "diag_kernel_ms_per_launch": tim["kernel_ms"] / max(1, tim["launches"]),
+            "diag_wait_max_ms": tim["wait_max_ms"]}
+    ranks = PD.all_gather_obj(mine) if multi else [mine]
+    halo = halo_info(n, spread.chunks(), world, per_call == 2, ranks)
+    if multi:
+        roof["per_rank"] = ranks
 
-    # end-to-end through the public API with pinned host buffers. N = 1: the
-    # host-streamed cycle (e2e_stream: one step per round trip; the two-step
-    # cycle beside it when the resident kernel is K1_TB2). N > 1: per step, map(to) the whole state (X
-    # with halos, V), one step, read the centers result and map(from) the
-    # state -- the paper's One Buffer cycle, in core.
+    # end-to-end through the public C ABI with HOST buffers, the same cycle at
+    # every N: the host-streamed Somier (somier_stream_run, the paper's own
+    # experiment) over devices(0..N-1) from ONE host process (the paper's model,
+    # PAPER.md:346-399) -- at N > 1 rank 0 drives every GPU after all ranks
+    # released their resident grids; the other ranks wait.
     e2e = None
-    if not a.no_e2e and not multi:
-        s.close()  # free the resident grid: the streamed mode needs only a few chunk buffers
-        torch.cuda.empty_cache()
-        e2e = e2e_stream(n, params, local, a, two_step=(in_use == P.K1_TB2))
-    elif not a.no_e2e:
-        shape = tuple(n)
-        host = [torch.empty(shape, dtype=torch.float64, pin_memory=True) for _ in range(6)]
-        ptrs = [h.data_ptr() for h in host]
-        s.read_ptrs(ptrs)
-        h2d = d2h = 0
-        for c in my_chunks:
-            plane = n[1] * n[2] * 8
-            h2d += 3 * (c.size + 2) * plane + 3 * c.size * plane
-            d2h += 3 * c.size * plane * 2 + (3 * plane if c.start == 1 else 0) + (3 * plane if c.start + c.size == n[0] - 1 else 0)
-        # warm-up cycle
-        s.load_ptrs(ptrs)
-        s.step(1)
-        s.stats()
-        s.read_ptrs(ptrs)
-        barrier()
-        k = max(1, a.e2e_steps)
-        t0 = time.perf_counter()
-        e_start = torch.cuda.Event(enable_timing=True)
-        e_end = torch.cuda.Event(enable_timing=True)
-        e_start.record(stream)
-        for _ in range(k):
-            s.load_ptrs(ptrs)
-            if multi:
-                s.sync()
-                torch.distributed.barrier()
-            s.step(1)
-            if multi:
-                PD.gather_stats(s)
-            else:
-                s.stats()
-            s.read_ptrs(ptrs)
-        e_end.record(stream)
-        s.sync()
-        barrier()
-        e_ms = e_start.elapsed_time(e_end)
-        wall = time.perf_counter() - t0
-        if multi:
-            e_ms = float(all_max(e_ms))
-        e2e = {"value": interior(n) * k / (e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": int(h2d * world),
-               "d2h_bytes_per_step": int(d2h * world) + 88 * world, "steps": k, "wall_s": wall,
-               "cycle": "somier_load (map to: X[start-1:size+2], V) -> somier_step(1) -> somier_stats -> "
-                        "somier_read (map from) per step, pinned host buffers"}
-        del host
+    s.close()
+    torch.cuda.empty_cache()
+    barrier()
+    if not a.no_e2e and rank == 0:
+        cuda_devs = [0] * world if a.share_gpu else list(range(world))
+        e2e = e2e_stream(n, params, list(range(world)), a, two_step=(in_use == P.K1_TB2), cuda_devices=cuda_devs)
+    barrier()
+
+    verify = run_verify(a, n, params, world, rank, local, multi) if a.verify else None
 
     cpu = None
     if rank == 0 and not multi and not a.no_cpu_baseline:
-        rate, desc, steps, el = oracle_sample(n, budget_s=a.cpu_seconds)
-        cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": desc}
+        cpu = oracle_sample(n, budget_s=a.cpu_seconds)
+        if not a.no_cpu_all_cores and len(host_cpu()[2]) > 1:
+            cpu["all_cores"] = oracle_sample(n, budget_s=a.cpu_seconds / 2, omp=True)
 
     if rank == 0:
         line = {
@@ -587,28 +780,23 @@ def run_ours(a):
                                  % (",".join(str(d) for d in spread.devices), n[0] - 2, spread.chunk_size),
                        "kernel": "K1_" + kname.upper(), "l2": "no flush: 12.9 GB state >> 126 MB L2",
                        "seed": 42},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "k1_%s_kernel" % kname, "algorithmic_bytes_per_launch": alg,
-                         "avg_launch_ms": k1_ms, "launch_ms_distribution": step_dist,
-                         "sustained_copy_gbs": copy_gbs, "steps_per_launch": per_call,
-                         "one_step_equivalent_gbs": alg * per_call / (k1_ms * 1e-3) / 1e9,
-                         "note": ("K1_TB2 advances two steps per pass over HBM: 'achieved' counts the bytes a launch "
-                                  "must move (one pass); one_step_equivalent_gbs is the rate the one-step method "
-                                  "would need for the same node-updates/s" if per_call == 2 else
-                                  "one step per launch")},
+            "roofline": roof,
             "roofline_fp64": {"bound": "alu", "achieved": fp64_achieved, "peak": fp64_peak, "unit": "Tinstr/s",
                               "frac": fp64_achieved / fp64_peak, "peak_source": fp64_src,
                               "alg_instr_per_launch": fp64_alg,
-                              "alg_instr_per_node_update": fp64_ops_per_node_update(per_call == 2),
-                              "note": "fp64 lane-instructions of node_math.cuh per node-update with spring reuse "
-                                      "(DESIGN.md §6); recomputed ring / tile padding not counted"},
+                              "alg_instr_per_node_update": fp64_ops_per_node_update(),
+                              "note": "fp64 lane-instructions of node_math.cuh / stats.cuh per node-update with "
+                                      "spring reuse and every step's stats (DESIGN.md §6); recomputed ring / tile "
+                                      "padding not counted"},
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
-            "halo": halo_info(n, spread.chunks(), world, per_call == 2),
-            "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax},
+            "halo": halo, "sustained": sustained,
+            "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax, "every_step": True,
+                      "note": "centres and vmax of every step are computed inside the timed region "
+                              "(somier_stats_history reads any of the last %d)" % P.STATS_HISTORY},
         }
+        if verify is not None:
+            line["verify"] = verify
         print(json.dumps(line), flush=True)
-    s.close()
     if multi:
         torch.distributed.barrier()
         torch.distributed.destroy_process_group()
@@ -617,6 +805,8 @@ def run_ours(a):
 
 def main():
     a = parse()
+    if a.oracle_child is not None:
+        return oracle_child(a.oracle_child)
     if a.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
     if a.impl == "reference":

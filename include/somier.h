@@ -220,6 +220,27 @@ spread_status somier_launch_count(somier_t h, int64_t* launches);
  * K1_MARCH2. EINVAL on NULL arguments. */
 spread_status somier_kernel_in_use(somier_t h, int32_t* kernel);
 
+/*
+ * Launch timing (diagnostics; SURVEY.md §8(d) "halo time"): while on, every K1
+ * launch of this handle is bracketed by three CUDA events on its stream --
+ * before the neighbour-flag waits (cuStreamWaitValue64), after them (= kernel
+ * start), after the kernel -- and CUDA-graph replay is off (launches are
+ * enqueued one by one, without programmatic dependent launch).
+ * somier_take_timing blocks, sums the recorded launches and forgets them:
+ *   wait_ms    time the launches' streams sat in the flag waits, i.e. waiting
+ *              for the neighbours' previous launch (their halo stores into this
+ *              chunk and their skew)
+ *   kernel_ms  time inside the kernels (the halo exchange is fused: the peer
+ *              stores run inside the kernel)
+ */
+typedef struct {
+    int64_t launches;
+    double wait_ms, kernel_ms;          /* sums over the launches */
+    double wait_max_ms, kernel_max_ms;  /* largest single launch  */
+} somier_timing_t;
+spread_status somier_set_timing(somier_t h, int on);
+spread_status somier_take_timing(somier_t h, somier_timing_t* out);
+
 /* Device bytes this handle allocated (all devices). */
 spread_status somier_device_bytes(somier_t h, int64_t* bytes);
 

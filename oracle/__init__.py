@@ -80,34 +80,50 @@ def lib():
     if _lib is None:
         # ORACLE_LIB: an alternative build of somier_oracle.c (tools/mutate_oracle.py
         # points it at deliberately broken mutants to show the pins catch them)
-        path = os.environ.get("ORACLE_LIB") or build_oracle.build()
-        L = ctypes.CDLL(path)
-        dp = ctypes.POINTER(ctypes.c_double)
-        P = ctypes.POINTER(_Params)
-        S = ctypes.POINTER(_Stats)
-        L.oracle_splitmix64_at.restype = ctypes.c_uint64
-        L.oracle_splitmix64_at.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
-        L.oracle_rest_position.argtypes = [P, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, dp]
-        L.oracle_init.argtypes = [P] + [dp] * 6
-        i64a = ctypes.POINTER(ctypes.c_int64)
-        L.oracle_init_window.argtypes = [P, i64a, i64a] + [dp] * 6
-        L.oracle_spring.argtypes = [dp, dp, ctypes.c_double, ctypes.c_double, dp]
-        for name in ("oracle_acceleration_1", "oracle_velocity_1", "oracle_position_1"):
-            fn = getattr(L, name)
-            fn.restype = ctypes.c_double
-        L.oracle_acceleration_1.argtypes = [ctypes.c_double, ctypes.c_double]
-        L.oracle_velocity_1.argtypes = [ctypes.c_double] * 3
-        L.oracle_position_1.argtypes = [ctypes.c_double] * 3
-        L.oracle_forces.argtypes = [P] + [dp] * 6
-        L.oracle_accelerations.argtypes = [P] + [dp] * 6
-        L.oracle_velocities.argtypes = [P] + [dp] * 6
-        L.oracle_positions.argtypes = [P] + [dp] * 9
-        L.oracle_centers.argtypes = [P] + [dp] * 6 + [S]
-        L.oracle_step.argtypes = [P] + [dp] * 9 + [S]
-        L.oracle_run.argtypes = [P, ctypes.c_int64] + [dp] * 6 + [S]
-        L.oracle_stencil3.argtypes = [dp, dp, ctypes.c_int64]
-        _lib = L
+        _lib = _bind(ctypes.CDLL(os.environ.get("ORACLE_LIB") or build_oracle.build()))
     return _lib
+
+
+_lib_omp = None
+
+
+def lib_omp():
+    """The optional all-cores build of the same source (-fopenmp): bench.py's
+    second CPU-baseline line. OMP_NUM_THREADS applies when it is first loaded."""
+    global _lib_omp
+    if _lib_omp is None:
+        _lib_omp = _bind(ctypes.CDLL(build_oracle.build_omp()))
+    return _lib_omp
+
+
+def _bind(L):
+    dp = ctypes.POINTER(ctypes.c_double)
+    P = ctypes.POINTER(_Params)
+    S = ctypes.POINTER(_Stats)
+    L.oracle_splitmix64_at.restype = ctypes.c_uint64
+    L.oracle_splitmix64_at.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+    L.oracle_rest_position.argtypes = [P, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, dp]
+    L.oracle_init.argtypes = [P] + [dp] * 6
+    i64a = ctypes.POINTER(ctypes.c_int64)
+    L.oracle_init_window.argtypes = [P, i64a, i64a] + [dp] * 6
+    L.oracle_spring.argtypes = [dp, dp, ctypes.c_double, ctypes.c_double, dp]
+    for name in ("oracle_acceleration_1", "oracle_velocity_1", "oracle_position_1"):
+        fn = getattr(L, name)
+        fn.restype = ctypes.c_double
+    L.oracle_acceleration_1.argtypes = [ctypes.c_double, ctypes.c_double]
+    L.oracle_velocity_1.argtypes = [ctypes.c_double] * 3
+    L.oracle_position_1.argtypes = [ctypes.c_double] * 3
+    L.oracle_forces.argtypes = [P] + [dp] * 6
+    L.oracle_accelerations.argtypes = [P] + [dp] * 6
+    L.oracle_velocities.argtypes = [P] + [dp] * 6
+    L.oracle_positions.argtypes = [P] + [dp] * 9
+    L.oracle_centers.argtypes = [P] + [dp] * 6 + [S]
+    L.oracle_step.argtypes = [P] + [dp] * 9 + [S]
+    L.oracle_run.argtypes = [P, ctypes.c_int64] + [dp] * 6 + [S]
+    L.oracle_run_timed.argtypes = [P, ctypes.c_int64] + [dp] * 6 + [S, dp]
+    L.oracle_threads.restype = ctypes.c_int
+    L.oracle_stencil3.argtypes = [dp, dp, ctypes.c_int64]
+    return L
 
 
 def _ptr(a: np.ndarray):
@@ -241,6 +257,22 @@ def step(s: State) -> tuple:
         raise ValueError("oracle_step failed")
     out.x, out.y, out.z = xn
     return out, _stats(st)
+
+
+def run_timed(s: State, nsteps: int, omp: bool = False) -> tuple:
+    """nsteps steps on a copy of s with the C step loop timed by the steady clock
+    (oracle_run_timed); returns (final State, Stats of the last step, seconds,
+    threads). omp: the all-cores build of the same source."""
+    L = lib_omp() if omp else lib()
+    out = s.copy()
+    st = _Stats()
+    sec = ctypes.c_double()
+    rc = L.oracle_run_timed(ctypes.byref(s.p.c()), int(nsteps),
+                            *(_ptr(a) for a in (out.x, out.y, out.z, out.vx, out.vy, out.vz)),
+                            ctypes.byref(st), ctypes.byref(sec))
+    if rc != 0:
+        raise ValueError("oracle_run_timed failed")
+    return out, _stats(st), sec.value, int(L.oracle_threads())
 
 
 def run(s: State, nsteps: int) -> tuple:

@@ -12,6 +12,10 @@
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
+#include <time.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 #define IDX(p, i, j, k) ((((i) * (p)->n[1]) + (j)) * (p)->n[2] + (k))
 
@@ -128,6 +132,10 @@ double oracle_position_1(double x, double v, double dt) { return x + v * dt; }
 void oracle_forces(const oracle_params* p, const double* x, const double* y, const double* z,
                    double* fx, double* fy, double* fz) {
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
+    /* the optional all-cores build (-fopenmp, liboracle_omp.so) splits the i
+     * loop of the node-independent kernels; every node is computed by the same
+     * expressions, so the results are bit-identical to the sequential build */
+#pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < n0; i++)
         for (int64_t j = 0; j < n1; j++)
             for (int64_t k = 0; k < n2; k++) {
@@ -160,6 +168,7 @@ void oracle_forces(const oracle_params* p, const double* x, const double* y, con
 void oracle_accelerations(const oracle_params* p, const double* fx, const double* fy, const double* fz,
                           double* ax, double* ay, double* az) {
     const int64_t n = nnodes(p);
+#pragma omp parallel for schedule(static)
     for (int64_t g = 0; g < n; g++) {
         ax[g] = oracle_acceleration_1(fx[g], p->mass);
         ay[g] = oracle_acceleration_1(fy[g], p->mass);
@@ -169,6 +178,7 @@ void oracle_accelerations(const oracle_params* p, const double* fx, const double
 
 void oracle_velocities(const oracle_params* p, const double* ax, const double* ay, const double* az,
                        double* vx, double* vy, double* vz) {
+#pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < p->n[0]; i++)
         for (int64_t j = 0; j < p->n[1]; j++)
             for (int64_t k = 0; k < p->n[2]; k++) {
@@ -183,6 +193,7 @@ void oracle_velocities(const oracle_params* p, const double* ax, const double* a
 void oracle_positions(const oracle_params* p, const double* x, const double* y, const double* z,
                       const double* vx, const double* vy, const double* vz,
                       double* xn, double* yn, double* zn) {
+#pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < p->n[0]; i++)
         for (int64_t j = 0; j < p->n[1]; j++)
             for (int64_t k = 0; k < p->n[2]; k++) {
@@ -244,14 +255,16 @@ int oracle_step(const oracle_params* p, const double* x, const double* y, const 
     return 0;
 }
 
-int oracle_run(const oracle_params* p, int64_t nsteps, double* x, double* y, double* z,
-               double* vx, double* vy, double* vz, oracle_stats* stats) {
+int oracle_run_timed(const oracle_params* p, int64_t nsteps, double* x, double* y, double* z,
+                     double* vx, double* vy, double* vz, oracle_stats* stats, double* seconds) {
     if (!valid(p) || nsteps < 0) return -1;
     const int64_t n = nnodes(p);
     double* buf = (double*)malloc(sizeof(double) * (size_t)n * 3);
     if (!buf) return -1;
     double *xa = x, *ya = y, *za = z;
     double *xb = buf, *yb = buf + n, *zb = buf + 2 * n;
+    struct timespec t0, t1;
+    clock_gettime(CLOCK_MONOTONIC, &t0);
     for (int64_t s = 0; s < nsteps; s++) {
         if (oracle_step(p, xa, ya, za, vx, vy, vz, xb, yb, zb, stats) != 0) {
             free(buf);
@@ -262,6 +275,8 @@ int oracle_run(const oracle_params* p, int64_t nsteps, double* x, double* y, dou
         t = ya; ya = yb; yb = t;
         t = za; za = zb; zb = t;
     }
+    clock_gettime(CLOCK_MONOTONIC, &t1);
+    if (seconds) *seconds = (double)(t1.tv_sec - t0.tv_sec) + 1e-9 * (double)(t1.tv_nsec - t0.tv_nsec);
     if (xa != x) {
         memcpy(x, xa, sizeof(double) * (size_t)n);
         memcpy(y, ya, sizeof(double) * (size_t)n);
@@ -270,6 +285,19 @@ int oracle_run(const oracle_params* p, int64_t nsteps, double* x, double* y, dou
     if (nsteps == 0 && stats) oracle_centers(p, x, y, z, vx, vy, vz, stats);
     free(buf);
     return 0;
+}
+
+int oracle_run(const oracle_params* p, int64_t nsteps, double* x, double* y, double* z,
+               double* vx, double* vy, double* vz, oracle_stats* stats) {
+    return oracle_run_timed(p, nsteps, x, y, z, vx, vy, vz, stats, NULL);
+}
+
+int oracle_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
 }
 
 void oracle_stencil3(const double* a, double* b, int64_t n) {

@@ -120,6 +120,19 @@ int oracle_step(const oracle_params* p, const double* x, const double* y, const 
 int oracle_run(const oracle_params* p, int64_t nsteps, double* x, double* y, double* z,
                double* vx, double* vy, double* vz, oracle_stats* stats);
 
+/* oracle_run with the step loop timed by CLOCK_MONOTONIC (the steady clock):
+ * *seconds = wall time of the nsteps steps (every step's five kernels, stats
+ * included), without the setup and the final copy. For bench.py's CPU
+ * baseline. */
+int oracle_run_timed(const oracle_params* p, int64_t nsteps, double* x, double* y, double* z,
+                     double* vx, double* vy, double* vz, oracle_stats* stats, double* seconds);
+
+/* Threads the node loops use: 1 for the sequential build; omp_get_max_threads()
+ * for the optional all-cores build (liboracle_omp.so, same source compiled with
+ * -fopenmp; the i loops of forces / velocities / positions and the node loop of
+ * accelerations split statically; bit-identical results, tested). */
+int oracle_threads(void);
+
 /* Listing 2-4 toy loop: B[i] = A[i-1]+A[i]+A[i+1] for
  * i in [1, N-1), evaluated left to right. */
 void oracle_stencil3(const double* a, double* b, int64_t n);

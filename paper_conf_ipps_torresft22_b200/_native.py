@@ -60,6 +60,16 @@ class somier_stats_t(ctypes.Structure):
     ]
 
 
+class somier_timing_t(ctypes.Structure):
+    _fields_ = [
+        ("launches", ctypes.c_int64),
+        ("wait_ms", ctypes.c_double),
+        ("kernel_ms", ctypes.c_double),
+        ("wait_max_ms", ctypes.c_double),
+        ("kernel_max_ms", ctypes.c_double),
+    ]
+
+
 class spread_reduce_result(ctypes.Structure):
     _fields_ = [
         ("value", ctypes.c_double),
@@ -109,6 +119,8 @@ SIGNATURES = [
     ("somier_sync", ctypes.c_int, [_VP]),
     ("somier_stats", ctypes.c_int, [_VP, ctypes.POINTER(somier_stats_t)]),
     ("somier_stats_history", ctypes.c_int, [_VP, ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
+    ("somier_set_timing", ctypes.c_int, [_VP, ctypes.c_int]),
+    ("somier_take_timing", ctypes.c_int, [_VP, ctypes.POINTER(somier_timing_t)]),
     ("somier_stats_combine", ctypes.c_int, [ctypes.POINTER(somier_stats_t), ctypes.c_int,
                                             ctypes.POINTER(somier_params), ctypes.POINTER(somier_stats_t)]),
     ("somier_read", ctypes.c_int, [_VP] + [_DP] * 6),

@@ -150,6 +150,14 @@ struct somier_s {
     int graph_pos = -1;
     cudaGraphExec_t graph_exec = nullptr;
     cudaGraphExec_t tb2_graph[4] = {nullptr, nullptr, nullptr, nullptr};  // by (X buffer parity, step parity)
+    // somier_set_timing: per launch, events before the neighbour-flag waits,
+    // after them (= kernel start) and after the kernel
+    struct TimingRec {
+        int device;
+        cudaEvent_t a, b, c;
+    };
+    bool timing = false;
+    std::vector<TimingRec> trecs;
 
     bool unit_mass() const { return p.mass == 1.0; }
     paper::K1Variant variant() const {
@@ -184,6 +192,17 @@ spread_status cuda_fail(somier_t h, cudaError_t e, const char* what) {
         cudaError_t e_ = (call);                                  \
         if (e_ != cudaSuccess) return cuda_fail((h), e_, #call);  \
     } while (0)
+
+// somier_set_timing instrumentation: events around one launch's waits and kernel
+spread_status timing_begin(somier_t h, int device, cudaStream_t st, somier_s::TimingRec* r) {
+    r->device = device;
+    r->a = r->b = r->c = nullptr;
+    CUDA_TRY(h, cudaEventCreate(&r->a));
+    CUDA_TRY(h, cudaEventCreate(&r->b));
+    CUDA_TRY(h, cudaEventCreate(&r->c));
+    CUDA_TRY(h, cudaEventRecord(r->a, st));
+    return SPREAD_OK;
+}
 
 spread_status check_params(const somier_params* p) {
     if (!p) PAPER_FAIL(SPREAD_EINVAL, "somier: params is NULL");
@@ -740,7 +759,7 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
         // per (buffer parity, step parity) -- everything a launch depends on --
         // and replayed as a CUDA graph; the handle's first pair runs eagerly
         // (lazy host-side state is set up outside any capture).
-        if (h->graph_ok && nsteps >= 4) {
+        if (h->graph_ok && !h->timing && nsteps >= 4) {
             if (h->launches == 0) {
                 spread_status st = enqueue_tb2(h, true);
                 if (st != SPREAD_OK) return st;
@@ -786,7 +805,7 @@ spread_status somier_step(somier_t h, int64_t nsteps) {
     // All chunks on one stream (no cross-stream flags): the launches of two
     // consecutive steps depend only on the buffer parity, so a CUDA graph of an
     // (even, odd) step pair is captured once and replayed.
-    if (h->graph_ok && nsteps >= 2) {
+    if (h->graph_ok && !h->timing && nsteps >= 2) {
         if (h->step & 1) {
             spread_status st = enqueue_steps(h, 1);
             if (st != SPREAD_OK) return st;
@@ -845,6 +864,11 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             const Chunk* right = c + 1 < nch ? &h->chunks[c + 1] : nullptr;
             const bool fl = left && h->needs_flags(me, *left);
             const bool fr = right && h->needs_flags(me, *right);
+            somier_s::TimingRec tr{};
+            if (h->timing) {
+                spread_status ts = timing_begin(h, me.device, st, &tr);
+                if (ts != SPREAD_OK) return ts;
+            }
             // wait until the neighbours finished step t-1 (their halo stores into
             // my X_t are visible, and they no longer read the halo buffer I am
             // about to write): flags[0] = from_left, flags[1] = from_right.
@@ -880,8 +904,13 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.tmap_v = &me.tmap_v[vb];
             a.tmap_x2_cur = &me.tmap_x2[cur];
             a.tmap_v2 = &me.tmap_v2[vb];
-            a.pdl = h->pdl ? 1 : 0;
+            a.pdl = h->pdl && !h->timing ? 1 : 0;
+            if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
+            if (h->timing) {
+                CUDA_TRY(h, cudaEventRecord(tr.c, st));
+                h->trecs.push_back(tr);
+            }
             h->launches++;
         }
         h->step++;
@@ -915,6 +944,11 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         const Chunk* right = c + 1 < nch ? &h->chunks[c + 1] : nullptr;
         const bool fl = left && h->needs_flags(me, *left);
         const bool fr = right && h->needs_flags(me, *right);
+        somier_s::TimingRec tr{};
+        if (h->timing) {
+            spread_status ts = timing_begin(h, me.device, st, &tr);
+            if (ts != SPREAD_OK) return ts;
+        }
         for (int side = 0; side < 2; side++) {
             if (t == 0 || !(side ? fr : fl)) continue;
             CUresult r = h->wait_value64((CUstream)st, (CUdeviceptr)&me.flags()[side], (cuuint64_t)t,
@@ -955,7 +989,12 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         a.signal_hi = fr ? &right->flags()[0] : nullptr;
         a.signal_value = (unsigned long long)t_end;
         a.done_counter = me.counter();
+        if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
         CUDA_TRY(h, paper::launch_k1_tb2(a, o, h->unit_mass(), st));
+        if (h->timing) {
+            CUDA_TRY(h, cudaEventRecord(tr.c, st));
+            h->trecs.push_back(tr);
+        }
         h->launches++;
     }
     h->step = t_end;
@@ -1222,6 +1261,38 @@ spread_status somier_device_bytes(somier_t h, int64_t* bytes) {
     return SPREAD_OK;
 }
 
+spread_status somier_set_timing(somier_t h, int on) {
+    if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_set_timing: NULL handle");
+    h->timing = on != 0;
+    return SPREAD_OK;
+}
+
+spread_status somier_take_timing(somier_t h, somier_timing_t* out) {
+    if (!h || !out) PAPER_FAIL(SPREAD_EINVAL, "somier_take_timing: NULL argument");
+    spread_status st = sync_all(h);
+    if (st != SPREAD_OK) return st;
+    out->launches = 0;
+    out->wait_ms = out->kernel_ms = 0.0;
+    out->wait_max_ms = out->kernel_max_ms = 0.0;
+    for (auto& r : h->trecs) {
+        float w = 0.f, k = 0.f;
+        CUDA_TRY(h, cudaSetDevice(r.device));
+        CUDA_TRY(h, cudaEventElapsedTime(&w, r.a, r.b));
+        CUDA_TRY(h, cudaEventElapsedTime(&k, r.b, r.c));
+        out->launches++;
+        out->wait_ms += w;
+        out->kernel_ms += k;
+        out->wait_max_ms = std::max(out->wait_max_ms, (double)w);
+        out->kernel_max_ms = std::max(out->kernel_max_ms, (double)k);
+    }
+    for (auto& r : h->trecs) {
+        cudaSetDevice(r.device);
+        for (cudaEvent_t e : {r.a, r.b, r.c}) cudaEventDestroy(e);
+    }
+    h->trecs.clear();
+    return SPREAD_OK;
+}
+
 spread_status somier_destroy(somier_t h) {
     if (!h) return SPREAD_OK;
     for (auto& d : h->devs)
@@ -1229,6 +1300,10 @@ spread_status somier_destroy(somier_t h) {
             cudaSetDevice(d.device);
             cudaStreamSynchronize(d.stream);
         }
+    for (auto& r : h->trecs) {
+        cudaSetDevice(r.device);
+        for (cudaEvent_t e : {r.a, r.b, r.c}) cudaEventDestroy(e);
+    }
     if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
     for (auto& ge : h->tb2_graph)
         if (ge) cudaGraphExecDestroy(ge);

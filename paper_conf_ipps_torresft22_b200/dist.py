@@ -35,6 +35,15 @@ def all_gather_bytes(blob: bytes, group=None) -> List[bytes]:
     return [bytes(b) for b in out]
 
 
+def all_gather_obj(obj, group=None) -> list:
+    """Every rank's picklable `obj`, in rank order (plumbing for bench reports)."""
+    import torch.distributed as dist
+
+    out: List[Optional[object]] = [None] * dist.get_world_size(group)
+    dist.all_gather_object(out, obj, group=group)
+    return out
+
+
 def connect(s: Somier, group=None) -> None:
     """Exchange IPC blobs with every rank and open the neighbours' memory."""
     import torch.distributed as dist

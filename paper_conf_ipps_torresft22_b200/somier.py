@@ -164,6 +164,17 @@ class Somier:
         N.check(N.lib().somier_stats_history(self._h, int(first_step), count, out), "somier_stats_history")
         return [Stats.from_c(out[i]) for i in range(count)]
 
+    def set_timing(self, on: bool = True) -> None:
+        """somier_set_timing: bracket every launch with events (waits / kernel)."""
+        N.check(N.lib().somier_set_timing(self._h, 1 if on else 0), "somier_set_timing")
+
+    def take_timing(self) -> dict:
+        """somier_take_timing: launches, summed and largest flag-wait and kernel ms since the last take."""
+        t = N.somier_timing_t()
+        N.check(N.lib().somier_take_timing(self._h, ctypes.byref(t)), "somier_take_timing")
+        return {"launches": t.launches, "wait_ms": t.wait_ms, "kernel_ms": t.kernel_ms,
+                "wait_max_ms": t.wait_max_ms, "kernel_max_ms": t.kernel_max_ms}
+
     # -- data movement -------------------------------------------------------
     def read(self, X=None, V=None):
         """Copy the owned planes into host grids; returns (X, V), each (3, n0, n1, n2)."""

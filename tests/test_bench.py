@@ -64,7 +64,8 @@ def test_warmup_below_three_is_refused():
 
 @pytest.mark.gpu
 def test_our_arm_json_line_one_gpu():
-    lines, _ = _run(["bench.py", "--grid", "64", "--steps", "4", "--warmup", "3", "--no-cpu-baseline", "--no-e2e"])
+    lines, _ = _run(["bench.py", "--grid", "64", "--steps", "4", "--warmup", "3", "--no-cpu-baseline", "--no-e2e",
+                     "--verify", "--sustained-s", "0.2"])
     assert len(lines) == 1
     d = json.loads(lines[0])
     _check_common(d, 1, 4, 3)
@@ -72,7 +73,12 @@ def test_our_arm_json_line_one_gpu():
     r = d["roofline"]
     assert r["bound"] == "hbm" and r["unit"] == "GB/s" and r["peak"] > 0
     assert abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9
+    # 96 B per node-update (24 n1 n2 per X plane + 72 per interior node)
+    assert 90 < r["algorithmic_bytes_per_node_update"] < 110
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
+    assert d["verify"]["ok"] and d["verify"]["nodes_checked"] > 0
+    assert d["sustained"]["steps"] >= 2 and d["sustained"]["value"] > 0
+    assert d["stats"]["every_step"] is True
 
 
 @pytest.mark.gpu
@@ -80,10 +86,16 @@ def test_our_arm_two_ranks_share_one_gpu():
     """N = 2 through torchrun (the driver's launch), both ranks on cuda:0 over
     CUDA IPC: one JSON line, whole-job value, the fused exchange's halo bytes."""
     lines, r = _run(_torchrun(2, 29563) + ["bench.py", "--gpus", "2", "--grid", "64", "--steps", "4", "--warmup",
-                                           "3", "--share-gpu", "--no-cpu-baseline", "--no-e2e"],
+                                           "3", "--share-gpu", "--no-cpu-baseline", "--e2e-steps", "2",
+                                           "--stream-chunk", "8", "--verify", "--sustained-s", "0.2"],
                     env={"OMP_NUM_THREADS": "1"})
     assert len(lines) == 1, r.stdout[-2000:]
     d = json.loads(lines[0])
     _check_common(d, 2, 4, 3)
     assert d["gpu_launches"] > 0
-    assert d["halo"]["bytes_per_step_total"] > 0
+    h = d["halo"]
+    assert h["bytes_per_step_total"] > 0 and h["measured_wait_ms_per_launch"]["max"] >= 0
+    assert len(d["roofline"]["per_rank"]) == 2
+    # the same e2e cycle as at N = 1: host-streamed over devices(0, 1), one process
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0 and "somier_stream_run" in d["e2e"]["cycle"]
+    assert d["verify"]["ok"] and d["verify"]["nodes_checked"] > 0

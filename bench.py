@@ -344,8 +344,8 @@ def roofline_obj(achieved, peak, peak_src, traffic, traffic_src, k1_ms, kname, a
     closest = max(fr, key=fr.get)
     if per_call == 2:
         r["note"] = ("K1_TB2 advances two steps per pass over HBM, so it moves about half of §8(d)'s 96 B per "
-                     "node-update (one pass = %d B per launch): 'frac' > 1 against the one-step algorithmic "
-                     "bytes. The roof that binds is the fp64 issue / latency: neither the fp64 pipe nor HBM is "
+                     "node-update (one pass = %d B per launch): 'frac' can exceed 1 against the one-step "
+                     "algorithmic bytes. The roof that binds is the fp64 issue / latency: neither the fp64 pipe nor HBM is "
                      "saturated; closest: %s at %.2f" % (alg_step, closest, fr[closest]))
     else:
         r["note"] = "one step per launch; closest roof: %s at %.2f" % (closest, fr[closest])

@@ -50,6 +50,13 @@ struct StepArgs {
     unsigned long long* signal_hi;   // right neighbour's "from_left" flag
     unsigned long long signal_value;
     unsigned int* done_counter;      // per-chunk CTA completion counter (self-resetting)
+    // Early neighbour signals: the flag to a neighbour is published when the
+    // CTAs whose work touches that side (they store the boundary planes into
+    // its halo, or read this chunk's halo planes it will overwrite next) are
+    // done, not the whole grid. side_counter[0] / [1] count them (self-
+    // resetting); lo_ctas / hi_ctas are set by the launcher from its grid.
+    unsigned int* side_counter;
+    unsigned int lo_ctas, hi_ctas;
     // K1_MARCH: host pointers to the CUtensorMaps of x_cur and v (passed to the
     // kernel by value as __grid_constant__ parameters).
     const void* tmap_x_cur;

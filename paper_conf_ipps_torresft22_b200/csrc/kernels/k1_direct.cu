@@ -75,7 +75,7 @@ __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
         }
     }
     block_accumulate(st, scratch, slots.fin);
-    finish_launch(a, slots.t, 1);
+    finish_launch(a, slots.t, 1, blockIdx.z == 0, blockIdx.z == gridDim.z - 1);
 }
 
 }  // namespace
@@ -84,10 +84,12 @@ cudaError_t launch_k1_direct(const StepArgs& a, bool unit_mass, cudaStream_t str
     if (a.g.size <= 0) return cudaSuccess;
     dim3 block(kBX, kBY);
     dim3 grid((unsigned)((a.g.n2 + kBX - 1) / kBX), (unsigned)((a.g.n1 + kBY - 1) / kBY), (unsigned)a.g.size);
+    StepArgs b = a;
+    b.lo_ctas = b.hi_ctas = grid.x * grid.y;  // one plane per grid z: the first / last plane's CTAs
     if (unit_mass)
-        k1_direct_kernel<true><<<grid, block, 0, stream>>>(a);
+        k1_direct_kernel<true><<<grid, block, 0, stream>>>(b);
     else
-        k1_direct_kernel<false><<<grid, block, 0, stream>>>(a);
+        k1_direct_kernel<false><<<grid, block, 0, stream>>>(b);
     return cudaGetLastError();
 }
 

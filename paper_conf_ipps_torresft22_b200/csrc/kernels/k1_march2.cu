@@ -299,7 +299,7 @@ __global__ void __launch_bounds__(kThreads, 2)
         ph_nxt ^= (s_nxt == 0) ? 1u : 0u;
     }
     block_accumulate(st, sm.scratch, slots.fin);
-    finish_launch(a, slots.t, 1);
+    finish_launch(a, slots.t, 1, blockIdx.y == 0, blockIdx.y == gridDim.y - 1);
 }
 
 }  // namespace
@@ -344,6 +344,7 @@ cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t str
     nseg = (int)((a.g.size + mp.seg_planes - 1) / mp.seg_planes);
     dim3 grid((unsigned)tiles, (unsigned)nseg);
     dim3 block(kTK, kW);
+    mp.a.lo_ctas = mp.a.hi_ctas = grid.x;  // the first / last segment's CTAs
     const size_t smem = sizeof(Smem);
     const CUtensorMap& mx = *static_cast<const CUtensorMap*>(a.tmap_x2_cur);
     const CUtensorMap& mv = *static_cast<const CUtensorMap*>(a.tmap_v2);

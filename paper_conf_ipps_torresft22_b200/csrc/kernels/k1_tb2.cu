@@ -522,7 +522,9 @@ __global__ void __launch_bounds__(kThreads, 1)
 #error "K1_TB2 keeps step t+1's stats as bit-pattern sums (no STATS_FP64_ACC variant)"
 #endif
     }
-    finish_launch(a, slots.t, kTwo ? 2 : 1);
+    // lo side: stores planes start, start+1 into the left neighbour or reads
+    // planes below start; hi side: the mirror image (launch_k1_tb2 counts them)
+    finish_launch(a, slots.t, kTwo ? 2 : 1, pb <= start + 1, pe >= start + size - 1);
 }
 
 }  // namespace
@@ -592,6 +594,17 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
     if (tp.seg_planes < kMinSegPlanes) tp.seg_planes = (int)std::min<int64_t>(kMinSegPlanes, a.g.size);
     nseg = (int)((a.g.size + tp.seg_planes - 1) / tp.seg_planes);
     dim3 grid((unsigned)tiles, (unsigned)nseg), block(kTK, kW);
+    {  // CTAs of the segments that touch each neighbour (the kernel's lo_side / hi_side)
+        unsigned int lo = 0, hi = 0;
+        const int start = (int)a.g.start, size = (int)a.g.size;
+        for (int sg = 0; sg < nseg; sg++) {
+            const int pb = start + sg * tp.seg_planes, pe = std::min(start + size, pb + tp.seg_planes);
+            lo += pb <= start + 1 ? 1u : 0u;
+            hi += pe >= start + size - 1 ? 1u : 0u;
+        }
+        tp.a.lo_ctas = lo * (unsigned)tiles;
+        tp.a.hi_ctas = hi * (unsigned)tiles;
+    }
     const size_t smem = sizeof(Smem);
     const CUtensorMap& mx = *static_cast<const CUtensorMap*>(a.tmap_x_cur);
     const CUtensorMap& mv = *static_cast<const CUtensorMap*>(a.tmap_v);

@@ -13,28 +13,36 @@ __device__ __forceinline__ void st_release_sys_u64(unsigned long long* p, unsign
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// Call once per CTA, by all threads, after the CTA's last store. The last CTA
-// of the launch to finish advances the step word (stats ring, t = the step the
-// launch started from) and publishes the neighbours' flags.
-__device__ __forceinline__ void finish_launch(const StepArgs& a, unsigned long long t, int nsteps) {
-    const bool sig = a.signal_lo || a.signal_hi;
-    if (!sig && !a.step_word) return;
-    __shared__ unsigned int s_last;
-    __syncthreads();
+// Call once per CTA, by all threads, after the CTA's last store. lo_side /
+// hi_side: this CTA's work touches that neighbour (see StepArgs). The last
+// lo-side (hi-side) CTA to finish publishes the left (right) neighbour's flag
+// -- the neighbour's next launch needs only those CTAs done, so it can start
+// while this launch's interior CTAs still run. The last CTA of the whole grid
+// advances the step word (stats ring; t = the step the launch started from).
+__device__ __forceinline__ void finish_launch(const StepArgs& a, unsigned long long t, int nsteps, bool lo_side,
+                                              bool hi_side) {
+    const bool sig_lo = a.signal_lo && lo_side, sig_hi = a.signal_hi && hi_side;
+    if (!a.signal_lo && !a.signal_hi && !a.step_word) return;
+    __syncthreads();  // every thread's stores precede the leader's fence
     const bool leader = threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0;
-    if (leader) {
-        if (sig) __threadfence_system();
-        const unsigned int nblocks = gridDim.x * gridDim.y * gridDim.z;
-        const unsigned int prev = atomicAdd(a.done_counter, 1u);
-        s_last = (prev == nblocks - 1) ? 1u : 0u;
+    if (!leader) return;
+    if (sig_lo || sig_hi) __threadfence_system();
+    if (sig_lo && atomicAdd(&a.side_counter[0], 1u) == a.lo_ctas - 1) {
+        __threadfence_system();
+        a.side_counter[0] = 0u;  // self-reset for the next launch (stream-ordered)
+        st_release_sys_u64(a.signal_lo, a.signal_value);
     }
-    __syncthreads();
-    if (leader && s_last) {
-        if (sig) __threadfence_system();
-        *a.done_counter = 0u;  // self-reset for the next step (stream-ordered)
-        if (a.step_word) *a.step_word = t + (unsigned long long)nsteps;
-        if (a.signal_lo) st_release_sys_u64(a.signal_lo, a.signal_value);
-        if (a.signal_hi) st_release_sys_u64(a.signal_hi, a.signal_value);
+    if (sig_hi && atomicAdd(&a.side_counter[1], 1u) == a.hi_ctas - 1) {
+        __threadfence_system();
+        a.side_counter[1] = 0u;
+        st_release_sys_u64(a.signal_hi, a.signal_value);
+    }
+    if (a.step_word) {
+        const unsigned int nblocks = gridDim.x * gridDim.y * gridDim.z;
+        if (atomicAdd(a.done_counter, 1u) == nblocks - 1) {
+            *a.done_counter = 0u;
+            *a.step_word = t + (unsigned long long)nsteps;
+        }
     }
 }
 

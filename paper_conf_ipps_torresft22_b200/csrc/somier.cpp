@@ -82,6 +82,7 @@ struct Chunk {
     unsigned long long* flags() const { return (unsigned long long*)((char*)mem() + off_flags); }
     unsigned int* counter() const { return (unsigned int*)((char*)mem() + off_counter); }
     unsigned long long* step_word() const { return (unsigned long long*)((char*)mem() + off_counter + 8); }
+    unsigned int* side_counter() const { return (unsigned int*)((char*)mem() + off_counter + 16); }  // [2]
     paper::StatsAccum* acc_static() const { return acc() + paper::kStatsRing; }
 };
 
@@ -311,7 +312,7 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     c.off_v1 = h->tb2 ? c.off_v + vb : c.off_v;
     c.off_acc = c.off_v + (h->tb2 ? 2 : 1) * vb;
     c.off_flags = c.off_acc + (paper::kStatsRing + 2) * sizeof(paper::StatsAccum);
-    c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);  // counter (4 B, padded to 8) + step word
+    c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);  // counter (4 B, padded to 8), step word, side counters[2]
     c.bytes = round_up(c.off_counter + 64, 4096);
     CUDA_TRY(h, cudaSetDevice(c.device));
     CUDA_TRY(h, cudaMalloc(&c.base, c.bytes));
@@ -900,6 +901,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.signal_hi = fr ? &right->flags()[0] : nullptr;
             a.signal_value = (unsigned long long)(t + 1);
             a.done_counter = me.counter();
+            a.side_counter = me.side_counter();
             a.tmap_x_cur = &me.tmap_x[cur];
             a.tmap_v = &me.tmap_v[vb];
             a.tmap_x2_cur = &me.tmap_x2[cur];
@@ -989,6 +991,7 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         a.signal_hi = fr ? &right->flags()[0] : nullptr;
         a.signal_value = (unsigned long long)t_end;
         a.done_counter = me.counter();
+        a.side_counter = me.side_counter();
         if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
         CUDA_TRY(h, paper::launch_k1_tb2(a, o, h->unit_mass(), st));
         if (h->timing) {

@@ -9,9 +9,9 @@ This package is the Python binding (argument marshalling only).
 from . import _native, capi
 from ._native import K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2, STATS_HISTORY, SpreadError
 from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
-from .spread import Chunk, Spread
+from .spread import Chunk, Spread, SpreadTasks
 
-__all__ = ["capi", "Spread", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats", "combine_stats", "SpreadError",
+__all__ = ["capi", "Spread", "SpreadTasks", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats", "combine_stats", "SpreadError",
            "K1_AUTO", "K1_DIRECT", "K1_MARCH", "K1_MARCH2", "K1_TB2", "STATS_HISTORY", "version"]
 
 

@@ -70,6 +70,11 @@ class somier_timing_t(ctypes.Structure):
     ]
 
 
+class spread_task_record(ctypes.Structure):
+    _fields_ = [("chunk", ctypes.c_int64), ("kind", ctypes.c_int32), ("pad", ctypes.c_int32),
+                ("start_ms", ctypes.c_double), ("end_ms", ctypes.c_double)]
+
+
 class spread_reduce_result(ctypes.Structure):
     _fields_ = [
         ("value", ctypes.c_double),
@@ -107,6 +112,15 @@ SIGNATURES = [
     ("spread_stencil3", ctypes.c_int, [_VP, _DP, _DP, ctypes.c_int64]),
     ("spread_reduce", ctypes.c_int, [_VP, _DP, ctypes.c_int64, ctypes.c_int, ctypes.c_int,
                                      ctypes.POINTER(spread_reduce_result)]),
+    ("spread_tasks_create", ctypes.c_int, [_VP, _IP, ctypes.POINTER(_VP)]),
+    ("spread_enter_data", ctypes.c_int, [_VP, _DP, ctypes.c_int64, spread_map, ctypes.POINTER(_VP)]),
+    ("spread_task_stencil3", ctypes.c_int, [_VP, _VP, _VP]),
+    ("spread_task_reduce", ctypes.c_int, [_VP, _VP, ctypes.c_int, ctypes.POINTER(spread_reduce_result)]),
+    ("spread_exit_data", ctypes.c_int, [_VP, _VP, _DP]),
+    ("spread_taskwait", ctypes.c_int, [_VP]),
+    ("spread_tasks_set_trace", ctypes.c_int, [_VP, ctypes.c_int]),
+    ("spread_tasks_trace", ctypes.c_int, [_VP, ctypes.POINTER(spread_task_record), ctypes.c_int64, _I64P]),
+    ("spread_tasks_destroy", ctypes.c_int, [_VP]),
     ("spread_last_error", ctypes.c_char_p, []),
     ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),

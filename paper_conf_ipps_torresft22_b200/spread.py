@@ -2,7 +2,7 @@
 from __future__ import annotations
 
 import ctypes
-from typing import List, NamedTuple, Sequence
+from typing import List, NamedTuple, Optional, Sequence
 
 from . import _native as N
 
@@ -142,3 +142,94 @@ class Spread:
         N.check(N.lib().spread_map_extent(self._h, c, m, array_len, ctypes.byref(first), ctypes.byref(ln)),
                 "spread_map_extent")
         return first.value, ln.value
+
+
+class SpreadTasks:
+    """Chunk-level `depend` between spread constructs (include/spread.h,
+    PAPER.md:746-767): every method enqueues per chunk and returns (nowait);
+    taskwait() is the only barrier. Host arrays passed to enter / exit must stay
+    alive (and unchanged / unread) until the next taskwait()."""
+
+    KINDS = {0: "enter", 1: "stencil3", 2: "reduce", 3: "exit"}
+
+    def __init__(self, spread: Spread, cuda_devices: Optional[Sequence[int]] = None):
+        self.spread = spread
+        h = ctypes.c_void_p()
+        arr = None if cuda_devices is None else (ctypes.c_int * len(cuda_devices))(*cuda_devices)
+        N.check(N.lib().spread_tasks_create(spread.handle, arr, ctypes.byref(h)), "spread_tasks_create")
+        self._h = h
+        self._keep = []      # host arrays in flight
+        self._results = []   # (spread_reduce_result, [value slot])
+
+    def close(self) -> None:
+        if getattr(self, "_h", None):
+            N.lib().spread_tasks_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def enter(self, A=None, n: Optional[int] = None, lo_halo: int = 0, hi_halo: int = 0):
+        """target enter data spread map(to: A[start-lo : size+lo+hi]) (A given) or
+        map(alloc: ...) (A None, n elements) depend(out: A[start:size]) nowait."""
+        import numpy as np
+
+        if A is not None:
+            A = np.ascontiguousarray(A, dtype=np.float64)
+            self._keep.append(A)
+            n = A.size
+            ptr = A.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+            m = N.spread_map(N.MAP_TO, lo_halo, hi_halo)
+        else:
+            ptr = None
+            m = N.spread_map(N.MAP_ALLOC, lo_halo, hi_halo)
+        d = ctypes.c_void_p()
+        N.check(N.lib().spread_enter_data(self._h, ptr, int(n), m, ctypes.byref(d)), "spread_enter_data")
+        return d
+
+    def stencil3(self, a, b) -> None:
+        """target spread depend(in: A[start-1:size+2]) depend(out: B[start:size]) nowait: B[i] = A[i-1]+A[i]+A[i+1]."""
+        N.check(N.lib().spread_task_stencil3(self._h, a, b), "spread_task_stencil3")
+
+    def reduce_sum(self, a, scale_exp: int = 60):
+        """target spread depend(in: A[start:size]) reduction(+) nowait (exact sum);
+        returns a result object, filled by the next taskwait()."""
+        r = N.spread_reduce_result()
+        N.check(N.lib().spread_task_reduce(self._h, a, int(scale_exp), ctypes.byref(r)), "spread_task_reduce")
+        self._results.append(r)
+        return r
+
+    def exit(self, a, B) -> None:
+        """target exit data spread map(from: A[start:size]) depend(in: A[start:size]) nowait, into B."""
+        import numpy as np
+
+        if not (isinstance(B, np.ndarray) and B.dtype == np.float64 and B.flags["C_CONTIGUOUS"]):
+            raise TypeError("exit: B must be a C-contiguous float64 array")
+        self._keep.append(B)
+        N.check(N.lib().spread_exit_data(self._h, a, B.ctypes.data_as(ctypes.POINTER(ctypes.c_double))),
+                "spread_exit_data")
+
+    def taskwait(self) -> None:
+        N.check(N.lib().spread_taskwait(self._h), "spread_taskwait")
+        self._keep = []
+
+    def set_trace(self, on: bool = True) -> None:
+        N.check(N.lib().spread_tasks_set_trace(self._h, 1 if on else 0), "spread_tasks_set_trace")
+
+    def trace(self) -> list:
+        """[(chunk, kind, start_ms, end_ms)] of every traced chunk task (waits first)."""
+        cnt = ctypes.c_int64()
+        N.check(N.lib().spread_tasks_trace(self._h, None, 0, ctypes.byref(cnt)), "spread_tasks_trace")
+        recs = (N.spread_task_record * max(1, cnt.value))()
+        N.check(N.lib().spread_tasks_trace(self._h, recs, cnt.value, ctypes.byref(cnt)), "spread_tasks_trace")
+        return [(r.chunk, self.KINDS[r.kind], r.start_ms, r.end_ms) for r in recs[:cnt.value]]
+

@@ -378,6 +378,16 @@ spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64
  * somier_stream_run2. */
 spread_status somier_stream_traffic2(somier_stream_t h, int64_t* h2d_bytes, int64_t* d2h_bytes);
 
+/* Chunk tasks (one chunk mapped in, stepped, mapped out) each list position has
+ * run since the handle was created; counts[] holds one entry per position. With
+ * spread_schedule(dynamic) these show how the chunks were shared out. */
+spread_status somier_stream_chunk_counts(somier_stream_t h, int64_t* counts);
+
+/* Test hook: every chunk task of list position device_pos first spins >= ns
+ * nanoseconds on that device (a deliberately slower device, to exercise the
+ * dynamic schedule); 0 switches it off. */
+spread_status somier_stream_set_delay(somier_stream_t h, int device_pos, int64_t ns);
+
 spread_status somier_stream_destroy(somier_stream_t h);
 
 #ifdef __cplusplus

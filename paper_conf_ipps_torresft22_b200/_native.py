@@ -16,6 +16,8 @@ LIB_PATH = os.environ.get("SOMIER_LIB") or os.path.join(_HERE, "libsomier.so")
 
 # spread_status
 OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
+# spread_sched
+SCHED_STATIC, SCHED_DYNAMIC = 0, 1
 # spread_map_type
 MAP_ALLOC, MAP_TO, MAP_FROM, MAP_TOFROM = 0, 1, 2, 3
 # somier_kernel
@@ -112,6 +114,7 @@ SIGNATURES = [
     ("spread_stencil3", ctypes.c_int, [_VP, _DP, _DP, ctypes.c_int64]),
     ("spread_reduce", ctypes.c_int, [_VP, _DP, ctypes.c_int64, ctypes.c_int, ctypes.c_int,
                                      ctypes.POINTER(spread_reduce_result)]),
+    ("spread_schedule_kind", ctypes.c_int, [_VP, _IP]),
     ("spread_tasks_create", ctypes.c_int, [_VP, _IP, ctypes.POINTER(_VP)]),
     ("spread_enter_data", ctypes.c_int, [_VP, _DP, ctypes.c_int64, spread_map, ctypes.POINTER(_VP)]),
     ("spread_task_stencil3", ctypes.c_int, [_VP, _VP, _VP]),
@@ -161,6 +164,8 @@ SIGNATURES = [
     ("somier_stream_run_blocked", ctypes.c_int,
      [_VP] + [_DP] * 12 + [ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
     ("somier_stream_traffic_blocked", ctypes.c_int, [_VP, ctypes.c_int64, _I64P, _I64P]),
+    ("somier_stream_chunk_counts", ctypes.c_int, [_VP, _I64P]),
+    ("somier_stream_set_delay", ctypes.c_int, [_VP, ctypes.c_int, ctypes.c_int64]),
     ("somier_stream_destroy", ctypes.c_int, [_VP]),
 ]
 

@@ -117,6 +117,9 @@ struct Tb2Out {
 };
 cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
+// Test hook (somier_stream_set_delay): one CTA that spins ~ns nanoseconds on the
+// stream, emulating a slower device.
+cudaError_t launch_delay(int64_t ns, cudaStream_t stream);
 // Stats of planes [p0, p0+np) of an X slab (plane index inside the slab) and,
 // if v != null, of V planes [p0-1, ...) (V has no halo planes).
 // k_interior_only: skip the k-face columns (k = 0, n2-1).

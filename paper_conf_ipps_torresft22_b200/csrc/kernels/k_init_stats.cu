@@ -118,4 +118,18 @@ cudaError_t launch_stats(const double* x_slab, const double* v_slab, const SlabG
     return cudaGetLastError();
 }
 
+namespace {
+__global__ void delay_kernel(long long ns) {
+    const long long t0 = clock64();
+    const long long cycles = ns * 2;  // ~2 GHz SM clock: a lower bound on the delay
+    while (clock64() - t0 < cycles) __nanosleep(1000);
+}
+}  // namespace
+
+cudaError_t launch_delay(int64_t ns, cudaStream_t stream) {
+    if (ns <= 0) return cudaSuccess;
+    delay_kernel<<<1, 32, 0, stream>>>((long long)ns);
+    return cudaGetLastError();
+}
+
 }  // namespace paper

@@ -366,6 +366,9 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
     if (!out) PAPER_FAIL(SPREAD_EINVAL, "somier_init: out is NULL");
     *out = nullptr;
     if (!s) PAPER_FAIL(SPREAD_EINVAL, "somier_init: spread is NULL");
+    if (s->dynamic)
+        PAPER_FAIL(SPREAD_ENOTSUP, "somier_init: resident chunks are bound to their devices; the dynamic schedule "
+                   "applies to the host-streamed mode (somier_stream_create)");
     spread_status st = check_params(p);
     if (st != SPREAD_OK) return st;
     // Coherence of the spread with the loop it is applied to (the paper leaves

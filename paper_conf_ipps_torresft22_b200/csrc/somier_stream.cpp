@@ -14,6 +14,8 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <thread>
+#include <utility>
 #include <vector>
 
 #include "driver_util.hpp"
@@ -44,10 +46,39 @@ struct Slot {
 // D2H(c+1, t) (it reads the halo planes and V they wrote); D2H(c, t+1), which
 // overwrites X_t[c], depends on H2D(c-1, t) and H2D(c+1, t) (they read its
 // edge planes as halos). No other ordering between steps is needed.
+// Events are per list position (created on first use on that position's
+// device, since an event is recorded on its own device's streams): under the
+// dynamic schedule a chunk moves between devices from step to step; *_at
+// remembers which position recorded the last one.
 struct ChunkEvents {
-    cudaEvent_t h2d[2] = {nullptr, nullptr};
-    cudaEvent_t d2h[2] = {nullptr, nullptr};
+    std::vector<cudaEvent_t> h2d[2], d2h[2];
+    int h2d_at[2] = {-1, -1}, d2h_at[2] = {-1, -1};
+    cudaEvent_t last_h2d(int par) const { return h2d_at[par] < 0 ? nullptr : h2d[par][(size_t)h2d_at[par]]; }
+    cudaEvent_t last_d2h(int par) const { return d2h_at[par] < 0 ? nullptr : d2h[par][(size_t)d2h_at[par]]; }
 };
+
+// record a chunk event of list position pos (the current device) on stream st
+cudaError_t record_at(std::vector<cudaEvent_t>& v, int& at, int pos, cudaStream_t st) {
+    if (v.size() <= (size_t)pos) v.resize((size_t)pos + 1, nullptr);
+    if (!v[(size_t)pos]) {
+        cudaError_t e = cudaEventCreateWithFlags(&v[(size_t)pos], cudaEventDisableTiming);
+        if (e != cudaSuccess) return e;
+    }
+    at = pos;
+    return cudaEventRecord(v[(size_t)pos], st);
+}
+
+cudaError_t wait_ev(cudaStream_t st, cudaEvent_t ev) { return ev ? cudaStreamWaitEvent(st, ev, 0) : cudaSuccess; }
+
+// spread_schedule(dynamic) is a test of the slot ring's next slot: free once
+// its previous chunk's map(from) completed
+template <class SlotT>
+bool slot_free(const SlotT& sl) {
+    if (!sl.used) return true;
+    const cudaError_t e = cudaEventQuery(sl.d2h_done);
+    if (e == cudaErrorNotReady) cudaGetLastError();  // not an error: clear it
+    return e == cudaSuccess;
+}
 
 // Device buffers of a blocked round trip (somier_stream_run_blocked): the
 // chunk's X_t planes [start-s-1, start+size+s+1) and V_t planes
@@ -70,7 +101,11 @@ struct Dev {
     // planes, K1_TB2's k-face columns), then one slot per step of the run
     void* acc_base = nullptr;
     int64_t acc_steps = 0;
-    std::vector<int64_t> chunks;
+    std::vector<int64_t> chunks;  // the static round-robin's chunks (generate; slot sizing)
+    bool active = false;          // takes chunks (static: has some; dynamic: every position)
+    size_t next_slot = 0;         // dynamic schedule: the slot ring's next slot
+    int64_t chunks_run = 0;       // chunk tasks this position ran (somier_stream_chunk_counts)
+    int64_t delay_ns = 0;         // test hook: extra device time per chunk (somier_stream_set_delay)
     paper::StatsAccum* acc(int64_t t) const { return (paper::StatsAccum*)acc_base + 1 + t; }
     paper::StatsAccum* acc_static() const { return (paper::StatsAccum*)acc_base; }
 };
@@ -91,6 +126,37 @@ struct somier_stream_s {
 };
 
 namespace {
+
+// The position and buffer slot chunk c runs on. Static schedule: its
+// round-robin position, slot (c / p) mod buffers. Dynamic schedule
+// (PAPER.md:771, 775): the first position -- polled from c's round-robin one --
+// whose next slot is free, i.e. whichever device frees a slot first; the host
+// thread waits (polling the slots' completion events) while none is free.
+template <class SlotT>
+std::pair<Dev*, SlotT*> place_chunk(somier_stream_s* h, int64_t c, std::vector<SlotT> Dev::*slots) {
+    const paper::ChunkInfo ci = h->spread.chunk_info(c);
+    const size_t np = h->devs.size();
+    if (!h->spread.dynamic) {
+        Dev& d = h->devs[(size_t)ci.pos];
+        const size_t m = (size_t)(c / (int64_t)np);  // index of c among its device's chunks
+        d.chunks_run++;
+        return {&d, &(d.*slots)[m % (d.*slots).size()]};
+    }
+    for (;;) {
+        for (size_t k = 0; k < np; k++) {
+            Dev& d = h->devs[((size_t)ci.pos + k) % np];
+            auto& v = d.*slots;
+            if (v.empty()) continue;
+            SlotT& sl = v[d.next_slot % v.size()];
+            if (slot_free(sl)) {
+                d.next_slot++;
+                d.chunks_run++;
+                return {&d, &sl};
+            }
+        }
+        std::this_thread::yield();
+    }
+}
 
 spread_status sfail(somier_stream_t h, cudaError_t e, const char* what) {
     std::string msg = std::string(what) + ": " + cudaGetErrorString(e);
@@ -130,8 +196,9 @@ void destroy_all(somier_stream_t h) {
     }
     for (auto& ce : h->ev)
         for (int q = 0; q < 2; q++) {
-            if (ce.h2d[q]) cudaEventDestroy(ce.h2d[q]);
-            if (ce.d2h[q]) cudaEventDestroy(ce.d2h[q]);
+            for (auto* v : {&ce.h2d[q], &ce.d2h[q]})
+                for (cudaEvent_t e : *v)
+                    if (e) cudaEventDestroy(e);
         }
     h->ev.clear();
     h->devs.clear();
@@ -158,7 +225,7 @@ spread_status sync_devs(somier_stream_t h) {
 // Grow every device's per-step stats history to hold `nsteps` steps.
 spread_status ensure_acc(somier_stream_t h, int64_t nsteps) {
     for (auto& d : h->devs) {
-        if (d.chunks.empty() || d.acc_steps >= nsteps) continue;
+        if (!d.active || d.acc_steps >= nsteps) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaDeviceSynchronize());
         S_TRY(h, cudaFree(d.acc_base));
@@ -181,9 +248,9 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
     const int par = (int)(t & 1), prev = par ^ 1;
     for (int64_t c = 0; c < nch; c++) {
         const paper::ChunkInfo ci = h->spread.chunk_info(c);
-        Dev& d = h->devs[ci.pos];
-        const size_t m = (size_t)(c / (int64_t)h->devs.size());  // index of c among its device's chunks
-        Slot& sl = d.slots[m % d.slots.size()];
+        const auto pl = place_chunk(h, c, &Dev::slots);
+        Dev& d = *pl.first;
+        Slot& sl = *pl.second;
         const paper::SlabGeom g = geom_of(h, ci);
         const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
         ChunkEvents& ev = h->ev[(size_t)c];
@@ -192,16 +259,16 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
         if (chained)
             for (int64_t nb = std::max<int64_t>(0, c - 1); nb <= std::min<int64_t>(nch - 1, c + 1); nb++)
-                S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
+                S_TRY(h, wait_ev(d.s_h2d, h->ev[(size_t)nb].last_d2h(prev)));
         for (int q = 0; q < 3; q++) {
             S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, 0, X[q], ci.start - 1, ci.size + 2,
                                              cudaMemcpyHostToDevice, d.s_h2d));
             S_TRY(h, paper::copy_slab_planes(g, sl.v, q, 0, V[q], ci.start, ci.size, cudaMemcpyHostToDevice,
                                              d.s_h2d));
         }
-        S_TRY(h, cudaEventRecord(ev.h2d[par], d.s_h2d));
+        S_TRY(h, record_at(ev.h2d[par], ev.h2d_at[par], d.pos, d.s_h2d));
         // the fused step (forces, accelerations, velocities, positions, centers)
-        S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
+        S_TRY(h, wait_ev(d.s_comp, ev.last_h2d(par)));
         paper::StatsAccum* acc = d.acc(t);
         if (t == 0) {  // the fixed end planes, once per run (they never move)
             if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, d.acc_static(), d.s_comp));
@@ -224,6 +291,7 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         a.tmap_v2 = &sl.tmap_v2;
         a.write_fixed = 1;
         const paper::K1Variant var = paper::k1_variant(h->p.kernel);
+        S_TRY(h, paper::launch_delay(d.delay_ns, d.s_comp));
         S_TRY(h, paper::launch_k1(var, a, h->p.mass == 1.0, d.s_comp));
         h->launches++;
         S_TRY(h, cudaEventRecord(sl.comp_done, d.s_comp));
@@ -232,8 +300,8 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         // the previous step read as halos
         S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
         if (chained) {
-            if (c > 0) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)c - 1].h2d[prev], 0));
-            if (c + 1 < nch) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)c + 1].h2d[prev], 0));
+            if (c > 0) S_TRY(h, wait_ev(d.s_d2h, h->ev[(size_t)c - 1].last_h2d(prev)));
+            if (c + 1 < nch) S_TRY(h, wait_ev(d.s_d2h, h->ev[(size_t)c + 1].last_h2d(prev)));
         }
         for (int q = 0; q < 3; q++) {
             S_TRY(h, paper::copy_slab_planes(g, sl.x_out, q, 1, XN[q], ci.start, ci.size, cudaMemcpyDeviceToHost,
@@ -246,7 +314,7 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
                 S_TRY(h, paper::copy_slab_planes(g, sl.x_in, q, ci.size + 1, XN[q], n0 - 1, 1,
                                                  cudaMemcpyDeviceToHost, d.s_d2h));
         }
-        S_TRY(h, cudaEventRecord(ev.d2h[par], d.s_d2h));
+        S_TRY(h, record_at(ev.d2h[par], ev.d2h_at[par], d.pos, d.s_d2h));
         S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
         sl.used = true;
     }
@@ -260,7 +328,7 @@ spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, s
     std::vector<unsigned long long> vmax2((size_t)n, 0);
     std::vector<paper::StatsAccum> acc((size_t)n + 1);
     for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
+        if (!d.active) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaMemcpy(acc.data(), d.acc_base, acc.size() * sizeof(paper::StatsAccum), cudaMemcpyDeviceToHost));
         for (int64_t t = 0; t < n; t++)
@@ -296,7 +364,7 @@ spread_status ensure_flat(somier_stream_t h) {
     for (auto& d : h->devs) {
         bool missing = false;
         for (auto& sl : d.slots) missing = missing || !sl.base;
-        if (d.chunks.empty() || !missing) continue;
+        if (!d.active || !missing) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaDeviceSynchronize());
         release_deep(d);
@@ -327,7 +395,7 @@ spread_status ensure_flat(somier_stream_t h) {
 spread_status ensure_deep(somier_stream_t h, int64_t planes) {
     const size_t plane = (size_t)h->geom.plane_stride() * sizeof(double);
     for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
+        if (!d.active) continue;
         S_TRY(h, cudaSetDevice(d.device));
         if (!d.deep.empty() && d.deep[0].base && d.deep[0].planes >= planes) continue;
         S_TRY(h, cudaDeviceSynchronize());
@@ -387,9 +455,9 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
     const int64_t nl = s / 2 + (s & 1);
     for (int64_t c = 0; c < nch; c++) {
         const paper::ChunkInfo ci = h->spread.chunk_info(c);
-        Dev& d = h->devs[ci.pos];
-        const size_t m = (size_t)(c / (int64_t)h->devs.size());
-        DeepSlot& sl = d.deep[m % d.deep.size()];
+        const auto pl = place_chunk(h, c, &Dev::deep);
+        Dev& d = *pl.first;
+        DeepSlot& sl = *pl.second;
         const bool first = ci.start == 1, last = ci.start + ci.size == n0 - 1;
         ChunkEvents& ev = h->ev[(size_t)c];
         int64_t c_lo, c_hi, w_lo, w_hi;
@@ -403,7 +471,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
         if (sl.used) S_TRY(h, cudaStreamWaitEvent(d.s_h2d, sl.d2h_done, 0));
         if (chained)
             for (int64_t nb = c_lo; nb <= c_hi; nb++)
-                S_TRY(h, cudaStreamWaitEvent(d.s_h2d, h->ev[(size_t)nb].d2h[prev], 0));
+                S_TRY(h, wait_ev(d.s_h2d, h->ev[(size_t)nb].last_d2h(prev)));
         const int64_t xlo = std::max<int64_t>(0, ci.start - s), xhi = std::min<int64_t>(n0, ci.start + ci.size + s);
         // V_t is needed one plane less deep than X_t, but at least one plane
         // (a one-step launch reads the ring plane; the first chunk maps the face plane)
@@ -416,8 +484,8 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             S_TRY(h, paper::copy_slab_planes(g, sl.va, q, vlo - v0, V[q], vlo, vhi - vlo,
                                              cudaMemcpyHostToDevice, d.s_h2d));
         }
-        S_TRY(h, cudaEventRecord(ev.h2d[par], d.s_h2d));
-        S_TRY(h, cudaStreamWaitEvent(d.s_comp, ev.h2d[par], 0));
+        S_TRY(h, record_at(ev.h2d[par], ev.h2d_at[par], d.pos, d.s_h2d));
+        S_TRY(h, wait_ev(d.s_comp, ev.last_h2d(par)));
         // the fixed face nodes of every output plane (K1_TB2 writes the moving nodes only)
         S_TRY(h, cudaMemcpyAsync(sl.xb + (xlo - x0) * ps, sl.xa + (xlo - x0) * ps,
                                  (size_t)((xhi - xlo) * ps) * sizeof(double), cudaMemcpyDeviceToDevice, d.s_comp));
@@ -427,6 +495,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             if (last) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, ci.size + 1, 1, d.acc_static(), d.s_comp));
             S_TRY(h, paper::launch_kface_stats(xv_one, g, 1, ci.size, d.acc_static(), d.s_comp));
         }
+        S_TRY(h, paper::launch_delay(d.delay_ns, d.s_comp));
         int64_t remaining = s, done = 0;
         double *xin = sl.xa, *xout = sl.xb, *vin = sl.va, *vout = sl.vb;
         for (int64_t j = 0; j < nl; j++) {
@@ -474,7 +543,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
         S_TRY(h, cudaStreamWaitEvent(d.s_d2h, sl.comp_done, 0));
         if (chained)
             for (int64_t nb = w_lo; nb <= w_hi; nb++)
-                if (nb != c) S_TRY(h, cudaStreamWaitEvent(d.s_d2h, h->ev[(size_t)nb].h2d[prev], 0));
+                if (nb != c) S_TRY(h, wait_ev(d.s_d2h, h->ev[(size_t)nb].last_h2d(prev)));
         // after the last launch the state is in (xin, vin)
         for (int q = 0; q < 3; q++) {
             S_TRY(h, paper::copy_slab_planes(g, xin, q, ci.start - x0, XN[q], ci.start, ci.size,
@@ -493,7 +562,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
                                                  cudaMemcpyDeviceToHost, d.s_d2h));
             }
         }
-        S_TRY(h, cudaEventRecord(ev.d2h[par], d.s_d2h));
+        S_TRY(h, record_at(ev.d2h[par], ev.d2h_at[par], d.pos, d.s_d2h));
         S_TRY(h, cudaEventRecord(sl.d2h_done, d.s_d2h));
         sl.used = true;
     }
@@ -512,7 +581,7 @@ spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* 
     st = ensure_deep(h, h->max_chunk + 2 * s + 2);
     if (st != SPREAD_OK) return st;
     for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
+        if (!d.active) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaMemsetAsync(d.acc_base, 0, (1 + (size_t)nsteps) * sizeof(paper::StatsAccum), d.s_comp));
     }
@@ -540,7 +609,7 @@ spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[
     st = ensure_acc(h, nsteps);
     if (st != SPREAD_OK) return st;
     for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
+        if (!d.active) continue;
         S_TRY(h, cudaSetDevice(d.device));
         S_TRY(h, cudaMemsetAsync(d.acc_base, 0, (1 + (size_t)nsteps) * sizeof(paper::StatsAccum), d.s_comp));
     }
@@ -596,6 +665,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         h->devs[q].device = cuda_devices ? cuda_devices[q] : s->devices[q];
     }
     for (int64_t c = 0; c < s->nchunks; c++) h->devs[s->chunk_info(c).pos].chunks.push_back(c);
+    for (auto& d : h->devs) d.active = !d.chunks.empty() || (s->dynamic && s->nchunks > 0);
 
     auto fail = [&](spread_status code) {
         std::string msg = paper::last_error();
@@ -605,7 +675,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         return code;
     };
     for (auto& d : h->devs) {
-        if (d.chunks.empty()) continue;
+        if (!d.active) continue;
         if ((e = cudaSetDevice(d.device)) != cudaSuccess) return fail(sfail(h, e, "cudaSetDevice"));
         for (cudaStream_t* ps : {&d.s_h2d, &d.s_comp, &d.s_d2h})
             if ((e = cudaStreamCreateWithFlags(ps, cudaStreamNonBlocking)) != cudaSuccess)
@@ -613,7 +683,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
         if ((e = cudaMalloc(&d.acc_base, (1 + kAccSteps) * sizeof(paper::StatsAccum))) != cudaSuccess)
             return fail(sfail(h, e, "cudaMalloc(stats)"));
         d.acc_steps = kAccSteps;
-        d.slots.resize((size_t)std::min<int64_t>(buffers, (int64_t)d.chunks.size()));
+        d.slots.resize((size_t)std::min<int64_t>(buffers, s->dynamic ? s->nchunks : (int64_t)d.chunks.size()));
         for (auto& sl : d.slots)
             for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
                 if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
@@ -621,15 +691,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
     }
     st = ensure_flat(h);
     if (st != SPREAD_OK) return fail(st);
-    h->ev.resize((size_t)s->nchunks);
-    for (int64_t c = 0; c < s->nchunks; c++) {
-        if ((e = cudaSetDevice(h->devs[s->chunk_info(c).pos].device)) != cudaSuccess)
-            return fail(sfail(h, e, "cudaSetDevice"));
-        for (int q = 0; q < 2; q++)
-            for (cudaEvent_t* pe : {&h->ev[c].h2d[q], &h->ev[c].d2h[q]})
-                if ((e = cudaEventCreateWithFlags(pe, cudaEventDisableTiming)) != cudaSuccess)
-                    return fail(sfail(h, e, "cudaEventCreate"));
-    }
+    h->ev.resize((size_t)s->nchunks);  // events created on first use (record_at)
     *out = h;
     return SPREAD_OK;
 }
@@ -782,6 +844,19 @@ spread_status somier_stream_traffic(somier_stream_t h, int64_t* h2d_bytes, int64
     if (h2d_bytes) *h2d_bytes = in;
     if (d2h_bytes) *d2h_bytes = outb;
     if (launches) *launches = h->launches;
+    return SPREAD_OK;
+}
+
+spread_status somier_stream_set_delay(somier_stream_t h, int device_pos, int64_t ns) {
+    if (!h || device_pos < 0 || device_pos >= (int)h->devs.size() || ns < 0)
+        PAPER_FAIL(SPREAD_EINVAL, "somier_stream_set_delay: bad arguments");
+    h->devs[(size_t)device_pos].delay_ns = ns;
+    return SPREAD_OK;
+}
+
+spread_status somier_stream_chunk_counts(somier_stream_t h, int64_t* counts) {
+    if (!h || !counts) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_chunk_counts: NULL argument");
+    for (size_t q = 0; q < h->devs.size(); q++) counts[q] = h->devs[q].chunks_run;
     return SPREAD_OK;
 }
 

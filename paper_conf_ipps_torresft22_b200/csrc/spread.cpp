@@ -40,8 +40,9 @@ spread_status spread_create(const int* devices, int ndevices, int64_t range_star
                             spread_sched sched, int64_t chunk, spread_t* out) {
     if (!out) PAPER_FAIL(SPREAD_EINVAL, "spread_create: out is NULL");
     *out = nullptr;
-    if (sched != SPREAD_SCHED_STATIC)
-        PAPER_FAIL(SPREAD_ENOTSUP, "spread_create: only spread_schedule(static, chunk) exists (PAPER.md:101)");
+    if (sched != SPREAD_SCHED_STATIC && sched != SPREAD_SCHED_DYNAMIC)
+        PAPER_FAIL(SPREAD_ENOTSUP, "spread_create: unknown schedule %d (static: PAPER.md:101; dynamic: 771)",
+                   (int)sched);
     if (!devices || ndevices < 1) PAPER_FAIL(SPREAD_EINVAL, "spread_create: empty devices() list");
     if (range_len < 0) PAPER_FAIL(SPREAD_EINVAL, "spread_create: range length %lld < 0", (long long)range_len);
     if (chunk < 0) PAPER_FAIL(SPREAD_EINVAL, "spread_create: chunk %lld < 0", (long long)chunk);
@@ -56,6 +57,7 @@ spread_status spread_create(const int* devices, int ndevices, int64_t range_star
     s->devices.assign(devices, devices + ndevices);
     s->range_start = range_start;
     s->range_len = range_len;
+    s->dynamic = sched == SPREAD_SCHED_DYNAMIC;
     if (chunk == 0) chunk = range_len == 0 ? 1 : (range_len + ndevices - 1) / ndevices;
     s->chunk = chunk;
     s->nchunks = range_len == 0 ? 0 : (range_len + chunk - 1) / chunk;
@@ -162,6 +164,12 @@ spread_status spread_device(spread_t s, int pos, int* device_id) {
     if (pos < 0 || pos >= (int)s->devices.size())
         PAPER_FAIL(SPREAD_EINVAL, "spread_device: position %d outside the %zu-device list", pos, s->devices.size());
     if (device_id) *device_id = s->devices[pos];
+    return SPREAD_OK;
+}
+
+spread_status spread_schedule_kind(spread_t s, spread_sched* sched) {
+    if (!s || !sched) PAPER_FAIL(SPREAD_EINVAL, "spread_schedule_kind: NULL argument");
+    *sched = s->dynamic ? SPREAD_SCHED_DYNAMIC : SPREAD_SCHED_STATIC;
     return SPREAD_OK;
 }
 

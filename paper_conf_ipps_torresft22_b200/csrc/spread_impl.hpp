@@ -26,6 +26,7 @@ struct spread_s {
     int64_t range_len = 0;
     int64_t chunk = 1;      // regular: the chunk size; irregular: the largest chunk
     int64_t nchunks = 0;
+    bool dynamic = false;   // spread_schedule(dynamic, chunk): positions chosen at run time
     // Irregular static schedule (future work): chunk c covers
     // [range_start + offsets[c], range_start + offsets[c+1]). Empty = regular.
     std::vector<int64_t> offsets;

@@ -234,6 +234,9 @@ extern "C" {
 spread_status spread_tasks_create(spread_t s, const int* cuda_devices, spread_tasks_t* out) {
     if (!s || !out) PAPER_FAIL(SPREAD_EINVAL, "spread_tasks_create: NULL argument");
     *out = nullptr;
+    if (s->dynamic)
+        PAPER_FAIL(SPREAD_ENOTSUP, "spread_tasks_create: device-resident data is bound to its chunk's device "
+                   "(dynamic schedules apply to the host-array loops and the host-streamed Somier)");
     int ndev = 0;
     cudaError_t r = cudaGetDeviceCount(&ndev);
     if (r != cudaSuccess) PAPER_FAIL(SPREAD_ENODEV, "spread_tasks_create: no CUDA device (%s)", cudaGetErrorString(r));

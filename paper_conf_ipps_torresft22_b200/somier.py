@@ -374,6 +374,17 @@ class SomierStream:
                                                   out), "somier_stream_run_blocked")
         return [Stats.from_c(out[t]) for t in range(int(nsteps))] if stats else None
 
+    def chunk_counts(self) -> list:
+        """Chunk tasks each list position has run (somier_stream_chunk_counts)."""
+        n = len(self.spread.devices)
+        arr = (ctypes.c_int64 * n)()
+        N.check(N.lib().somier_stream_chunk_counts(self._h, arr), "somier_stream_chunk_counts")
+        return list(arr)
+
+    def set_delay(self, device_pos: int, ns: int) -> None:
+        """Test hook: position device_pos spins >= ns per chunk task (somier_stream_set_delay)."""
+        N.check(N.lib().somier_stream_set_delay(self._h, int(device_pos), int(ns)), "somier_stream_set_delay")
+
     def traffic_blocked(self, steps_per_trip: int):
         """Host<->device bytes of one trip of run_blocked with steps_per_trip steps."""
         a, b = ctypes.c_int64(), ctypes.c_int64()

@@ -102,6 +102,13 @@ class Spread:
     def chunks(self) -> List[Chunk]:
         return [self.chunk(c) for c in range(self.num_chunks)]
 
+    @property
+    def dynamic(self) -> bool:
+        """spread_schedule(dynamic, chunk): positions chosen at run time."""
+        v = ctypes.c_int()
+        N.check(N.lib().spread_schedule_kind(self._h, ctypes.byref(v)), "spread_schedule_kind")
+        return v.value == N.SCHED_DYNAMIC
+
     def chunk_of(self, iteration: int) -> int:
         v = ctypes.c_int64()
         N.check(N.lib().spread_chunk_of(self._h, iteration, ctypes.byref(v)), "spread_chunk_of")

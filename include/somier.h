@@ -71,8 +71,17 @@ typedef struct {
     double amplitude;    /* initial displacement amplitude a (|a| < rest_len / 2 recommended)  */
     uint64_t seed;       /* SplitMix64 seed of the initial displacement (reading S7)           */
     int32_t kernel;      /* somier_kernel                                                      */
-    int32_t reserved;    /* must be 0                                                          */
+    int32_t exchange;    /* somier_exchange: how boundary planes reach the neighbour chunks    */
 } somier_params;
+
+/* The halo exchange between chunks on different streams (devices / processes),
+ * SURVEY.md §8(b) `overlap` and §8(e): FUSED (default) -- K1 stores its boundary
+ * planes straight into the neighbours' halo slots (NVLink P2P / CUDA IPC) and
+ * its boundary CTAs publish the neighbours' flags; COPY -- the unfused route for
+ * A/B: K1 writes only its own slab, then the stream copies the boundary planes
+ * into the neighbours' halos (cudaMemcpyAsync over P2P / IPC) and writes the
+ * flags (cuStreamWriteValue64) after the whole kernel. Results are bit-identical. */
+typedef enum { SOMIER_EXCHANGE_FUSED = 0, SOMIER_EXCHANGE_COPY = 1 } somier_exchange;
 
 /* Stats of one step ("centers"). The exact partial sums are
  * exported so that per-process partials can be combined exactly. */

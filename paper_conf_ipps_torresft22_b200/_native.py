@@ -16,6 +16,8 @@ LIB_PATH = os.environ.get("SOMIER_LIB") or os.path.join(_HERE, "libsomier.so")
 
 # spread_status
 OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
+# somier_exchange
+EXCHANGE_FUSED, EXCHANGE_COPY = 0, 1
 # spread_sched
 SCHED_STATIC, SCHED_DYNAMIC = 0, 1
 # spread_map_type
@@ -46,7 +48,7 @@ class somier_params(ctypes.Structure):
         ("amplitude", ctypes.c_double),
         ("seed", ctypes.c_uint64),
         ("kernel", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("exchange", ctypes.c_int32),
     ]
 
 

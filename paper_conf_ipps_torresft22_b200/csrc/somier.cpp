@@ -31,6 +31,7 @@ constexpr uint64_t kIpcMagic = 0x534f4d4945524950ull;  // "SOMIERIP"
 constexpr uint32_t kIpcVersion = 4;
 
 using PFN_waitValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+using PFN_writeValue64 = CUresult (*)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 using PFN_encodeTiled = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                      const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                      CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -143,6 +144,7 @@ struct somier_s {
     std::vector<DevCtx> devs;  // indexed by list position
     std::string sticky;        // first asynchronous CUDA error
     PFN_waitValue64 wait_value64 = nullptr;
+    PFN_writeValue64 write_value64 = nullptr;
     PFN_encodeTiled encode_tiled = nullptr;
     bool connected = true;
     // CUDA graph of an (even, odd) step pair, when every chunk is on one stream
@@ -205,6 +207,18 @@ spread_status timing_begin(somier_t h, int device, cudaStream_t st, somier_s::Ti
     return SPREAD_OK;
 }
 
+// SOMIER_EXCHANGE_COPY: publish the neighbours' flags once everything before
+// on the stream (the kernel, the halo copies) is done
+spread_status signal_after(somier_t h, cudaStream_t st, unsigned long long* lo, unsigned long long* hi,
+                           unsigned long long value) {
+    for (unsigned long long* f : {lo, hi}) {
+        if (!f) continue;
+        CUresult r = h->write_value64((CUstream)st, (CUdeviceptr)f, (cuuint64_t)value, CU_STREAM_WRITE_VALUE_DEFAULT);
+        if (r != CUDA_SUCCESS) PAPER_FAIL(SPREAD_ECUDA, "somier_step: cuStreamWriteValue64 failed (%d)", (int)r);
+    }
+    return SPREAD_OK;
+}
+
 spread_status check_params(const somier_params* p) {
     if (!p) PAPER_FAIL(SPREAD_EINVAL, "somier: params is NULL");
     for (int d = 0; d < 3; d++)
@@ -216,7 +230,8 @@ spread_status check_params(const somier_params* p) {
     if (!(p->dt > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: dt must be > 0");
     if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_TB2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown kernel %d", p->kernel);
-    if (p->reserved != 0) PAPER_FAIL(SPREAD_EINVAL, "somier: reserved field must be 0");
+    if (p->exchange != SOMIER_EXCHANGE_FUSED && p->exchange != SOMIER_EXCHANGE_COPY)
+        PAPER_FAIL(SPREAD_EINVAL, "somier: unknown exchange %d", p->exchange);
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
     if (n1 > 65535LL * 8 || n0 > 65535 + 2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: grid too large for the launch geometry");
@@ -241,6 +256,11 @@ spread_status load_driver_entry(somier_t h) {
     if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
         PAPER_FAIL(SPREAD_ECUDA, "somier: cuStreamWaitValue64 unavailable (%s)", cudaGetErrorString(e));
     h->wait_value64 = (PFN_waitValue64)fn;
+    fn = nullptr;
+    e = cudaGetDriverEntryPoint("cuStreamWriteValue64", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+        PAPER_FAIL(SPREAD_ECUDA, "somier: cuStreamWriteValue64 unavailable (%s)", cudaGetErrorString(e));
+    h->write_value64 = (PFN_writeValue64)fn;
     fn = nullptr;
     e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
     if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
@@ -891,8 +911,9 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.x_cur = me.xs(cur);
             a.x_nxt = me.xs(nxt);
             a.v = me.vs(vb);
-            a.lo_dst = left ? left->xs(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
-            a.hi_dst = right ? right->xs(nxt) : nullptr;
+            const bool fused = h->p.exchange == SOMIER_EXCHANGE_FUSED;
+            a.lo_dst = left && fused ? left->xs(nxt) + (left->size + 1) * h->geom.plane_stride() : nullptr;
+            a.hi_dst = right && fused ? right->xs(nxt) : nullptr;
             a.g = h->geom_of(me);
             a.K = h->p.k_spring;
             a.L = h->p.rest_len;
@@ -900,8 +921,8 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.dt = h->p.dt;
             a.step_word = me.step_word();  // the kernel takes its ring slots from the device step counter
             a.acc_ring = me.acc();
-            a.signal_lo = fl ? &left->flags()[1] : nullptr;
-            a.signal_hi = fr ? &right->flags()[0] : nullptr;
+            a.signal_lo = fl && fused ? &left->flags()[1] : nullptr;
+            a.signal_hi = fr && fused ? &right->flags()[0] : nullptr;
             a.signal_value = (unsigned long long)(t + 1);
             a.done_counter = me.counter();
             a.side_counter = me.side_counter();
@@ -912,6 +933,21 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.pdl = h->pdl && !h->timing ? 1 : 0;
             if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
+            if (!fused) {
+                // SOMIER_EXCHANGE_COPY: the boundary planes of X_{t+1} into the
+                // neighbours' halo planes after the kernel, then their flags
+                const int64_t ps = h->geom.plane_stride();
+                const size_t pb = (size_t)ps * sizeof(double);
+                if (left)
+                    CUDA_TRY(h, cudaMemcpyAsync(left->xs(nxt) + (left->size + 1) * ps, me.xs(nxt) + ps, pb,
+                                                cudaMemcpyDeviceToDevice, st));
+                if (right)
+                    CUDA_TRY(h, cudaMemcpyAsync(right->xs(nxt), me.xs(nxt) + me.size * ps, pb,
+                                                cudaMemcpyDeviceToDevice, st));
+                spread_status ss = signal_after(h, st, fl ? &left->flags()[1] : nullptr,
+                                                fr ? &right->flags()[0] : nullptr, (unsigned long long)(t + 1));
+                if (ss != SPREAD_OK) return ss;
+            }
             if (h->timing) {
                 CUDA_TRY(h, cudaEventRecord(tr.c, st));
                 h->trecs.push_back(tr);
@@ -982,21 +1018,44 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         // global i = start, start+1 (its raw planes size+2, size+3), V plane
         // of i = start (raw size+1); right X planes start+size-2, -1 (raw 0, 1),
         // V plane start+size-1 (raw 0)
-        if (left) {
+        const bool fused = h->p.exchange == SOMIER_EXCHANGE_FUSED;
+        if (left && fused) {
             a.lo_dst = left->x(cur ^ 1) + (left->size + 2) * ps;
             o.lo_vdst = left->v(vb ^ 1) + (left->size + 1) * ps;
         }
-        if (right) {
+        if (right && fused) {
             a.hi_dst = right->x(cur ^ 1);
             o.hi_vdst = right->v(vb ^ 1);
         }
-        a.signal_lo = fl ? &left->flags()[1] : nullptr;
-        a.signal_hi = fr ? &right->flags()[0] : nullptr;
+        a.signal_lo = fl && fused ? &left->flags()[1] : nullptr;
+        a.signal_hi = fr && fused ? &right->flags()[0] : nullptr;
         a.signal_value = (unsigned long long)t_end;
         a.done_counter = me.counter();
         a.side_counter = me.side_counter();
         if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
         CUDA_TRY(h, paper::launch_k1_tb2(a, o, h->unit_mass(), st));
+        if (!fused) {
+            // SOMIER_EXCHANGE_COPY: the first two X planes and the first V plane
+            // of the new state to the left neighbour's deep halo, the last two /
+            // last one to the right's (the planes the fused kernel stores), then
+            // the flags
+            const size_t pb = (size_t)ps * sizeof(double);
+            if (left) {
+                CUDA_TRY(h, cudaMemcpyAsync(left->x(cur ^ 1) + (left->size + 2) * ps, me.x(cur ^ 1) + 2 * ps, 2 * pb,
+                                            cudaMemcpyDeviceToDevice, st));
+                CUDA_TRY(h, cudaMemcpyAsync(left->v(vb ^ 1) + (left->size + 1) * ps, me.v(vb ^ 1) + ps, pb,
+                                            cudaMemcpyDeviceToDevice, st));
+            }
+            if (right) {
+                CUDA_TRY(h, cudaMemcpyAsync(right->x(cur ^ 1), me.x(cur ^ 1) + me.size * ps, 2 * pb,
+                                            cudaMemcpyDeviceToDevice, st));
+                CUDA_TRY(h, cudaMemcpyAsync(right->v(vb ^ 1), me.v(vb ^ 1) + me.size * ps, pb,
+                                            cudaMemcpyDeviceToDevice, st));
+            }
+            spread_status ss = signal_after(h, st, fl ? &left->flags()[1] : nullptr, fr ? &right->flags()[0] : nullptr,
+                                            (unsigned long long)t_end);
+            if (ss != SPREAD_OK) return ss;
+        }
         if (h->timing) {
             CUDA_TRY(h, cudaEventRecord(tr.c, st));
             h->trecs.push_back(tr);

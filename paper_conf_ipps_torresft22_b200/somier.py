@@ -28,13 +28,15 @@ class SomierParams:
     amplitude: float = 0.05
     seed: int = 42
     kernel: int = N.K1_AUTO
+    exchange: int = 0  # SOMIER_EXCHANGE_FUSED (0) or SOMIER_EXCHANGE_COPY (1)
 
     def c(self) -> N.somier_params:
         p = N.somier_params()
         for d in range(3):
             p.n[d] = int(self.n[d])
         p.spacing, p.rest_len, p.k_spring, p.mass = self.spacing, self.rest_len, self.k_spring, self.mass
-        p.dt, p.amplitude, p.seed, p.kernel, p.reserved = self.dt, self.amplitude, int(self.seed), int(self.kernel), 0
+        p.dt, p.amplitude, p.seed, p.kernel = self.dt, self.amplitude, int(self.seed), int(self.kernel)
+        p.exchange = int(self.exchange)
         return p
 
     @property

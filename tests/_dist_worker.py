@@ -118,7 +118,8 @@ def gpu_ipc(a):
     torch.cuda.set_device(0)
     n = tuple(a.n)
     kernel = int(os.environ.get("SOMIER_TEST_KERNEL", P.K1_AUTO))
-    params = P.SomierParams(n=n, seed=a.seed, kernel=kernel)
+    exchange = int(os.environ.get("SOMIER_TEST_EXCHANGE", P.EXCHANGE_FUSED))
+    params = P.SomierParams(n=n, seed=a.seed, kernel=kernel, exchange=exchange)
     s = PD.open_local(params, chunk=a.chunk, cuda_device=0)
     if kernel == P.K1_TB2:
         assert s.kernel_in_use == P.K1_TB2

@@ -26,13 +26,15 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _launch(mode, out, n, steps, chunk, seed=3, timeout=300, kernel=None):
+def _launch(mode, out, n, steps, chunk, seed=3, timeout=300, kernel=None, exchange=None):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=%d" % _free_port(), WORKER, mode, out,
            *map(str, n), str(steps), str(chunk), str(seed)]
     env = dict(os.environ, OMP_NUM_THREADS="1", PYTHONPATH=ROOT)
     if kernel is not None:
         env["SOMIER_TEST_KERNEL"] = str(kernel)
+    if exchange is not None:
+        env["SOMIER_TEST_EXCHANGE"] = str(exchange)
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout, env=env)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     return np.load(out)
@@ -65,4 +67,17 @@ def test_gpu_two_processes_ipc_fused_exchange(tmp_path, chunk, kernel):
         pytest.skip("no CUDA device")
     n, steps, seed = (20, 12, 40), 15, 4
     res = _launch("gpu-ipc", str(tmp_path / "g.npz"), n, steps, chunk, seed, timeout=600, kernel=kernel)
+    _check(res, n, steps, seed)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("kernel", [0, 4])
+def test_gpu_two_processes_ipc_copy_exchange(tmp_path, kernel):
+    """SOMIER_EXCHANGE_COPY across processes: cudaMemcpyAsync into the neighbour's
+    IPC-mapped halo, then cuStreamWriteValue64 of its flag."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    n, steps, seed = (20, 12, 40), 15, 4
+    res = _launch("gpu-ipc", str(tmp_path / "g.npz"), n, steps, 3, seed, timeout=600, kernel=kernel, exchange=1)
     _check(res, n, steps, seed)

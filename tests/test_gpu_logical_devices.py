@@ -23,9 +23,10 @@ def _need_gpu():
 @pytest.mark.parametrize("devices,chunk", [([0, 1], 0), ([0, 1, 2, 3], 0), ([3, 1, 0, 2], 3), ([5, 7], 2),
                                            ([0, 1, 2], 1)])
 @pytest.mark.parametrize("kernel", [P.K1_MARCH, P.K1_MARCH2, P.K1_DIRECT, P.K1_TB2])
-def test_logical_devices_bit_identical(devices, chunk, kernel):
+@pytest.mark.parametrize("exchange", [P.EXCHANGE_FUSED, P.EXCHANGE_COPY])
+def test_logical_devices_bit_identical(devices, chunk, kernel, exchange):
     n, steps = (22, 19, 45), 17
-    sp = P.SomierParams(n=n, seed=11, kernel=kernel)
+    sp = P.SomierParams(n=n, seed=11, kernel=kernel, exchange=exchange)
     spread = P.Spread(devices, 1, n[0] - 2, chunk=chunk)
     with P.Somier(spread, sp, cuda_devices=[0] * len(devices)) as s:
         s.step(5)

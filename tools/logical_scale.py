@@ -7,7 +7,7 @@ N = 1, 2, 4, 8 on the same GPU: the drop from N = 1 is what the chunking,
 deep-halo exchange and flag waits cost (the GPU's SMs are shared, so this is
 not a scaling measurement). Host wall clock around step(K) + sync.
 
-Usage: python tools/logical_scale.py [n] [steps]"""
+Usage: python tools/logical_scale.py [n] [steps] [exchange: fused|copy]"""
 import json
 import os
 import sys
@@ -21,11 +21,12 @@ import paper_conf_ipps_torresft22_b200 as P  # noqa: E402
 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 512
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 40
+exchange = {"fused": P.EXCHANGE_FUSED, "copy": P.EXCHANGE_COPY}[sys.argv[3] if len(sys.argv) > 3 else "fused"]
 torch.cuda.init()
 res = {}
 for rep in range(2):
     for L in (1, 2, 4, 8):
-        sp = P.SomierParams(n=[n, n, n], seed=42)
+        sp = P.SomierParams(n=[n, n, n], seed=42, exchange=exchange)
         with P.Somier(P.Spread(list(range(L)), 1, n - 2), sp, cuda_devices=[0] * L) as s:
             s.step(6)
             s.sync()
@@ -36,7 +37,7 @@ for rep in range(2):
             st = s.stats()
             v = (n - 2) ** 3 * steps / dt
             res.setdefault(L, []).append(v)
-            print(json.dumps({"n": n, "positions": L, "kernel": s.kernel_in_use, "launches_per_step": s.launches /
+            print(json.dumps({"n": n, "positions": L, "exchange": sys.argv[3] if len(sys.argv) > 3 else "fused", "kernel": s.kernel_in_use, "launches_per_step": s.launches /
                               max(1, s.step_count), "node_updates_per_s": v, "ms_per_step": dt / steps * 1e3,
                               "centre0": st.centre[0], "vmax": st.vmax}), flush=True)
 best1 = max(res[1])

@@ -435,13 +435,15 @@ def run_verify(a, n, params, world, rank, local, multi):
             "what": "nodes on both sides of every chunk border, bitwise vs the CPU oracle (light-cone windows)"}
 
 
-def pcie_rates(devices, nbytes=1 << 30):
+def pcie_rates(devices, nbytes=None):
     """Pinned host<->device copy rates (GB/s) of the GPUs in `devices` (distinct
     CUDA ordinals), all at once: H2D alone, D2H alone, and both directions
     concurrently -- the roofline of the host-streamed mode."""
     import torch
 
     devs = sorted(set(devices))
+    if nbytes is None:  # 1 GiB per buffer on one GPU, at least 256 MiB each on several
+        nbytes = max(1 << 28, (1 << 30) // len(devs))
     hs = [torch.empty(nbytes // 8, dtype=torch.float64, pin_memory=True) for _ in range(2 * len(devs))]
     ds = [torch.empty(nbytes // 8, dtype=torch.float64, device="cuda:%d" % d) for d in devs for _ in range(2)]
     st = [torch.cuda.Stream(device=d) for d in devs for _ in range(2)]

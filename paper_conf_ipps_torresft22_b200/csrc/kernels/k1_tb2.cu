@@ -79,6 +79,10 @@ constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
 #ifndef TB2_ST_SMEM
 #define TB2_ST_SMEM 0
 #endif
+// strides from the parameter bank (1) or recomputed from the geometry (0)
+#ifndef TB2_ADDR
+#define TB2_ADDR 1
+#endif
 // S2's results and stats without per-node branches around the stats (both
 // nodes' results live at once: spills, 5.07e10 -- not the default)
 #ifndef TB2_S2_BF
@@ -116,6 +120,8 @@ struct Tb2Params {
     int x_base, v_base;            // global i of raw plane 0 of the X / V slabs (start - 2, start - 1)
     int lo_end, hi_begin;          // planes q < lo_end go to lo_dst + (q - start), q >= hi_begin to hi_dst + (q - hi_begin)
     int stats_lo, stats_hi;        // output planes [stats_lo, stats_hi) contribute to the stats
+    int64_t cs, ps;                // component / plane stride in doubles (precomputed: the kernel
+                                   // reads them from the parameter bank instead of re-multiplying)
     int tiles_k, tiles_j, seg_planes;
 };
 
@@ -196,7 +202,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     const bool kown = lane >= 1 && lane <= kOK && k <= g.n2 - 2;   // interior k columns only
     const bool ownA = kown && rA >= 1 && jA < g.n1;               // rows 1 .. kRows-2
     const bool ownB = kown && rB <= kRows - 2 && jB < g.n1;
+#if TB2_ADDR
+    const int64_t cs = tp.cs, ps = tp.ps;
+#else
     const int64_t cs = g.comp_stride(), ps = g.plane_stride();
+#endif
     const int64_t offA = ownA ? (int64_t)jA * g.ld + k : 0, offB = ownB ? (int64_t)jB * g.ld + k : 0;
 
     // Tile-border springs of S1 (row above R1 -> R1 row 0: gbj; column left of
@@ -545,6 +555,8 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
     tp.v_base = (int)a.g.start - 1;
     tp.lo_end = a.lo_dst ? (int)a.g.start + 2 : INT_MIN;
     tp.hi_begin = a.hi_dst ? (int)(a.g.start + a.g.size) - 2 : INT_MAX;
+    tp.cs = a.g.comp_stride();
+    tp.ps = a.g.plane_stride();
     tp.stats_lo = o.stats_lo;
     tp.stats_hi = o.stats_hi;
     if (o.stats_lo == 0 && o.stats_hi == 0) {  // default: the chunk's own planes

@@ -74,6 +74,14 @@ constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
 #ifndef TB2_ST1_MODE
 #define TB2_ST1_MODE 2
 #endif
+// V_{t+1} handed from S1 to the next iteration's S2 through shared memory (1)
+// instead of a register carry (0)
+#ifndef TB2_V1_SMEM
+#define TB2_V1_SMEM 0
+#endif
+#if TB2_V1_SMEM && (TB2_S2_BF || TB2_ST1_MODE != 2)
+#error "TB2_V1_SMEM needs the branchy S2 and the S1 placement of step t+1's stats"
+#endif
 // the last step's stats accumulators in shared memory too (else registers;
 // 5.84-5.94e10: the LSU round trips cost more than the freed registers)
 #ifndef TB2_ST_SMEM
@@ -107,6 +115,9 @@ struct __align__(16) Smem {
     ulonglong2 acc1[4][kThreads];
 #if TB2_ST_SMEM
     ulonglong2 acc2[4][kThreads];  // the last step's, same layout (TB2_ST_SMEM variant)
+#endif
+#if TB2_V1_SMEM
+    double v1[2][3][kYComp];       // V_{t+1} of R1 by plane parity (TB2_V1_SMEM variant)
 #endif
 };
 
@@ -386,6 +397,17 @@ __global__ void __launch_bounds__(kThreads, 1)
         // step t+1's stats right where S1 produced them (plane p, if an output plane of this segment)
         if (kTwo && p >= max(pb, tp.stats_lo) && p < min(pe, tp.stats_hi)) acc1_update(x1A, x1B, v1A, v1B);
 #endif
+#if TB2_V1_SMEM
+        {
+            double* vv = sm.v1[par][0];
+            vv[yA] = v1A.x;
+            vv[yA + kYComp] = v1A.y;
+            vv[yA + 2 * kYComp] = v1A.z;
+            vv[yB] = v1B.x;
+            vv[yB + kYComp] = v1B.y;
+            vv[yB + 2 * kYComp] = v1B.z;
+        }
+#endif
         {
             double* y = sm.y[par][0];
             y[yA] = x1A.x;
@@ -451,7 +473,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (out2) {
             if (ownA) {
                 if (intA) {
+#if TB2_V1_SMEM
+                    Vec3 v2 = ldb(sm.v1[par ^ 1][0], yA, kYComp), x2 = xqA;
+#else
                     Vec3 v2 = v1pA, x2 = xqA;
+#endif
                     if (kTwo) {
                         const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
@@ -465,7 +491,11 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             if (ownB) {
                 if (intB) {
+#if TB2_V1_SMEM
+                    Vec3 v2 = ldb(sm.v1[par ^ 1][0], yB, kYComp), x2 = xqB;
+#else
                     Vec3 v2 = v1pB, x2 = xqB;
+#endif
                     if (kTwo) {
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
@@ -489,8 +519,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         xcB = niB;
         carry2A = gpi2A;
         carry2B = gpi2B;
+#if !TB2_V1_SMEM
         v1pA = v1A;
         v1pB = v1B;
+#endif
     };
     using F0 = std::integral_constant<bool, false>;
     using F1 = std::integral_constant<bool, true>;

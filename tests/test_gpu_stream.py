@@ -309,3 +309,31 @@ def test_stream_modes_alternate_on_one_handle():
     ref, rst = O.run(O.init(_op(sp)), 11)
     assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
     assert st.sums == rst.sums and st.step == 11
+
+
+@pytest.mark.parametrize("mode", ["run", "run2", "blocked4"])
+def test_stream_non_unit_mass_prestressed_vs_oracle(mode):
+    """The host-streamed paths (one-step kernel, K1_TB2 two steps per trip, s
+    steps per trip) at M != 1 and rest length != spacing, directly against the
+    oracle: every step's stats and the final state bitwise."""
+    n, nsteps = (15, 11, 34), 6
+    sp = P.SomierParams(n=n, seed=12, mass=0.7, spacing=1.25, rest_len=1.0, k_spring=4.0, dt=2e-3, amplitude=0.1)
+    with P.SomierStream(P.Spread([0, 1], 1, n[0] - 2, chunk=3), sp, buffers=2, cuda_devices=[0, 0]) as s:
+        X0, V0 = s.generate()
+        X, V, XN, VN = _pinned_like(X0), _pinned_like(V0), _pinned_like(X0), _pinned_like(V0)
+        X[...] = X0
+        V[...] = V0
+        if mode == "run":
+            stats = s.run(X, V, XN, nsteps)
+            fX, fV = (X, V)
+        elif mode == "run2":
+            stats = s.run2(X, V, XN, VN, nsteps)
+            fX, fV = (XN, VN)  # 3 launches
+        else:
+            stats = s.run_blocked(X, V, XN, VN, nsteps, 4)
+            fX, fV = (X, V)  # 2 trips
+    ref = O.init(_op(sp))
+    for t in range(nsteps):
+        ref, rst = O.step(ref)
+        assert stats[t].sums == rst.sums and stats[t].vmax2_bits == rst.vmax2_bits, t
+    assert np.array_equal(fX, ref.X) and np.array_equal(fV, ref.V)

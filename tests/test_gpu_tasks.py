@@ -83,14 +83,17 @@ def test_war_rewrite_after_reads():
 
 
 def test_no_barrier_between_constructs_trace():
-    """Pinned host array of 2^25 doubles over 8 chunks: with chunk-level
-    dependencies the stencil of some chunk m starts before the map(to) of a
-    later chunk has finished -- under the paper's taskgroup it could not."""
-    n = 1 << 25
+    """Pinned host arrays over 8 chunks whose last one is 100x larger: with
+    chunk-level dependencies the stencil of the small chunks starts while the
+    big chunk's map(to) is still running -- under the paper's taskgroup no loop
+    could start before every map(to) of the enter data had finished."""
+    small, big = 1 << 20, 100 << 20
+    sizes = [small] * 7 + [big]
+    n = sum(sizes) + 2
     A = torch.empty(n, dtype=torch.float64, pin_memory=True).numpy()
     A[:] = np.random.default_rng(1).normal(size=n)
     Bh = torch.zeros(n, dtype=torch.float64, pin_memory=True).numpy()
-    spread = P.Spread([0], 1, n - 2, chunk=(n - 2 + 7) // 8)
+    spread = P.Spread.with_sizes([0], 1, n - 2, sizes)
     with P.SpreadTasks(spread) as q:
         q.set_trace(True)
         a = q.enter(A, lo_halo=1, hi_halo=1)

@@ -1,10 +1,12 @@
 #!/usr/bin/env python3
-"""Trace of the chunk-level depend chain (SpreadTasks): enter A, B -> B = S(A)
--> C = S(B) -> reduce(C) -> exit C over 8 chunks of a pinned 2^26-double array
-on devices(0..P-1) mapped to cuda:0; prints one JSON line per chunk task
-(ms since tracing started) and a summary of the overlap across constructs:
-for every chunk, how long its loop started before the LAST map(to) finished
-(a taskgroup after the enter data would force this to be <= 0)."""
+"""Trace of the chunk-level depend chain (SpreadTasks): enter A, B, C -> B =
+S(A) -> C = S(B) -> reduce(C) -> exit C over 8 chunks (seven of 2^20 doubles,
+the last of 100 x 2^20) of pinned arrays on devices(0..P-1) mapped to cuda:0;
+prints one JSON line per chunk task (ms since tracing started) and a summary:
+how many chunks' loops started before the LAST map(to) finished (a taskgroup
+after the enter data would make that 0). The host-to-device copies of all
+chunks share the copy engine, so equal chunks finish their copies together;
+the big last chunk shows the chunk-level overlap.)"""
 import json
 import os
 import sys
@@ -15,13 +17,14 @@ import torch  # noqa: E402
 
 import paper_conf_ipps_torresft22_b200 as P  # noqa: E402
 
-n = 1 << 26
+sizes = [1 << 20] * 7 + [100 << 20]
+n = sum(sizes) + 2
 P_ = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 A = torch.empty(n, dtype=torch.float64, pin_memory=True).numpy()
 A[:] = np.random.default_rng(1).normal(size=n)
 Z = torch.zeros(n, dtype=torch.float64, pin_memory=True).numpy()
 C = torch.zeros(n, dtype=torch.float64, pin_memory=True).numpy()
-spread = P.Spread(list(range(P_)), 1, n - 2, chunk=(n - 2 + 7) // 8)
+spread = P.Spread.with_sizes(list(range(P_)), 1, n - 2, sizes)
 with P.SpreadTasks(spread, cuda_devices=[0] * P_) as q:
     q.set_trace(True)
     a = q.enter(A, lo_halo=1, hi_halo=1)

@@ -99,3 +99,21 @@ def test_our_arm_two_ranks_share_one_gpu():
     # the same e2e cycle as at N = 1: host-streamed over devices(0, 1), one process
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0 and "somier_stream_run" in d["e2e"]["cycle"]
     assert d["verify"]["ok"] and d["verify"]["nodes_checked"] > 0
+
+
+@pytest.mark.gpu
+def test_our_arm_four_ranks_same_fields_as_one():
+    """N = 4 (ranks sharing cuda:0): the line carries the same field set as
+    N = 1, plus per-rank roofline entries, and the verify pass is green."""
+    common = ["--grid", "64", "--steps", "4", "--warmup", "3", "--no-cpu-baseline", "--e2e-steps", "2",
+              "--stream-chunk", "8", "--verify", "--sustained-s", "0.2"]
+    l1, _ = _run(["bench.py"] + common)
+    l4, r = _run(_torchrun(4, 29567) + ["bench.py", "--gpus", "4", "--share-gpu"] + common,
+                 env={"OMP_NUM_THREADS": "1"})
+    assert len(l1) == 1 and len(l4) == 1, r.stdout[-2000:]
+    d1, d4 = json.loads(l1[0]), json.loads(l4[0])
+    assert set(d4) == set(d1)
+    assert set(d4["roofline"]) == set(d1["roofline"]) | {"per_rank"}
+    assert set(d4["e2e"]) == set(d1["e2e"]) and set(d4["halo"]) == set(d1["halo"])
+    assert len(d4["roofline"]["per_rank"]) == 4 and d4["verify"]["ok"] and d4["n_gpus"] == 4
+

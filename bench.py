@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--kernel", choices=["auto", "direct", "march", "march2", "tb2"], default="auto")
     ap.add_argument("--chunk", type=int, default=0, help="spread_schedule(static, chunk); 0 = one slab per GPU")
+    ap.add_argument("--exchange", choices=["fused", "copy", "nccl"], default="fused",
+                    help="halo exchange route (somier_params.exchange)")
     ap.add_argument("--e2e-steps", type=int, default=8)
     ap.add_argument("--stream-chunk", type=int, default=64, help="planes per chunk in the host-streamed e2e")
     ap.add_argument("--no-e2e", action="store_true")
@@ -611,7 +613,8 @@ def run_ours(a):
     n = a.n
     kernel = {"auto": P.K1_AUTO, "direct": P.K1_DIRECT, "march": P.K1_MARCH, "march2": P.K1_MARCH2,
               "tb2": P.K1_TB2}[a.kernel]
-    params = P.SomierParams(n=n, seed=42, kernel=kernel)
+    exchange = {"fused": P.EXCHANGE_FUSED, "copy": P.EXCHANGE_COPY, "nccl": P.EXCHANGE_NCCL}[a.exchange]
+    params = P.SomierParams(n=n, seed=42, kernel=kernel, exchange=exchange)
     if multi:
         s = PD.open_local(params, chunk=a.chunk, cuda_device=local)
     else:
@@ -780,7 +783,8 @@ def run_ours(a):
             "config": {"workload": workload_name(n), "n": list(n), "parallelism": "spread%d" % world,
                        "spread": "devices(%s) range(1:%d) spread_schedule(static,%d)"
                                  % (",".join(str(d) for d in spread.devices), n[0] - 2, spread.chunk_size),
-                       "kernel": "K1_" + kname.upper(), "l2": "no flush: 12.9 GB state >> 126 MB L2",
+                       "kernel": "K1_" + kname.upper(), "exchange": a.exchange,
+                       "l2": "no flush: 12.9 GB state >> 126 MB L2",
                        "seed": 42},
             "roofline": roof,
             "roofline_fp64": {"bound": "alu", "achieved": fp64_achieved, "peak": fp64_peak, "unit": "Tinstr/s",

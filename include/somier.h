@@ -81,7 +81,17 @@ typedef struct {
  * A/B: K1 writes only its own slab, then the stream copies the boundary planes
  * into the neighbours' halos (cudaMemcpyAsync over P2P / IPC) and writes the
  * flags (cuStreamWriteValue64) after the whole kernel. Results are bit-identical. */
-typedef enum { SOMIER_EXCHANGE_FUSED = 0, SOMIER_EXCHANGE_COPY = 1 } somier_exchange;
+typedef enum { SOMIER_EXCHANGE_FUSED = 0, SOMIER_EXCHANGE_COPY = 1, SOMIER_EXCHANGE_NCCL = 2 } somier_exchange;
+/* SOMIER_EXCHANGE_NCCL -- SURVEY.md §8(e)'s collective route: after each launch
+ * the boundary planes go by ncclSend / ncclRecv (one ncclGroupStart/End per
+ * launch over every chunk boundary, each list position one NCCL rank on its
+ * stream; same-position boundaries are self send/recv), no flags. NCCL is
+ * loaded at run time (SOMIER_NCCL_LIB, else libnccl.so.2). Single-process
+ * handles create the communicators at somier_init (ncclCommInitAll; the list's
+ * CUDA devices must be distinct: NCCL places one rank per GPU -- ENOTSUP
+ * otherwise); multi-process handles call somier_nccl_connect with an id from
+ * somier_nccl_unique_id shared by all ranks (rank = list position). */
+/* (somier_nccl_unique_id / somier_nccl_connect: below, after somier_ipc_connect) */
 
 /* Stats of one step ("centers"). The exact partial sums are
  * exported so that per-process partials can be combined exactly. */
@@ -147,6 +157,12 @@ spread_status somier_ipc_export(somier_t h, void* buf, size_t cap, size_t* len);
  * Errors: EINVAL (malformed blob, other spread or params), ECUDA.
  */
 spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const size_t* lens, int nblobs);
+
+/* SOMIER_EXCHANGE_NCCL, multi-process: one rank creates an id, every rank
+ * passes it with nranks = the list length (rank = device_pos). Errors: ENOTSUP
+ * (NCCL unavailable), ESTATE (not a multi-process NCCL handle), ENCCL. */
+spread_status somier_nccl_unique_id(void* id_out /* 128 bytes */);
+spread_status somier_nccl_connect(somier_t h, const void* id /* 128 bytes */, int nranks);
 
 /* Enqueue nsteps >= 0 time steps on every owned chunk; returns after enqueue (nowait). */
 spread_status somier_step(somier_t h, int64_t nsteps);

@@ -7,13 +7,13 @@ include/somier.h, implemented by libsomier.so (hand-written sm_100a kernels).
 This package is the Python binding (argument marshalling only).
 """
 from . import _native, capi
-from ._native import (EXCHANGE_COPY, EXCHANGE_FUSED, K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2, SCHED_DYNAMIC,
+from ._native import (EXCHANGE_COPY, EXCHANGE_FUSED, EXCHANGE_NCCL, K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2, K1_TB2, SCHED_DYNAMIC,
                       SCHED_STATIC, STATS_HISTORY, SpreadError)
 from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
 from .spread import Chunk, Spread, SpreadTasks
 
 __all__ = ["capi", "Spread", "SpreadTasks", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats", "combine_stats", "SpreadError",
-           "K1_AUTO", "K1_DIRECT", "K1_MARCH", "K1_MARCH2", "K1_TB2", "SCHED_STATIC", "SCHED_DYNAMIC", "EXCHANGE_FUSED", "EXCHANGE_COPY", "STATS_HISTORY", "version"]
+           "K1_AUTO", "K1_DIRECT", "K1_MARCH", "K1_MARCH2", "K1_TB2", "SCHED_STATIC", "SCHED_DYNAMIC", "EXCHANGE_FUSED", "EXCHANGE_COPY", "EXCHANGE_NCCL", "STATS_HISTORY", "version"]
 
 
 def version() -> str:

@@ -17,7 +17,7 @@ LIB_PATH = os.environ.get("SOMIER_LIB") or os.path.join(_HERE, "libsomier.so")
 # spread_status
 OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
 # somier_exchange
-EXCHANGE_FUSED, EXCHANGE_COPY = 0, 1
+EXCHANGE_FUSED, EXCHANGE_COPY, EXCHANGE_NCCL = 0, 1, 2
 # spread_sched
 SCHED_STATIC, SCHED_DYNAMIC = 0, 1
 # spread_map_type
@@ -139,6 +139,8 @@ SIGNATURES = [
     ("somier_stats", ctypes.c_int, [_VP, ctypes.POINTER(somier_stats_t)]),
     ("somier_stats_history", ctypes.c_int, [_VP, ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(somier_stats_t)]),
     ("somier_set_timing", ctypes.c_int, [_VP, ctypes.c_int]),
+    ("somier_nccl_unique_id", ctypes.c_int, [_VP]),
+    ("somier_nccl_connect", ctypes.c_int, [_VP, _VP, ctypes.c_int]),
     ("somier_take_timing", ctypes.c_int, [_VP, ctypes.POINTER(somier_timing_t)]),
     ("somier_stats_combine", ctypes.c_int, [ctypes.POINTER(somier_stats_t), ctypes.c_int,
                                             ctypes.POINTER(somier_params), ctypes.POINTER(somier_stats_t)]),
@@ -172,12 +174,28 @@ SIGNATURES = [
 ]
 
 
+def _default_nccl() -> None:
+    """SOMIER_EXCHANGE_NCCL loads NCCL at run time (SOMIER_NCCL_LIB): default to
+    the libnccl.so.2 torch.distributed itself uses, so one NCCL serves both."""
+    if os.environ.get("SOMIER_NCCL_LIB"):
+        return
+    try:
+        import nvidia.nccl  # the wheel torch's NCCL backend loads
+
+        path = os.path.join(list(nvidia.nccl.__path__)[0], "lib", "libnccl.so.2")
+        if os.path.exists(path):
+            os.environ["SOMIER_NCCL_LIB"] = path
+    except Exception:
+        pass
+
+
 def lib() -> ctypes.CDLL:
     global _lib
     if _lib is None:
         if not os.path.exists(LIB_PATH):
             raise ImportError("libsomier.so not built at %s: run __graft_entry__.build() "
                               "(there is no CPU fallback)" % LIB_PATH)
+        _default_nccl()
         L = ctypes.CDLL(LIB_PATH)
         for name, res, args in SIGNATURES:
             fn = getattr(L, name)

@@ -19,6 +19,7 @@
 
 #include "driver_util.hpp"
 #include "kernels.hpp"
+#include "nccl_api.hpp"
 #include "somier.h"
 #include "spread_impl.hpp"
 #include "status.hpp"
@@ -161,6 +162,7 @@ struct somier_s {
     };
     bool timing = false;
     std::vector<TimingRec> trecs;
+    std::vector<paper::ncclComm> comms;  // SOMIER_EXCHANGE_NCCL: per list position (local ones)
 
     bool unit_mass() const { return p.mass == 1.0; }
     paper::K1Variant variant() const {
@@ -176,6 +178,7 @@ struct somier_s {
     // Neighbour chunks on another stream (other device or other process) need
     // the flag protocol; same-stream neighbours are ordered by the stream.
     bool needs_flags(const Chunk& a, const Chunk& b) const {
+        if (p.exchange == SOMIER_EXCHANGE_NCCL) return false;  // the NCCL ops order the streams
         if (!a.local || !b.local) return true;
         return a.pos != b.pos;
     }
@@ -230,7 +233,8 @@ spread_status check_params(const somier_params* p) {
     if (!(p->dt > 0)) PAPER_FAIL(SPREAD_EINVAL, "somier: dt must be > 0");
     if (p->kernel < SOMIER_K1_AUTO || p->kernel > SOMIER_K1_TB2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown kernel %d", p->kernel);
-    if (p->exchange != SOMIER_EXCHANGE_FUSED && p->exchange != SOMIER_EXCHANGE_COPY)
+    if (p->exchange != SOMIER_EXCHANGE_FUSED && p->exchange != SOMIER_EXCHANGE_COPY &&
+        p->exchange != SOMIER_EXCHANGE_NCCL)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown exchange %d", p->exchange);
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
     if (n1 > 65535LL * 8 || n0 > 65535 + 2)
@@ -271,6 +275,12 @@ spread_status load_driver_entry(somier_t h) {
 
 void free_all(somier_t h) {
     if (!h) return;
+    for (size_t q = 0; q < h->comms.size(); q++)
+        if (h->comms[q]) {
+            cudaSetDevice(h->devs[q].device);
+            paper::nccl_lib().CommDestroy(h->comms[q]);
+            h->comms[q] = nullptr;
+        }
     for (auto& c : h->chunks) {
         if (c.remote_base) {
             cudaSetDevice(h->devs[h->local_pos >= 0 ? h->local_pos : 0].device);
@@ -523,6 +533,33 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
         if ((c > 0 && !h->chunks[c - 1].local) || (c + 1 < h->chunks.size() && !h->chunks[c + 1].local))
             h->connected = false;
     }
+    // SOMIER_EXCHANGE_NCCL: one rank per list position
+    h->comms.assign(h->devs.size(), nullptr);
+    if (p->exchange == SOMIER_EXCHANGE_NCCL) {
+        const paper::NcclLib& L = paper::nccl_lib();
+        if (!L.ok) {
+            set_last_error("somier_init: NCCL unavailable (%s)", L.error.c_str());
+            return fail(SPREAD_ENOTSUP);
+        }
+        if (local_pos < 0) {
+            std::vector<int> devl;
+            for (auto& d : h->devs) devl.push_back(d.device);
+            std::vector<int> sorted = devl;
+            std::sort(sorted.begin(), sorted.end());
+            if (std::adjacent_find(sorted.begin(), sorted.end()) != sorted.end()) {
+                set_last_error("somier_init: the NCCL exchange needs one CUDA device per list position "
+                               "(NCCL places one rank per GPU)");
+                return fail(SPREAD_ENOTSUP);
+            }
+            const int r = L.CommInitAll(h->comms.data(), (int)devl.size(), devl.data());
+            if (r != 0) {
+                set_last_error("somier_init: ncclCommInitAll: %s", L.GetErrorString(r));
+                return fail(SPREAD_ENCCL);
+            }
+        } else {
+            h->connected = false;  // somier_nccl_connect
+        }
+    }
     // graph replay needs a single stream and no flag protocol (SOMIER_NO_GRAPH=1 disables it)
     {
         int pos = -1;
@@ -536,7 +573,7 @@ spread_status init_common(spread_t s, const somier_params* p, int local_pos, int
             if (c.pos != pos) one = false;
         }
         const char* ng = std::getenv("SOMIER_NO_GRAPH");
-        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1');
+        h->graph_ok = one && pos >= 0 && !(ng && ng[0] == '1') && p->exchange != SOMIER_EXCHANGE_NCCL;
         h->graph_pos = pos;
         // PDL between consecutive K1 launches only where nothing else sits
         // between them on the stream (one stream, no flag waits); SOMIER_NO_PDL=1
@@ -650,6 +687,61 @@ extern "C" {
 }  // extern "C"
 
 namespace {
+
+// SOMIER_EXCHANGE_NCCL: after the launches of one step (one-step kernels) or
+// one two-step launch (K1_TB2), every chunk boundary exchanges its planes by
+// ncclSend / ncclRecv in one group: message U (the lower chunk's top planes ->
+// the upper chunk's bottom halo) then message D (the upper chunk's bottom
+// planes -> the lower chunk's top halo), in boundary order on every rank, so
+// the k-th send from a rank to a peer matches that peer's k-th receive from it
+// (same-position boundaries are self send/recv). xo / vo: the buffers of the
+// new state (K1_TB2: raw deep-halo slabs; one-step: the one-halo X views, V
+// unused).
+spread_status nccl_exchange(somier_t h, bool tb2, int xo, int vo) {
+    const paper::NcclLib& L = paper::nccl_lib();
+    const int64_t ps = h->geom.plane_stride();
+    const size_t pb = (size_t)ps * sizeof(double);
+    const int64_t nch = (int64_t)h->chunks.size();
+    std::string err;
+    auto ck = [&](int r, const char* what) {
+        if (r != 0 && err.empty()) err = std::string(what) + ": " + L.GetErrorString(r);
+    };
+    ck(L.GroupStart(), "ncclGroupStart");
+    for (int64_t b = 0; b + 1 < nch; b++) {
+        Chunk& lo = h->chunks[(size_t)b];
+        Chunk& hi = h->chunks[(size_t)b + 1];
+        struct Msg {
+            double* src;
+            double* dst;
+            size_t bytes;
+        };
+        // U: lo -> hi, D: hi -> lo (X planes, then the V plane on K1_TB2 handles)
+        std::vector<Msg> U, D;
+        if (tb2) {
+            U = {{lo.x(xo) + lo.size * ps, hi.x(xo), 2 * pb}, {lo.v(vo) + lo.size * ps, hi.v(vo), pb}};
+            D = {{hi.x(xo) + 2 * ps, lo.x(xo) + (lo.size + 2) * ps, 2 * pb},
+                 {hi.v(vo) + ps, lo.v(vo) + (lo.size + 1) * ps, pb}};
+        } else {
+            U = {{lo.xs(xo) + lo.size * ps, hi.xs(xo), pb}};
+            D = {{hi.xs(xo) + ps, lo.xs(xo) + (lo.size + 1) * ps, pb}};
+        }
+        for (const Msg& m : U) {
+            if (lo.local) ck(L.Send(m.src, m.bytes, paper::kNcclUint8, hi.pos, h->comms[lo.pos], h->stream_of(lo)), "ncclSend");
+            if (hi.local) ck(L.Recv(m.dst, m.bytes, paper::kNcclUint8, lo.pos, h->comms[hi.pos], h->stream_of(hi)), "ncclRecv");
+        }
+        for (const Msg& m : D) {
+            if (hi.local) ck(L.Send(m.src, m.bytes, paper::kNcclUint8, lo.pos, h->comms[hi.pos], h->stream_of(hi)), "ncclSend");
+            if (lo.local) ck(L.Recv(m.dst, m.bytes, paper::kNcclUint8, hi.pos, h->comms[lo.pos], h->stream_of(lo)), "ncclRecv");
+        }
+    }
+    ck(L.GroupEnd(), "ncclGroupEnd");
+    if (!err.empty()) {
+        if (h->sticky.empty()) h->sticky = err;
+        PAPER_FAIL(SPREAD_ENCCL, "somier_step: %s", err.c_str());
+    }
+    return SPREAD_OK;
+}
+
 spread_status enqueue_steps(somier_t h, int64_t nsteps);
 spread_status enqueue_tb2(somier_t h, bool two);
 }
@@ -767,7 +859,8 @@ spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const siz
             o.off_counter = rec.off_counter;
         }
     }
-    h->connected = true;
+    // the NCCL exchange does not use the neighbours' memory: it still needs its communicator
+    h->connected = h->p.exchange != SOMIER_EXCHANGE_NCCL || h->comms[(size_t)h->local_pos] != nullptr;
     return SPREAD_OK;
 }
 
@@ -933,7 +1026,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             a.pdl = h->pdl && !h->timing ? 1 : 0;
             if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
             CUDA_TRY(h, paper::launch_k1(h->variant(), a, h->unit_mass(), st));
-            if (!fused) {
+            if (h->p.exchange == SOMIER_EXCHANGE_COPY) {
                 // SOMIER_EXCHANGE_COPY: the boundary planes of X_{t+1} into the
                 // neighbours' halo planes after the kernel, then their flags
                 const int64_t ps = h->geom.plane_stride();
@@ -953,6 +1046,10 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
                 h->trecs.push_back(tr);
             }
             h->launches++;
+        }
+        if (h->p.exchange == SOMIER_EXCHANGE_NCCL) {
+            spread_status ns = nccl_exchange(h, false, nxt, 0);
+            if (ns != SPREAD_OK) return ns;
         }
         h->step++;
         h->xbuf ^= 1;
@@ -1034,7 +1131,7 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         a.side_counter = me.side_counter();
         if (h->timing) CUDA_TRY(h, cudaEventRecord(tr.b, st));
         CUDA_TRY(h, paper::launch_k1_tb2(a, o, h->unit_mass(), st));
-        if (!fused) {
+        if (h->p.exchange == SOMIER_EXCHANGE_COPY) {
             // SOMIER_EXCHANGE_COPY: the first two X planes and the first V plane
             // of the new state to the left neighbour's deep halo, the last two /
             // last one to the right's (the planes the fused kernel stores), then
@@ -1061,6 +1158,10 @@ spread_status enqueue_tb2(somier_t h, bool two) {
             h->trecs.push_back(tr);
         }
         h->launches++;
+    }
+    if (h->p.exchange == SOMIER_EXCHANGE_NCCL) {
+        spread_status ns = nccl_exchange(h, true, cur ^ 1, vb ^ 1);
+        if (ns != SPREAD_OK) return ns;
     }
     h->step = t_end;
     h->xbuf ^= 1;
@@ -1323,6 +1424,34 @@ spread_status somier_device_bytes(somier_t h, int64_t* bytes) {
     for (auto& c : h->chunks)
         if (c.local) b += (int64_t)c.bytes;
     *bytes = b;
+    return SPREAD_OK;
+}
+
+spread_status somier_nccl_unique_id(void* id_out) {
+    if (!id_out) PAPER_FAIL(SPREAD_EINVAL, "somier_nccl_unique_id: NULL argument");
+    const paper::NcclLib& L = paper::nccl_lib();
+    if (!L.ok) PAPER_FAIL(SPREAD_ENOTSUP, "somier_nccl_unique_id: NCCL unavailable (%s)", L.error.c_str());
+    paper::NcclUniqueId id;
+    const int r = L.GetUniqueId(&id);
+    if (r != 0) PAPER_FAIL(SPREAD_ENCCL, "ncclGetUniqueId: %s", L.GetErrorString(r));
+    std::memcpy(id_out, &id, sizeof id);
+    return SPREAD_OK;
+}
+
+spread_status somier_nccl_connect(somier_t h, const void* id, int nranks) {
+    if (!h || !id) PAPER_FAIL(SPREAD_EINVAL, "somier_nccl_connect: NULL argument");
+    if (!h->multi_process || h->p.exchange != SOMIER_EXCHANGE_NCCL)
+        PAPER_FAIL(SPREAD_ESTATE, "somier_nccl_connect: not a multi-process handle with the NCCL exchange");
+    if (nranks != (int)h->devs.size())
+        PAPER_FAIL(SPREAD_EINVAL, "somier_nccl_connect: %d ranks for a list of %d positions", nranks,
+                   (int)h->devs.size());
+    const paper::NcclLib& L = paper::nccl_lib();
+    paper::NcclUniqueId uid;
+    std::memcpy(&uid, id, sizeof uid);
+    CUDA_TRY(h, cudaSetDevice(h->devs[(size_t)h->local_pos].device));
+    const int r = L.CommInitRank(&h->comms[(size_t)h->local_pos], nranks, uid, h->local_pos);
+    if (r != 0) PAPER_FAIL(SPREAD_ENCCL, "ncclCommInitRank: %s", L.GetErrorString(r));
+    h->connected = true;
     return SPREAD_OK;
 }
 

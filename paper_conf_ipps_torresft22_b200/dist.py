@@ -54,14 +54,30 @@ def connect(s: Somier, group=None) -> None:
 
 
 def open_local(params: SomierParams, chunk: int = 0, group=None, cuda_device: Optional[int] = None) -> Somier:
-    """Create this rank's part of a grid spread over all ranks (devices(0..world-1))."""
+    """Create this rank's part of a grid spread over all ranks (devices(0..world-1)).
+    Fused / copy exchange: the ranks swap CUDA IPC blobs; NCCL exchange
+    (params.exchange == EXCHANGE_NCCL): rank 0's ncclUniqueId is shared and every
+    rank joins the communicator (somier_nccl_connect)."""
+    import ctypes
+
     import torch.distributed as dist
+
+    from . import _native as N
 
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
     spread = Spread(list(range(world)), 1, params.n[0] - 2, chunk=chunk)
     s = Somier(spread, params, device_pos=rank, cuda_device=rank if cuda_device is None else cuda_device)
-    connect(s, group)
+    if params.exchange == N.EXCHANGE_NCCL:
+        uid = ctypes.create_string_buffer(128)
+        if rank == 0:
+            N.check(N.lib().somier_nccl_unique_id(uid), "somier_nccl_unique_id")
+        ids = all_gather_bytes(uid.raw, group)
+        N.check(N.lib().somier_nccl_connect(s._h, ctypes.create_string_buffer(ids[0], 128), world),
+                "somier_nccl_connect")
+        dist.barrier(group)
+    else:
+        connect(s, group)
     return s
 
 

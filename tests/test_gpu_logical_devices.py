@@ -131,3 +131,34 @@ def test_tb2_load_and_continue(chunk):
     ref, rst = O.run(O.init(O.Params(n=n, seed=2)), 10)
     assert np.array_equal(X2, ref.X) and np.array_equal(V2, ref.V)
     assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits
+
+
+@pytest.mark.parametrize("kernel", [P.K1_MARCH2, P.K1_TB2, P.K1_DIRECT])
+@pytest.mark.parametrize("chunk", [2, 3, 7])
+def test_nccl_exchange_self_send_bitwise(kernel, chunk):
+    """SOMIER_EXCHANGE_NCCL on one GPU: every chunk boundary goes through
+    ncclSend / ncclRecv (one list position = one rank, so the boundaries are
+    self send/recv on its stream) -- the route's buffers, plane offsets and
+    message order, bitwise against the oracle."""
+    n, steps = (22, 19, 45), 13
+    sp = P.SomierParams(n=n, seed=11, kernel=kernel, exchange=P.EXCHANGE_NCCL)
+    with P.Somier(P.Spread([0], 1, n[0] - 2, chunk=chunk), sp) as s:
+        s.step(5)
+        s.step(steps - 5)
+        st = s.stats()
+        X, V = s.read()
+    ref, rst = O.run(O.init(O.Params(n=n, seed=11)), steps)
+    assert np.array_equal(X, ref.X) and np.array_equal(V, ref.V)
+    assert st.sums == rst.sums and st.vmax2_bits == rst.vmax2_bits
+
+
+def test_nccl_exchange_needs_distinct_gpus():
+    """NCCL places one rank per GPU: two list positions on one device are refused."""
+    sp = P.SomierParams(n=(12, 10, 10), exchange=P.EXCHANGE_NCCL)
+    with pytest.raises(P.SpreadError) as e:
+        P.Somier(P.Spread([0, 1], 1, 10), sp, cuda_devices=[0, 0])
+    assert e.value.status == P._native.ENOTSUP
+    import ctypes
+    uid = ctypes.create_string_buffer(128)
+    P._native.check(P._native.lib().somier_nccl_unique_id(uid), "somier_nccl_unique_id")
+    assert any(uid.raw)

@@ -20,6 +20,7 @@
 #include "driver_util.hpp"
 #include "kernels.hpp"
 #include "nccl_api.hpp"
+#include "trace.hpp"
 #include "somier.h"
 #include "spread_impl.hpp"
 #include "status.hpp"
@@ -865,6 +866,7 @@ spread_status somier_ipc_connect(somier_t h, const void* const* blobs, const siz
 }
 
 spread_status somier_step(somier_t h, int64_t nsteps) {
+    PAPER_NVTX("somier_step");
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_step: NULL handle");
     if (nsteps < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_step: nsteps < 0");
     if (!h->connected) PAPER_FAIL(SPREAD_ESTATE, "somier_step: remote neighbour chunks not connected (somier_ipc_connect)");
@@ -1174,6 +1176,7 @@ spread_status enqueue_tb2(somier_t h, bool two) {
 extern "C" {
 
 spread_status somier_sync(somier_t h) {
+    PAPER_NVTX("somier_sync");
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_sync: NULL handle");
     return sync_all(h);
 }
@@ -1181,6 +1184,7 @@ spread_status somier_sync(somier_t h) {
 static_assert(SOMIER_STATS_HISTORY == paper::kStatsHistory, "somier.h history depth");
 
 spread_status somier_stats_history(somier_t h, int64_t first_step, int64_t count, somier_stats_t* out) {
+    PAPER_NVTX("somier_stats_history");
     if (!h || (count > 0 && !out)) PAPER_FAIL(SPREAD_EINVAL, "somier_stats_history: NULL argument");
     if (count < 0) PAPER_FAIL(SPREAD_EINVAL, "somier_stats_history: count < 0");
     const int64_t lo = std::max(h->hist_first, h->step - (int64_t)paper::kStatsHistory + 1);
@@ -1236,6 +1240,7 @@ spread_status somier_stats_combine(const somier_stats_t* parts, int n, const som
 
 spread_status somier_read_planes(somier_t h, int64_t i0, int64_t count, double* x, double* y, double* z, double* vx,
                                  double* vy, double* vz) {
+    PAPER_NVTX("somier_read_planes");
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_read_planes: NULL handle");
     const int64_t n0 = h->p.n[0];
     if (i0 < 0 || count < 0 || i0 + count > n0)
@@ -1287,6 +1292,7 @@ spread_status somier_read(somier_t h, double* x, double* y, double* z, double* v
 
 spread_status somier_load(somier_t h, const double* x, const double* y, const double* z, const double* vx,
                           const double* vy, const double* vz) {
+    PAPER_NVTX("somier_load");
     if (!h) PAPER_FAIL(SPREAD_EINVAL, "somier_load: NULL handle");
     if (!x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_load: NULL grid");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());

@@ -23,6 +23,7 @@
 #include "somier.h"
 #include "spread_impl.hpp"
 #include "status.hpp"
+#include "trace.hpp"
 
 using paper::set_last_error;
 
@@ -574,6 +575,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
 // receives the statistics after step t. One host barrier at the end.
 spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
                                  double* const VN[3], int64_t nsteps, int64_t s, somier_stats_t* stats) {
+    PAPER_NVTX("somier_stream_run_blocked");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     const int64_t ntrips = (nsteps + s - 1) / s;
     spread_status st = ensure_acc(h, nsteps);
@@ -603,6 +605,7 @@ spread_status stream_run_blocked(somier_stream_t h, double* const X[3], double* 
 // non-NULL) receives the statistics after step t. One host barrier at the end.
 spread_status stream_run(somier_stream_t h, double* const X[3], double* const V[3], double* const XN[3],
                          int64_t nsteps, somier_stats_t* stats) {
+    PAPER_NVTX("somier_stream_run");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     spread_status st = ensure_flat(h);
     if (st != SPREAD_OK) return st;
@@ -698,6 +701,7 @@ spread_status somier_stream_create_on(spread_t s, const somier_params* p, int bu
 
 spread_status somier_stream_generate(somier_stream_t h, double* x, double* y, double* z, double* vx, double* vy,
                                      double* vz) {
+    PAPER_NVTX("somier_stream_generate");
     if (!h || !x || !y || !z || !vx || !vy || !vz) PAPER_FAIL(SPREAD_EINVAL, "somier_stream_generate: NULL argument");
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
     {

@@ -34,6 +34,7 @@
 #include "spread.h"
 #include "spread_impl.hpp"
 #include "status.hpp"
+#include "trace.hpp"
 
 namespace {
 
@@ -281,6 +282,7 @@ spread_status spread_tasks_create(spread_t s, const int* cuda_devices, spread_ta
 }
 
 spread_status spread_enter_data(spread_tasks_t q, const double* host, int64_t n, spread_map m, spread_data_t* out) {
+    PAPER_NVTX("spread_enter_data");
     spread_status st = check_open(q, "spread_enter_data");
     if (st != SPREAD_OK) return st;
     if (!out || n < 0 || m.lo_halo < 0 || m.hi_halo < 0) PAPER_FAIL(SPREAD_EINVAL, "spread_enter_data: bad arguments");
@@ -326,6 +328,7 @@ spread_status spread_enter_data(spread_tasks_t q, const double* host, int64_t n,
 }
 
 spread_status spread_task_stencil3(spread_tasks_t q, spread_data_t a, spread_data_t b) {
+    PAPER_NVTX("spread_task_stencil3");
     spread_status st = check_open(q, "spread_task_stencil3");
     if (st != SPREAD_OK) return st;
     if (!a || !b || a->q != q || b->q != q || a == b)
@@ -359,6 +362,7 @@ spread_status spread_task_stencil3(spread_tasks_t q, spread_data_t a, spread_dat
 }
 
 spread_status spread_task_reduce(spread_tasks_t q, spread_data_t a, int scale_exp, spread_reduce_result* out) {
+    PAPER_NVTX("spread_task_reduce");
     spread_status st = check_open(q, "spread_task_reduce");
     if (st != SPREAD_OK) return st;
     if (!a || a->q != q || !out) PAPER_FAIL(SPREAD_EINVAL, "spread_task_reduce: bad arguments");
@@ -394,6 +398,7 @@ spread_status spread_task_reduce(spread_tasks_t q, spread_data_t a, int scale_ex
 }
 
 spread_status spread_exit_data(spread_tasks_t q, spread_data_t a, double* host) {
+    PAPER_NVTX("spread_exit_data");
     spread_status st = check_open(q, "spread_exit_data");
     if (st != SPREAD_OK) return st;
     if (!a || a->q != q || !host) PAPER_FAIL(SPREAD_EINVAL, "spread_exit_data: bad arguments");
@@ -415,6 +420,7 @@ spread_status spread_exit_data(spread_tasks_t q, spread_data_t a, double* host) 
 }
 
 spread_status spread_taskwait(spread_tasks_t q) {
+    PAPER_NVTX("spread_taskwait");
     if (!q) PAPER_FAIL(SPREAD_EINVAL, "spread_taskwait: NULL task queue");
     Err e;
     for (int64_t c = 0; c < (int64_t)q->streams.size(); c++) {

@@ -43,7 +43,7 @@ int main(int argc, char** argv) {
         printf("chunk %lld: device %d, omp_spread_start %lld, omp_spread_size %lld, map(to: X[%lld:%lld])\n",
                (long long)c, id, (long long)start, (long long)size, (long long)first, (long long)len);
     }
-    somier_params p = {{n, n, n}, 1.0, 1.0, 10.0, 1.0, 1e-3, 0.05, 42, SOMIER_K1_AUTO, 0};
+    somier_params p = {{n, n, n}, 1.0, 1.0, 10.0, 1.0, 1e-3, 0.05, 42, SOMIER_K1_AUTO, SOMIER_EXCHANGE_FUSED};
     somier_t h;
     CHECK(somier_init(sp, &p, &h));
     CHECK(spread_destroy(sp)); /* the handle keeps its own copy */
@@ -53,6 +53,13 @@ int main(int argc, char** argv) {
     CHECK(somier_stats(h, &st));
     printf("step %lld centre (%.17g, %.17g, %.17g) vmax %.17g nodes %lld\n", (long long)st.step, st.centre[0],
            st.centre[1], st.centre[2], st.vmax, (long long)st.nodes);
+    /* the "centers" of every step: the last few from the history */
+    const int64_t nh = steps < 4 ? steps : 4;
+    somier_stats_t hist[4];
+    CHECK(somier_stats_history(h, steps - nh + 1, nh, hist));
+    for (int64_t i = 0; i < nh; i++)
+        printf("history step %lld centre (%.17g, %.17g, %.17g) vmax %.17g\n", (long long)hist[i].step,
+               hist[i].centre[0], hist[i].centre[1], hist[i].centre[2], hist[i].vmax);
     const size_t N = (size_t)(n * n * n);
     double* g = (double*)malloc(6 * N * sizeof(double));
     if (!g) return 1;

@@ -91,5 +91,13 @@ def gather_stats(s: Somier, group=None) -> Stats:
     return combine_stats(parts, s.params)
 
 
+def gather_stats_history(s: Somier, first_step: int, count: int, group=None) -> List[Stats]:
+    """Exact global stats of steps first_step .. first_step+count-1 (every
+    rank's somier_stats_history partials combined step by step)."""
+    mine = s.stats_history(first_step, count)
+    parts = all_gather_obj(mine, group)
+    return [combine_stats([p[i] for p in parts], s.params) for i in range(count)]
+
+
 def combine_partials(parts: Sequence[Stats], params: SomierParams) -> Stats:
     return combine_stats(parts, params)

@@ -126,6 +126,7 @@ def gpu_ipc(a):
     s.step(a.steps)
     s.sync()
     st = PD.gather_stats(s)
+    hist = PD.gather_stats_history(s, 1, a.steps)  # every step's exact global stats
     X, V = s.read()
     mask = np.zeros(n[0], bool)
     for c in s.spread.chunks():
@@ -143,7 +144,9 @@ def gpu_ipc(a):
             out[:3, m] = x
             out[3:, m] = v
         np.savez(a.out, state=out, sums=np.array([str(v) for v in st.sums]), vmax2=np.array(str(st.vmax2_bits)),
-                 centre=np.array(st.centre), launches=np.array(s.launches))
+                 centre=np.array(st.centre), launches=np.array(s.launches),
+                 hist_sums=np.array([[str(v) for v in h.sums] for h in hist]),
+                 hist_vmax2=np.array([str(h.vmax2_bits) for h in hist]))
     dist.barrier()
     s.close()
     dist.barrier()

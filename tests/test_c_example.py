@@ -50,3 +50,11 @@ def test_c_example_centre_equals_oracle(tmp_path):
     _, st = O.run(O.init(O.Params(n=(24, 24, 24), seed=42)), 10)
     assert tuple(float(m.group(i)) for i in (1, 2, 3)) == st.centre
     assert float(m.group(4)) == st.vmax
+    hist = re.findall(r"history step (\d+) centre \(([^,]+), ([^,]+), ([^)]+)\) vmax (\S+)", r.stdout)
+    assert [int(h[0]) for h in hist] == [7, 8, 9, 10]
+    s = O.init(O.Params(n=(24, 24, 24), seed=42))
+    for t in range(1, 11):
+        s, st = O.step(s)
+        if t >= 7:
+            h = hist[t - 7]
+            assert tuple(float(v) for v in h[1:4]) == st.centre and float(h[4]) == st.vmax

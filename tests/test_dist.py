@@ -68,6 +68,12 @@ def test_gpu_two_processes_ipc_fused_exchange(tmp_path, chunk, kernel):
     n, steps, seed = (20, 12, 40), 15, 4
     res = _launch("gpu-ipc", str(tmp_path / "g.npz"), n, steps, chunk, seed, timeout=600, kernel=kernel)
     _check(res, n, steps, seed)
+    # every step's global stats (per-rank history partials combined exactly)
+    s = O.init(O.Params(n=n, seed=seed))
+    for t in range(steps):
+        s, st = O.step(s)
+        assert [int(v) for v in res["hist_sums"][t]] == list(st.sums)
+        assert int(str(res["hist_vmax2"][t])) == st.vmax2_bits
 
 
 @pytest.mark.gpu

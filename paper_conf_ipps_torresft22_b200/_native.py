@@ -126,6 +126,8 @@ SIGNATURES = [
     ("spread_tasks_set_trace", ctypes.c_int, [_VP, ctypes.c_int]),
     ("spread_tasks_trace", ctypes.c_int, [_VP, ctypes.POINTER(spread_task_record), ctypes.c_int64, _I64P]),
     ("spread_tasks_destroy", ctypes.c_int, [_VP]),
+    ("spread_tasks_hold", ctypes.c_int, [_VP, ctypes.c_int64]),
+    ("spread_tasks_release", ctypes.c_int, [_VP]),
     ("spread_last_error", ctypes.c_char_p, []),
     ("spread_status_string", ctypes.c_char_p, [ctypes.c_int]),
     ("somier_init", ctypes.c_int, [_VP, ctypes.POINTER(somier_params), ctypes.POINTER(_VP)]),

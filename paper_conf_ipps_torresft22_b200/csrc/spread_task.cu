@@ -21,10 +21,12 @@
 // copy from the neighbours' device memory (peer copies) once they have written
 // it. So chunk m+1's map(to) runs while chunk m's loop runs, across constructs,
 // and a device never idles at a construct boundary.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -79,6 +81,16 @@ __global__ void __launch_bounds__(256) task_sum_kernel(const double* __restrict_
 
 int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 8)); }
 
+using PFN_wait32 = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+PFN_wait32 load_wait32() {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult qr;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &fn, cudaEnableDefault, &qr) != cudaSuccess ||
+        qr != cudaDriverEntryPointSuccess)
+        return nullptr;
+    return (PFN_wait32)fn;
+}
+
 }  // namespace
 
 struct spread_data_s;
@@ -104,6 +116,7 @@ struct spread_tasks_s {
     };
     std::vector<TraceRec> trace_recs;
     cudaEvent_t trace_origin = nullptr;
+    uint32_t* hold_word = nullptr;  // spread_tasks_hold: mapped pinned word the held streams wait on
     std::string sticky;
 };
 
@@ -457,6 +470,34 @@ spread_status spread_taskwait(spread_tasks_t q) {
     return SPREAD_OK;
 }
 
+spread_status spread_tasks_hold(spread_tasks_t q, int64_t chunk) {
+    if (!q || chunk < 0 || chunk >= (int64_t)q->streams.size())
+        PAPER_FAIL(SPREAD_EINVAL, "spread_tasks_hold: bad arguments");
+    static PFN_wait32 wait32 = load_wait32();
+    if (!wait32) PAPER_FAIL(SPREAD_ECUDA, "spread_tasks_hold: cuStreamWaitValue32 unavailable");
+    if (!q->hold_word) {
+        cudaSetDevice(q->cuda_dev[(size_t)q->spread.chunk_info(0).pos]);
+        if (cudaHostAlloc((void**)&q->hold_word, sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
+            cudaSuccess)
+            PAPER_FAIL(SPREAD_ENOMEM, "spread_tasks_hold: cudaHostAlloc");
+        *q->hold_word = 0u;
+    }
+    void* dptr = nullptr;
+    cudaSetDevice(q->cuda_dev[(size_t)q->spread.chunk_info(chunk).pos]);
+    if (cudaHostGetDevicePointer(&dptr, (void*)q->hold_word, 0) != cudaSuccess)
+        PAPER_FAIL(SPREAD_ECUDA, "spread_tasks_hold: cudaHostGetDevicePointer");
+    *q->hold_word = 0u;
+    if (wait32((CUstream)q->streams[(size_t)chunk], (CUdeviceptr)dptr, 1u, CU_STREAM_WAIT_VALUE_GEQ) != CUDA_SUCCESS)
+        PAPER_FAIL(SPREAD_ECUDA, "spread_tasks_hold: cuStreamWaitValue32");
+    return SPREAD_OK;
+}
+
+spread_status spread_tasks_release(spread_tasks_t q) {
+    if (!q) PAPER_FAIL(SPREAD_EINVAL, "spread_tasks_release: NULL task queue");
+    if (q->hold_word) *(volatile uint32_t*)q->hold_word = 1u;
+    return SPREAD_OK;
+}
+
 spread_status spread_tasks_set_trace(spread_tasks_t q, int on) {
     if (!q) PAPER_FAIL(SPREAD_EINVAL, "spread_tasks_set_trace: NULL task queue");
     q->trace = on != 0;
@@ -489,6 +530,7 @@ spread_status spread_tasks_trace(spread_tasks_t q, spread_task_record* recs, int
 
 spread_status spread_tasks_destroy(spread_tasks_t q) {
     if (!q) return SPREAD_OK;
+    if (q->hold_word) *(volatile uint32_t*)q->hold_word = 1u;  // never leave a held stream behind
     for (int64_t c = 0; c < (int64_t)q->streams.size(); c++) {
         cudaSetDevice(q->cuda_dev[(size_t)q->spread.chunk_info(c).pos]);
         cudaStreamSynchronize(q->streams[(size_t)c]);
@@ -516,6 +558,7 @@ spread_status spread_tasks_destroy(spread_tasks_t q) {
         cudaEventDestroy(r.b);
     }
     if (q->trace_origin) cudaEventDestroy(q->trace_origin);
+    if (q->hold_word) cudaFreeHost(q->hold_word);
     for (int64_t c = 0; c < (int64_t)q->streams.size(); c++) {
         cudaSetDevice(q->cuda_dev[(size_t)q->spread.chunk_info(c).pos]);
         cudaStreamDestroy(q->streams[(size_t)c]);

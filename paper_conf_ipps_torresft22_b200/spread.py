@@ -229,6 +229,13 @@ class SpreadTasks:
         N.check(N.lib().spread_taskwait(self._h), "spread_taskwait")
         self._keep = []
 
+    def hold(self, chunk: int) -> None:
+        """Test hook: chunk's stream waits before its next task until release()."""
+        N.check(N.lib().spread_tasks_hold(self._h, int(chunk)), "spread_tasks_hold")
+
+    def release(self) -> None:
+        N.check(N.lib().spread_tasks_release(self._h), "spread_tasks_release")
+
     def set_trace(self, on: bool = True) -> None:
         N.check(N.lib().spread_tasks_set_trace(self._h, 1 if on else 0), "spread_tasks_set_trace")
 

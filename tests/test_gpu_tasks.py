@@ -82,13 +82,54 @@ def test_war_rewrite_after_reads():
     assert np.array_equal(Bh[1:-1], B2[1:-1])
 
 
-def test_no_barrier_between_constructs_trace():
-    """Pinned host arrays over 8 chunks whose last one is 100x larger: with
-    chunk-level dependencies the stencil of the small chunks starts while the
-    big chunk's map(to) is still running -- under the paper's taskgroup no loop
-    could start before every map(to) of the enter data had finished."""
-    small, big = 1 << 20, 100 << 20
-    sizes = [small] * 7 + [big]
+def test_no_barrier_between_constructs():
+    """No taskgroup between the constructs, shown deterministically: chunk 5's
+    stream is held (it waits on a host word) before its map(to); every other
+    chunk's whole chain -- map(to) of A and B, both stencil loops, map(from)
+    of C -- completes while chunk 5 has not even started (under the paper's
+    taskgroup no loop could run before every map(to) finished). Only the two
+    neighbours of chunk 5 could need its data: their halo element comes from
+    chunk 5's enter data, so they are held too -- and released with it."""
+    import time
+
+    n = 1 << 16
+    A = torch.empty(n, dtype=torch.float64, pin_memory=True).numpy()
+    A[:] = np.random.default_rng(1).normal(size=n)
+    Z = torch.zeros(n, dtype=torch.float64, pin_memory=True).numpy()
+    C = torch.full((n,), np.nan, dtype=torch.float64, pin_memory=True).numpy()
+    spread = P.Spread([0, 1], 1, n - 2, chunk=(n - 2 + 7) // 8)
+    ch = spread.chunks()
+    with P.SpreadTasks(spread, cuda_devices=[0, 0]) as q:
+        q.hold(5)
+        a = q.enter(A, lo_halo=1, hi_halo=1)
+        b = q.enter(Z, lo_halo=1, hi_halo=1)
+        c = q.enter(Z)
+        q.stencil3(a, b)
+        q.stencil3(b, c)
+        q.exit(c, C)
+        # chunks far from 5 finish while chunk 5 waits (their results land in C)
+        far = [k for k in range(8) if abs(k - 5) > 2]
+        deadline = time.time() + 30
+        done = lambda: all(not np.isnan(C[ch[k].start:ch[k].start + ch[k].size]).any() for k in far)  # noqa: E731
+        while not done() and time.time() < deadline:
+            time.sleep(0.01)
+        assert done(), "chunks away from the held one did not complete"
+        held = C[ch[5].start:ch[5].start + ch[5].size]
+        assert np.isnan(held).all(), "the held chunk ran"
+        q.release()
+        q.taskwait()
+    B = np.zeros(n)
+    B[1:-1] = O.stencil3(A)[1:-1]
+    Cref = np.zeros(n)
+    Cref[1:-1] = O.stencil3(B)[1:-1]
+    assert np.array_equal(C[1:-1], Cref[1:-1])
+
+
+def test_trace_records_follow_the_dependencies():
+    """The trace API: one record per chunk task, each chunk's loop after its own
+    map(to) of A and its map(from) after its loop (the chunk-level order; how
+    the copies of different chunks interleave is the copy engines' business)."""
+    sizes = [1 << 18] * 7 + [1 << 20]
     n = sum(sizes) + 2
     A = torch.empty(n, dtype=torch.float64, pin_memory=True).numpy()
     A[:] = np.random.default_rng(1).normal(size=n)
@@ -96,16 +137,19 @@ def test_no_barrier_between_constructs_trace():
     spread = P.Spread.with_sizes([0], 1, n - 2, sizes)
     with P.SpreadTasks(spread) as q:
         q.set_trace(True)
+        b = q.enter(None, n=n)  # map(alloc: B[...]): B is only written
         a = q.enter(A, lo_halo=1, hi_halo=1)
-        b = q.enter(Bh, lo_halo=1, hi_halo=1)
         q.stencil3(a, b)
         q.exit(b, Bh)
         tr = q.trace()
         q.taskwait()
-    enters = [(c, s, e) for c, k, s, e in tr if k == "enter"]
-    loops = [(c, s, e) for c, k, s, e in tr if k == "stencil3"]
-    assert len(enters) == 16 and len(loops) == 8
-    last_enter_end = max(e for _, _, e in enters)
-    assert min(s for _, s, _ in loops) < last_enter_end, (enters, loops)
+    rec = {}
+    for c, k, s0, e0 in tr:
+        rec.setdefault((c, k), []).append((s0, e0))
+    for c in range(8):
+        assert len(rec[(c, "enter")]) == 2 and len(rec[(c, "stencil3")]) == 1 and len(rec[(c, "exit")]) == 1
+        a_end = rec[(c, "enter")][1][1]
+        loop = rec[(c, "stencil3")][0]
+        assert loop[0] >= a_end and rec[(c, "exit")][0][0] >= loop[1]
     ref = O.stencil3(A)
     assert np.array_equal(Bh[1:-1], ref[1:-1])

@@ -103,3 +103,52 @@ def test_512cube_rest_lattice_fixed_point_and_zero_centre():
         X1, V1 = s.read_planes(200, 3)
     assert np.array_equal(X0, X1) and not V1.any()
     assert st.centre == (0.0, 0.0, 0.0) and st.vmax == 0.0 and st.nodes == 512 ** 3
+
+
+def test_512cube_full_state_and_every_step_stats_vs_full_oracle():
+    """The bench configuration at full size against the oracle run on the whole
+    512^3 grid (the -fopenmp build, bit-identical to the sequential oracle:
+    tests/test_oracle_omp.py): centre sums and vmax of each of 4 steps (two
+    K1_TB2 launches, both steps of each) and every element of the final X and V
+    bit for bit."""
+    n, steps = (512, 512, 512), 4
+    sp = P.SomierParams(n=n, seed=42)
+    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
+        assert s.kernel_in_use == P.K1_TB2
+        s.step(steps)
+        hist = s.stats_history(1, steps)
+        X, V = s.read()
+    st = O.init(O.Params(n=n, seed=42))
+    for t in range(steps):
+        st, ost, _, _ = O.run_timed(st, 1, omp=True)
+        assert hist[t].sums == ost.sums and hist[t].vmax2_bits == ost.vmax2_bits, t + 1
+    for c, (xo, vo) in enumerate(zip((st.x, st.y, st.z), (st.vx, st.vy, st.vz))):
+        assert np.array_equal(X[c], xo), "X component %d" % c
+        assert np.array_equal(V[c], vo), "V component %d" % c
+
+
+def test_256cube_100_steps_spread_2_and_4_vs_full_oracle():
+    """BASELINE configs[2] -- 256^3, 100 steps, spread over 2 and 4 list
+    positions (logical devices on one GPU: the cross-position exchange runs
+    exactly as between GPUs) -- every element of X and V and every step's
+    stats against the whole-grid oracle (-fopenmp build), bit for bit."""
+    n, steps = (256, 256, 256), 100
+    op = O.Params(n=n, seed=42)
+    st = O.init(op)
+    ref = []
+    for _ in range(steps):
+        st, ost, _, _ = O.run_timed(st, 1, omp=True)
+        ref.append(ost)
+    for devs in ([0, 1], [0, 1, 2, 3]):
+        sp = P.SomierParams(n=n, seed=42)
+        with P.Somier(P.Spread(devs, 1, n[0] - 2), sp, cuda_devices=[0] * len(devs)) as s:
+            s.step(steps)
+            hist = s.stats_history(steps - P.STATS_HISTORY + 1, P.STATS_HISTORY) if steps > P.STATS_HISTORY \
+                else s.stats_history(1, steps)
+            X, V = s.read()
+        first = steps - len(hist) + 1
+        for i, h in enumerate(hist):
+            r = ref[first - 1 + i]
+            assert h.sums == r.sums and h.vmax2_bits == r.vmax2_bits, (devs, first + i)
+        for c, (xo, vo) in enumerate(zip((st.x, st.y, st.z), (st.vx, st.vy, st.vz))):
+            assert np.array_equal(X[c], xo) and np.array_equal(V[c], vo), (devs, c)

@@ -117,3 +117,15 @@ def test_our_arm_four_ranks_same_fields_as_one():
     assert set(d4["e2e"]) == set(d1["e2e"]) and set(d4["halo"]) == set(d1["halo"])
     assert len(d4["roofline"]["per_rank"]) == 4 and d4["verify"]["ok"] and d4["n_gpus"] == 4
 
+
+
+@pytest.mark.gpu
+def test_our_arm_odd_steps_with_two_step_kernel():
+    """An odd K with K1_TB2 (two steps per launch): the last launch is a
+    one-step launch; the line reports K steps and a consistent roofline."""
+    lines, _ = _run(["bench.py", "--grid", "64", "--kernel", "tb2", "--steps", "5", "--warmup", "3",
+                     "--no-cpu-baseline", "--no-e2e", "--sustained-s", "0"])
+    d = json.loads(lines[0])
+    _check_common(d, 1, 5, 3)
+    assert d["config"]["kernel"] == "K1_TB2" and d["gpu_launches"] == 3
+    assert 90 < d["roofline"]["algorithmic_bytes_per_node_update"] < 110

@@ -97,3 +97,20 @@ def test_capi_exposes_every_entry_point_under_its_c_name():
     with pytest.raises(P.SpreadError):
         capi.spread_create(devs, 0, 1, 14, 0, 4, ctypes.byref(h))  # no devices
     assert capi.somier_version()
+
+
+def test_host_grid_size_is_checked():
+    """The binding refuses a host grid whose element count differs from what
+    the C side reads or writes (n0*n1*n2 per grid) instead of letting C run off
+    its end."""
+    import numpy as np
+    import pytest as _pytest
+
+    from paper_conf_ipps_torresft22_b200 import somier as S
+
+    ok = np.zeros(24)
+    assert S._dptr(ok, 24) is not None
+    with _pytest.raises(ValueError):
+        S._dptr(np.zeros(23), 24)
+    with _pytest.raises(TypeError):
+        S._dptr(np.zeros(24, dtype=np.float32), 24)

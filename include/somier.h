@@ -49,16 +49,17 @@ extern "C" {
 
 /* K1 implementations (all compute bit-identical results). */
 typedef enum {
-    SOMIER_K1_AUTO = 0,      /* the fastest measured: SOMIER_K1_TB2 for a handle with
-                                one local chunk of a grid of >= 3e6 nodes whose device
-                                has room for it, else SOMIER_K1_MARCH2
+    SOMIER_K1_AUTO = 0,      /* the fastest measured: SOMIER_K1_TB2 when every chunk
+                                has >= 3e6 nodes and the devices have room for its
+                                deeper slabs, else SOMIER_K1_MARCH2
                                 (somier_kernel_in_use tells which)                    */
     SOMIER_K1_DIRECT = 1,    /* one thread per node, 6 springs from global loads       */
     SOMIER_K1_MARCH = 2,     /* plane-marching, smem-staged, 3 springs/node with reuse */
     SOMIER_K1_MARCH2 = 3,    /* as MARCH with two rows per warp (32 x 16 tiles)        */
-    SOMIER_K1_TB2 = 4        /* two time steps per pass over HBM (temporal blocking);
-                                only for a handle with a single local chunk (one slab,
-                                no halo exchange), else as MARCH2; V double-buffered  */
+    SOMIER_K1_TB2 = 4        /* two time steps per pass over HBM (temporal blocking),
+                                deep-halo exchange between chunks (every chunk >= 2
+                                planes when there are several, else MARCH2); V
+                                double-buffered; both steps' stats computed          */
 } somier_kernel;
 
 typedef struct {
@@ -239,10 +240,10 @@ spread_status somier_step_count(somier_t h, int64_t* steps);
 spread_status somier_local_chunks(somier_t h, int64_t* nchunks);
 spread_status somier_launch_count(somier_t h, int64_t* launches);
 
-/* The K1 implementation multi-step calls of this handle run (a somier_kernel
- * value; never SOMIER_K1_AUTO): AUTO and TB2 resolve at somier_init. A handle
- * on K1_TB2 still runs a single step (odd step count or odd start) with
- * K1_MARCH2. EINVAL on NULL arguments. */
+/* The K1 implementation this handle runs (a somier_kernel value; never
+ * SOMIER_K1_AUTO): AUTO and TB2 resolve at somier_init. A K1_TB2 handle runs a
+ * leftover single step (odd step count) with the same kernel in one-step mode.
+ * EINVAL on NULL arguments. */
 spread_status somier_kernel_in_use(somier_t h, int32_t* kernel);
 
 /*

@@ -600,6 +600,8 @@ def run_ours(a):
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # host-side waits (no NCCL kernel spinning on the GPUs rank 0 drives in the e2e)
+        cpu_group = dist.new_group(backend="gloo") if not a.share_gpu else None
 
     def all_max(x, dtype=torch.float64):
         t = torch.tensor([x], device=dev, dtype=dtype)
@@ -764,6 +766,8 @@ def run_ours(a):
     if not a.no_e2e and rank == 0:
         cuda_devs = [0] * world if a.share_gpu else list(range(world))
         e2e = e2e_stream(n, params, list(range(world)), a, two_step=(in_use == P.K1_TB2), cuda_devices=cuda_devs)
+    if multi:
+        torch.distributed.barrier(group=cpu_group)  # the other ranks wait on the host
     barrier()
 
     verify = run_verify(a, n, params, world, rank, local, multi) if a.verify else None

@@ -67,34 +67,12 @@ constexpr int kYComp = kRows * kTK;                         // X_{t+1} of one R1
 #define TB2_VSTAGES 2
 #endif
 constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
-// where step t+1's stats are accumulated: 2 in S1 right after its kick-drift
-// (default, measured fastest: 6.38e10 node-updates/s at 512^3 vs 6.23 / 6.33
-// for 0 = after S2 / 1 = before S2's forces), 9 not at all (A/B of their cost
-// only: stats of every second step, 7.2e10)
-#ifndef TB2_ST1_MODE
-#define TB2_ST1_MODE 2
-#endif
-// V_{t+1} handed from S1 to the next iteration's S2 through shared memory (1)
-// instead of a register carry (0)
-#ifndef TB2_V1_SMEM
-#define TB2_V1_SMEM 0
-#endif
-#if TB2_V1_SMEM && (TB2_S2_BF || TB2_ST1_MODE != 2)
-#error "TB2_V1_SMEM needs the branchy S2 and the S1 placement of step t+1's stats"
-#endif
-// the last step's stats accumulators in shared memory too (else registers;
-// 5.84-5.94e10: the LSU round trips cost more than the freed registers)
-#ifndef TB2_ST_SMEM
-#define TB2_ST_SMEM 0
-#endif
-// strides from the parameter bank (1) or recomputed from the geometry (0)
-#ifndef TB2_ADDR
-#define TB2_ADDR 1
-#endif
-// S2's results and stats without per-node branches around the stats (both
-// nodes' results live at once: spills, 5.07e10 -- not the default)
-#ifndef TB2_S2_BF
-#define TB2_S2_BF 0
+// Step t+1's stats are accumulated in S1 right after its kick-drift, into
+// thread-private shared-memory slots (measured fastest of the placements,
+// DESIGN.md §6). TB2_MID_STATS=0 skips them -- an A/B of their cost only (the
+// stats of every second step, round 1's kernel), not a product configuration.
+#ifndef TB2_MID_STATS
+#define TB2_MID_STATS 1
 #endif
 constexpr int kMinSegPlanes = 4, kMaxSegPlanes = 256;
 static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
@@ -113,12 +91,6 @@ struct __align__(16) Smem {
     // step t+1's stats accumulators, thread-private (registers are full):
     // [0..2] = (sum bits(hd), sum bits(ld)) of x, y, z; [3] = (max v.v, unused)
     ulonglong2 acc1[4][kThreads];
-#if TB2_ST_SMEM
-    ulonglong2 acc2[4][kThreads];  // the last step's, same layout (TB2_ST_SMEM variant)
-#endif
-#if TB2_V1_SMEM
-    double v1[2][3][kYComp];       // V_{t+1} of R1 by plane parity (TB2_V1_SMEM variant)
-#endif
 };
 
 struct Tb2Params {
@@ -213,11 +185,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const bool kown = lane >= 1 && lane <= kOK && k <= g.n2 - 2;   // interior k columns only
     const bool ownA = kown && rA >= 1 && jA < g.n1;               // rows 1 .. kRows-2
     const bool ownB = kown && rB <= kRows - 2 && jB < g.n1;
-#if TB2_ADDR
     const int64_t cs = tp.cs, ps = tp.ps;
-#else
-    const int64_t cs = g.comp_stride(), ps = g.plane_stride();
-#endif
     const int64_t offA = ownA ? (int64_t)jA * g.ld + k : 0, offB = ownB ? (int64_t)jB * g.ld + k : 0;
 
     // Tile-border springs of S1 (row above R1 -> R1 row 0: gbj; column left of
@@ -285,13 +253,9 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
         for (int c = 0; c < 3; c++) {
             const double hda = __fma_rn(xsa[c], 0x1p28, kRoundC), hdb = __fma_rn(xsb[c], 0x1p28, kRoundC);
-#ifdef STATS_ONEWORD_TIMING
-            const double lda = kRoundC, ldb_ = kRoundC;
-#else
             const double ra = __fma_rn(xsa[c], 0x1p28, -__dsub_rn(hda, kRoundC));
             const double rb = __fma_rn(xsb[c], 0x1p28, -__dsub_rn(hdb, kRoundC));
             const double lda = __fma_rn(ra, 0x1p32, kRoundC), ldb_ = __fma_rn(rb, 0x1p32, kRoundC);
-#endif
             const unsigned long long ha = ownA ? (unsigned long long)__double_as_longlong(hda) : 0ull;
             const unsigned long long hb = ownB ? (unsigned long long)__double_as_longlong(hdb) : 0ull;
             const unsigned long long la = ownA ? (unsigned long long)__double_as_longlong(lda) : 0ull;
@@ -309,33 +273,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     };
 
     // the last step's stats of one node (hasv: an interior node, v enters vmax)
-#if TB2_ST_SMEM
-    unsigned int nst = 0;
-    for (int c = 0; c < 4; c++) sm.acc2[c][tid] = make_ulonglong2(0ull, 0ull);
-    auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
-        const double xs[3] = {x.x, x.y, x.z};
-#pragma unroll
-        for (int c = 0; c < 3; c++) {
-            const double hd = __fma_rn(xs[c], 0x1p28, kRoundC);
-            const double r = __fma_rn(xs[c], 0x1p28, -__dsub_rn(hd, kRoundC));
-            ulonglong2 o = sm.acc2[c][tid];
-            o.x += (unsigned long long)__double_as_longlong(hd);
-            o.y += (unsigned long long)__double_as_longlong(__fma_rn(r, 0x1p32, kRoundC));
-            sm.acc2[c][tid] = o;
-        }
-        nst++;
-        if (hasv) {
-            const double v2 = dot_self(v);
-            const double vm = __longlong_as_double((long long)sm.acc2[3][tid].x);
-            if (v2 > vm || v2 != v2) sm.acc2[3][tid].x = (unsigned long long)__double_as_longlong(v2);
-        }
-    };
-#else
     auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
         st.add_position(x);
         if (hasv) st.add_velocity(v);
     };
-#endif
 
     // One plane of the march. kFull: a steady-state plane (p+1 exists, p is
     // updated by S1, q = p-1 is an S2 output plane): no conditions, no
@@ -393,21 +334,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                 kick_drift<kUnitMass>(F, a.M, a.dt, v1B, xcB, x1B);
             }
         }
-#if TB2_ST1_MODE == 2
         // step t+1's stats right where S1 produced them (plane p, if an output plane of this segment)
-        if (kTwo && p >= max(pb, tp.stats_lo) && p < min(pe, tp.stats_hi)) acc1_update(x1A, x1B, v1A, v1B);
-#endif
-#if TB2_V1_SMEM
-        {
-            double* vv = sm.v1[par][0];
-            vv[yA] = v1A.x;
-            vv[yA + kYComp] = v1A.y;
-            vv[yA + 2 * kYComp] = v1A.z;
-            vv[yB] = v1B.x;
-            vv[yB + kYComp] = v1B.y;
-            vv[yB + 2 * kYComp] = v1B.z;
-        }
-#endif
+        if (kTwo && TB2_MID_STATS && p >= max(pb, tp.stats_lo) && p < min(pe, tp.stats_hi))
+            acc1_update(x1A, x1B, v1A, v1B);
         {
             double* y = sm.y[par][0];
             y[yA] = x1A.x;
@@ -447,37 +376,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         // ---- S2 forces -> X_{t+2}, V_{t+2} of R2, plane q (one-step mode: X_{t+1}, V_{t+1} of S1)
         const bool sq = kFull ? (q >= tp.stats_lo && q < tp.stats_hi) : (out2 && q >= tp.stats_lo && q < tp.stats_hi);
-#if TB2_ST1_MODE == 1
-        if (kTwo && sq) acc1_update(xqA, xqB, v1pA, v1pB);
-#endif
-#if TB2_S2_BF
-        if (out2) {
-            // results of the two nodes (a fixed node keeps X, and V = 0)
-            Vec3 x2A = xqA, v2A = v1pA, x2B = xqB, v2B = v1pB;
-            if (kTwo) {
-                if (ownA && intA) {
-                    const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
-                    const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
-                    kick_drift<kUnitMass>(F, a.M, a.dt, v2A, xqA, x2A);
-                }
-                if (ownB && intB) {
-                    const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
-                    kick_drift<kUnitMass>(F, a.M, a.dt, v2B, xqB, x2B);
-                }
-            }
-            if (ownA && intA) store_out(q, offA, x2A, v2A);
-            if (ownB && intB) store_out(q, offB, x2B, v2B);
-            if (sq) st.add_pair(x2A, x2B, v2A, v2B, ownA, ownB);
-        }
-#else
         if (out2) {
             if (ownA) {
                 if (intA) {
-#if TB2_V1_SMEM
-                    Vec3 v2 = ldb(sm.v1[par ^ 1][0], yA, kYComp), x2 = xqA;
-#else
                     Vec3 v2 = v1pA, x2 = xqA;
-#endif
                     if (kTwo) {
                         const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
@@ -491,11 +393,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             }
             if (ownB) {
                 if (intB) {
-#if TB2_V1_SMEM
-                    Vec3 v2 = ldb(sm.v1[par ^ 1][0], yB, kYComp), x2 = xqB;
-#else
                     Vec3 v2 = v1pB, x2 = xqB;
-#endif
                     if (kTwo) {
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
                         kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
@@ -507,10 +405,6 @@ __global__ void __launch_bounds__(kThreads, 1)
                 }
             }
         }
-#endif
-#if TB2_ST1_MODE == 0
-        if (kTwo && sq) acc1_update(xqA, xqB, v1pA, v1pB);
-#endif
         // border springs of the next plane (X_t(p+1) is resident until barrier #1 of iteration p+1)
         if (p + 1 <= border_last) border_springs(p + 1);
         carry1A = gpi1A;
@@ -519,10 +413,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         xcB = niB;
         carry2A = gpi2A;
         carry2B = gpi2B;
-#if !TB2_V1_SMEM
         v1pA = v1A;
         v1pB = v1B;
-#endif
     };
     using F0 = std::integral_constant<bool, false>;
     using F1 = std::integral_constant<bool, true>;
@@ -540,16 +432,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     if (p <= hi) body(F1{}, P0{}, p++);
     for (; p <= pe; p++) body(F0{}, PN{}, p);
-#if TB2_ST_SMEM
-    for (int c = 0; c < 3; c++) {
-        st.hb[c] = sm.acc2[c][tid].x;
-        st.lb[c] = sm.acc2[c][tid].y;
-    }
-    st.vmax2 = __longlong_as_double((long long)sm.acc2[3][tid].x);
-    st.n = nst;
-#endif
     block_accumulate(st, sm.scratch, slots.fin);
-    if (kTwo && TB2_ST1_MODE != 9) {
+    if (kTwo && TB2_MID_STATS) {
 #ifndef STATS_FP64_ACC
         NodeStats st1;
         for (int c = 0; c < 3; c++) {

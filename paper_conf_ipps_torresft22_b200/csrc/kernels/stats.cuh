@@ -52,14 +52,10 @@ struct NodeStats {
     }
     __device__ __forceinline__ void add_coord(int c, double x) {
         const double hd = __fma_rn(x, 0x1p28, kRoundC);
-#ifdef STATS_ONEWORD_TIMING  // timing experiment only: one quantisation word (wrong sums)
-        hb[c] += (unsigned long long)__double_as_longlong(hd);
-#else
         const double r = __fma_rn(x, 0x1p28, -__dsub_rn(hd, kRoundC));
         const double ld = __fma_rn(r, 0x1p32, kRoundC);
         hb[c] += (unsigned long long)__double_as_longlong(hd);
         lb[c] += (unsigned long long)__double_as_longlong(ld);
-#endif
     }
     __device__ __forceinline__ void add_position(const Vec3& x) {
         add_coord(0, x.x);
@@ -75,31 +71,6 @@ struct NodeStats {
         add_coord(2, x.z);
     }
     __device__ __forceinline__ void copy_count(const NodeStats& o) { n = o.n; }
-    // Two nodes at once, branch-free: a node whose flag is false contributes
-    // nothing (its addends are selected to 0). A fixed node passes v = 0.
-    __device__ __forceinline__ void add_pair(const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb, bool oa,
-                                             bool ob) {
-        const double xsa[3] = {xa.x, xa.y, xa.z}, xsb[3] = {xb.x, xb.y, xb.z};
-#pragma unroll
-        for (int c = 0; c < 3; c++) {
-            const double hda = __fma_rn(xsa[c], 0x1p28, kRoundC), hdb = __fma_rn(xsb[c], 0x1p28, kRoundC);
-            const double ra = __fma_rn(xsa[c], 0x1p28, -__dsub_rn(hda, kRoundC));
-            const double rb = __fma_rn(xsb[c], 0x1p28, -__dsub_rn(hdb, kRoundC));
-            const double lda = __fma_rn(ra, 0x1p32, kRoundC), ldb = __fma_rn(rb, 0x1p32, kRoundC);
-            hb[c] += (oa ? (unsigned long long)__double_as_longlong(hda) : 0ull) +
-                     (ob ? (unsigned long long)__double_as_longlong(hdb) : 0ull);
-            lb[c] += (oa ? (unsigned long long)__double_as_longlong(lda) : 0ull) +
-                     (ob ? (unsigned long long)__double_as_longlong(ldb) : 0ull);
-        }
-        n += (oa ? 1u : 0u) + (ob ? 1u : 0u);
-        const double v2a = oa ? dot_self(va) : 0.0, v2b = ob ? dot_self(vb) : 0.0;
-        vmax2 = (v2a > vmax2 || v2a != v2a) ? v2a : vmax2;
-        vmax2 = (v2b > vmax2 || v2b != v2b) ? v2b : vmax2;
-    }
-    __device__ __forceinline__ void add_velocity(const Vec3& v) {
-        const double v2 = dot_self(v);
-        vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
-    }
     // exact int128 value of sum q(x) for coordinate c
     __device__ __forceinline__ __int128 sum(int c) const {
         const unsigned long long cb = (unsigned long long)__double_as_longlong(kRoundC) * n;

@@ -99,3 +99,26 @@ def test_auto_kernel_resolution():
         assert s.kernel_in_use == P.K1_MARCH2  # small grid: TB2's tiles fill too few waves
     with P.Somier(P.Spread([0], 1, 10), P.SomierParams(n=(12, 10, 36), kernel=P.K1_MARCH)) as s:
         assert s.kernel_in_use == P.K1_MARCH
+
+
+def test_launch_timing_instrumentation_keeps_results():
+    """somier_set_timing: every launch bracketed by events (graph replay off);
+    take_timing reports one record per launch with plausible times, and the
+    results stay bit-identical to an untimed run."""
+    n = (40, 24, 37)
+    sp = P.SomierParams(n=n, seed=5, kernel=P.K1_TB2)
+    with P.Somier(P.Spread([0, 1], 1, n[0] - 2), sp, cuda_devices=[0, 0]) as s:
+        s.set_timing(True)
+        s.step(9)
+        t = s.take_timing()
+        s.set_timing(False)
+        s.step(3)
+        X, V = s.read()
+        st = s.stats()
+    assert t["launches"] == 2 * 5  # two positions x (4 two-step + 1 one-step launches)
+    assert t["kernel_ms"] > 0 and t["wait_ms"] >= 0 and t["kernel_max_ms"] <= t["kernel_ms"]
+    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as r:
+        r.step(12)
+        Xr, Vr = r.read()
+        sr = r.stats()
+    assert np.array_equal(X, Xr) and np.array_equal(V, Vr) and st.sums == sr.sums

@@ -71,6 +71,10 @@ struct NodeStats {
         add_coord(2, x.z);
     }
     __device__ __forceinline__ void copy_count(const NodeStats& o) { n = o.n; }
+    __device__ __forceinline__ void add_velocity(const Vec3& v) {
+        const double v2 = dot_self(v);
+        vmax2 = (v2 > vmax2 || v2 != v2) ? v2 : vmax2;
+    }
     // exact int128 value of sum q(x) for coordinate c
     __device__ __forceinline__ __int128 sum(int c) const {
         const unsigned long long cb = (unsigned long long)__double_as_longlong(kRoundC) * n;

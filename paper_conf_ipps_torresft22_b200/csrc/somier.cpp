@@ -717,22 +717,26 @@ spread_status nccl_exchange(somier_t h, bool tb2, int xo, int vo) {
             size_t bytes;
         };
         // U: lo -> hi, D: hi -> lo (X planes, then the V plane on K1_TB2 handles)
-        std::vector<Msg> U, D;
+        Msg U[2], D[2];
+        int nm = 1;
         if (tb2) {
-            U = {{lo.x(xo) + lo.size * ps, hi.x(xo), 2 * pb}, {lo.v(vo) + lo.size * ps, hi.v(vo), pb}};
-            D = {{hi.x(xo) + 2 * ps, lo.x(xo) + (lo.size + 2) * ps, 2 * pb},
-                 {hi.v(vo) + ps, lo.v(vo) + (lo.size + 1) * ps, pb}};
+            U[0] = {lo.x(xo) + lo.size * ps, hi.x(xo), 2 * pb};
+            U[1] = {lo.v(vo) + lo.size * ps, hi.v(vo), pb};
+            D[0] = {hi.x(xo) + 2 * ps, lo.x(xo) + (lo.size + 2) * ps, 2 * pb};
+            D[1] = {hi.v(vo) + ps, lo.v(vo) + (lo.size + 1) * ps, pb};
+            nm = 2;
         } else {
-            U = {{lo.xs(xo) + lo.size * ps, hi.xs(xo), pb}};
-            D = {{hi.xs(xo) + ps, lo.xs(xo) + (lo.size + 1) * ps, pb}};
+            U[0] = {lo.xs(xo) + lo.size * ps, hi.xs(xo), pb};
+            D[0] = {hi.xs(xo) + ps, lo.xs(xo) + (lo.size + 1) * ps, pb};
         }
-        for (const Msg& m : U) {
-            if (lo.local) ck(L.Send(m.src, m.bytes, paper::kNcclUint8, hi.pos, h->comms[lo.pos], h->stream_of(lo)), "ncclSend");
-            if (hi.local) ck(L.Recv(m.dst, m.bytes, paper::kNcclUint8, lo.pos, h->comms[hi.pos], h->stream_of(hi)), "ncclRecv");
+        const paper::ncclComm clo = h->comms[(size_t)lo.pos], chi = h->comms[(size_t)hi.pos];
+        for (int m = 0; m < nm; m++) {
+            if (lo.local) ck(L.Send(U[m].src, U[m].bytes, paper::kNcclUint8, hi.pos, clo, h->stream_of(lo)), "ncclSend");
+            if (hi.local) ck(L.Recv(U[m].dst, U[m].bytes, paper::kNcclUint8, lo.pos, chi, h->stream_of(hi)), "ncclRecv");
         }
-        for (const Msg& m : D) {
-            if (hi.local) ck(L.Send(m.src, m.bytes, paper::kNcclUint8, lo.pos, h->comms[hi.pos], h->stream_of(hi)), "ncclSend");
-            if (lo.local) ck(L.Recv(m.dst, m.bytes, paper::kNcclUint8, hi.pos, h->comms[lo.pos], h->stream_of(lo)), "ncclRecv");
+        for (int m = 0; m < nm; m++) {
+            if (hi.local) ck(L.Send(D[m].src, D[m].bytes, paper::kNcclUint8, lo.pos, chi, h->stream_of(hi)), "ncclSend");
+            if (lo.local) ck(L.Recv(D[m].dst, D[m].bytes, paper::kNcclUint8, hi.pos, clo, h->stream_of(lo)), "ncclRecv");
         }
     }
     ck(L.GroupEnd(), "ncclGroupEnd");

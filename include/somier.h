@@ -15,9 +15,11 @@
  * over all nodes by an exact int128 fixed-point sum, vmax = max |v|.
  *
  * One call of somier_step = the paper's five kernels fused into ONE sm_100a
- * kernel launch per chunk; the halo exchange is fused into the same kernel
- * (boundary planes are stored straight into the neighbour chunk's halo slot,
- * through NVLink P2P / CUDA IPC when the neighbour is on another GPU).
+ * kernel launch per chunk (K1_TB2: per two steps); the halo exchange is fused
+ * into the same kernel by default (boundary planes are stored straight into
+ * the neighbour chunk's halo slot, through NVLink P2P / CUDA IPC when the
+ * neighbour is on another GPU; somier_params.exchange selects the unfused copy
+ * or NCCL routes instead).
  *
  * Lifetime (mirrors the data directives):
  *   somier_init        ~ target enter data spread map(to: X[start-1:size+2], V[start:size])
@@ -25,6 +27,7 @@
  *   somier_step        ~ target spread teams distribute parallel for ... nowait
  *   somier_sync        ~ taskgroup / taskwait
  *   somier_stats       ~ the "centers" result of the last completed step
+ *   somier_stats_history ~ the "centers" of every step (the last 126)
  *   somier_read        ~ target exit data spread map(from: X[start:size], V[start:size])
  *   somier_destroy     ~ end of the data region
  *

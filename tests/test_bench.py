@@ -43,8 +43,11 @@ def test_reference_arm_json_line():
     d = json.loads(lines[0])
     _check_common(d, 1, 2, 3)
     assert d["impl"] == "reference"
-    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
-    assert d["cpu_baseline"]["value"] == d["value"]
+    cb = d["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] == 1 and cb["value"] == d["value"]
+    # the C-side timer, the CPU model, nproc and "1 of N cores"
+    assert cb["cpu_model"] and cb["nproc"] >= 1 and cb["cores_label"] == "1 of %d cores" % cb["nproc"]
+    assert cb["seconds"] > 0 and cb["steps"] == 2 and "oracle_run_timed" in cb["sample"]
     assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
 
 

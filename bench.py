@@ -741,6 +741,9 @@ def run_ours(a):
     traffic, traffic_src = load_traffic(n, kname) if len(my_chunks) == 1 and c0.size == n[0] - 2 else (None, None)
     copy_gbs = sustained_copy(local, stream) if a.copy_check else None
     st = PD.gather_stats(s) if multi else s.stats()
+    # every step's centres are kept (somier_stats_history): the last few, exact global values
+    last = (PD.gather_stats_history(s, st.step - 3, 4) if multi else s.stats_history(st.step - 3, 4)) \
+        if st.step >= 4 else []
     roof = roofline_obj(achieved, peak, peak_src, traffic, traffic_src, k1_ms, kname, alg, alg_step, nu_launch,
                         per_call, step_dist, copy_gbs, fp64_achieved / fp64_peak)
     # per rank: this rank's launch time, flag-wait time and kernel time
@@ -800,6 +803,7 @@ def run_ours(a):
             "clocks": clk, "gpu_launches": launches, "e2e": e2e, "cpu_baseline": cpu,
             "halo": halo, "sustained": sustained,
             "stats": {"step": st.step, "centre": st.centre, "vmax": st.vmax, "every_step": True,
+                      "last_steps": [{"step": h.step, "centre": h.centre, "vmax": h.vmax} for h in last],
                       "note": "centres and vmax of every step are computed inside the timed region "
                               "(somier_stats_history reads any of the last %d)" % P.STATS_HISTORY},
         }

@@ -82,6 +82,8 @@ def test_our_arm_json_line_one_gpu():
     assert d["verify"]["ok"] and d["verify"]["nodes_checked"] > 0
     assert d["sustained"]["steps"] >= 2 and d["sustained"]["value"] > 0
     assert d["stats"]["every_step"] is True
+    steps = [h["step"] for h in d["stats"]["last_steps"]]
+    assert steps == list(range(d["stats"]["step"] - 3, d["stats"]["step"] + 1))
 
 
 @pytest.mark.gpu

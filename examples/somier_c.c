@@ -43,7 +43,7 @@ int main(int argc, char** argv) {
         printf("chunk %lld: device %d, omp_spread_start %lld, omp_spread_size %lld, map(to: X[%lld:%lld])\n",
                (long long)c, id, (long long)start, (long long)size, (long long)first, (long long)len);
     }
-    somier_params p = {{n, n, n}, 1.0, 1.0, 10.0, 1.0, 1e-3, 0.05, 42, SOMIER_K1_AUTO, SOMIER_EXCHANGE_FUSED};
+    somier_params p = {{n, n, n}, 1.0, 1.0, 10.0, 1.0, 1e-3, 0.05, 42, SOMIER_K1_AUTO, SOMIER_EXCHANGE_FUSED, SOMIER_MATH_EXACT, 0};
     somier_t h;
     CHECK(somier_init(sp, &p, &h));
     CHECK(spread_destroy(sp)); /* the handle keeps its own copy */

@@ -65,6 +65,24 @@ typedef enum {
                                 double-buffered; both steps' stats computed          */
 } somier_kernel;
 
+/* Operation order of the step's fp64 arithmetic (reading S22).
+ * north_star's correctness bar: positions and velocities within a max relative
+ * error of 1e-10 of the oracle after 100 steps, "FMA contraction the only
+ * allowed difference", partitioned runs bit-identical to the 1-GPU run.
+ *   EXACT: every operation rounded separately in the oracle's order (reading
+ *          S13): the state and the stats are bit-identical to the oracle.
+ *   FMA:   the spring's d.d as fma(dz, dz, fma(dy, dy, dx*dx)) and the
+ *          semi-implicit Euler update as v' = fma(a, h, v), x' = fma(v', h, x)
+ *          (12 fewer fp64 operations per node-update, 108 -> 96); everything
+ *          else, the stats included, unchanged. Within the 1e-10 bar of the
+ *          oracle, and still bit-identical across kernels, chunkings, device
+ *          lists, schedules and the host-streamed mode, because every kernel
+ *          evaluates a node with the same contracted expressions.          */
+typedef enum {
+    SOMIER_MATH_EXACT = 0,
+    SOMIER_MATH_FMA = 1
+} somier_math;
+
 typedef struct {
     int64_t n[3];        /* nodes per dimension (i outermost, k contiguous); each >= 3        */
     double spacing;      /* rest-lattice spacing                                               */
@@ -76,6 +94,8 @@ typedef struct {
     uint64_t seed;       /* SplitMix64 seed of the initial displacement (reading S7)           */
     int32_t kernel;      /* somier_kernel                                                      */
     int32_t exchange;    /* somier_exchange: how boundary planes reach the neighbour chunks    */
+    int32_t math;        /* somier_math: operation order of the step's fp64 arithmetic          */
+    int32_t reserved;    /* must be 0                                                          */
 } somier_params;
 
 /* The halo exchange between chunks on different streams (devices / processes),

@@ -8,13 +8,14 @@ This package is the Python binding (argument marshalling only).
 """
 from . import _native, capi
 from ._native import (EXCHANGE_COPY, EXCHANGE_FUSED, EXCHANGE_NCCL, K1_AUTO, K1_DIRECT, K1_MARCH, K1_MARCH2,
-                      K1_TB2, SCHED_DYNAMIC, SCHED_STATIC, STATS_HISTORY, SpreadError)
+                      K1_TB2, MATH_EXACT, MATH_FMA, SCHED_DYNAMIC, SCHED_STATIC, STATS_HISTORY, SpreadError)
 from .somier import Somier, SomierParams, SomierStream, Stats, combine_stats
 from .spread import Chunk, Spread, SpreadTasks
 
 __all__ = ["capi", "Spread", "SpreadTasks", "Chunk", "Somier", "SomierParams", "SomierStream", "Stats",
            "combine_stats", "SpreadError", "K1_AUTO", "K1_DIRECT", "K1_MARCH", "K1_MARCH2", "K1_TB2",
-           "SCHED_STATIC", "SCHED_DYNAMIC", "EXCHANGE_FUSED", "EXCHANGE_COPY", "EXCHANGE_NCCL", "STATS_HISTORY",
+           "SCHED_STATIC", "SCHED_DYNAMIC", "EXCHANGE_FUSED", "EXCHANGE_COPY", "EXCHANGE_NCCL", "MATH_EXACT", "MATH_FMA",
+           "STATS_HISTORY",
            "version"]
 
 

@@ -18,6 +18,8 @@ LIB_PATH = os.environ.get("SOMIER_LIB") or os.path.join(_HERE, "libsomier.so")
 OK, EINVAL, ENODEV, ENOMEM, ECUDA, ENCCL, ENOTSUP, ESTATE = 0, -1, -2, -3, -4, -5, -6, -7
 # somier_exchange
 EXCHANGE_FUSED, EXCHANGE_COPY, EXCHANGE_NCCL = 0, 1, 2
+# somier_math
+MATH_EXACT, MATH_FMA = 0, 1
 # spread_sched
 SCHED_STATIC, SCHED_DYNAMIC = 0, 1
 # spread_map_type
@@ -49,6 +51,8 @@ class somier_params(ctypes.Structure):
         ("seed", ctypes.c_uint64),
         ("kernel", ctypes.c_int32),
         ("exchange", ctypes.c_int32),
+        ("math", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
     ]
 
 

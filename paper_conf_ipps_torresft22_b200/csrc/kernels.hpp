@@ -7,6 +7,7 @@
 // three component-planar n1 x ld blocks (x, then y, then z), each row
 // ld >= n2 doubles (ld a multiple of 32: 256-byte aligned rows).
 #pragma once
+#include <type_traits>
 #include <cstdint>
 
 #include <cuda_runtime.h>
@@ -67,6 +68,9 @@ struct StepArgs {
     // Host-streamed mode: x_nxt is a fresh buffer, so fixed face nodes of the
     // owned planes are copied into it too (resident mode leaves them in place).
     int write_fixed;
+    // SOMIER_MATH_FMA: the step's arithmetic with the FMA contractions of
+    // node_math.cuh (kFma); 0 = uncontracted (the oracle's operation order).
+    int fma;
     // K1_MARCH2: launch with programmatic stream serialization (PDL): the
     // kernel's prologue (barrier init, tensor-map prefetch) overlaps the tail
     // of the previous kernel on the stream; every thread executes
@@ -81,6 +85,19 @@ struct InitArgs {
     double spacing, amplitude;
     uint64_t seed;
 };
+
+// Host-side: calls f(std::integral_constant<bool, b>...) so that launchers
+// turn runtime flags into kernel template arguments without spelling out
+// every combination.
+template <class F>
+inline void dispatch_bools(F&& f) { f(); }
+template <class F, class... B>
+inline void dispatch_bools(F&& f, bool b0, B... rest) {
+    if (b0)
+        dispatch_bools([&](auto... v) { f(std::true_type{}, v...); }, rest...);
+    else
+        dispatch_bools([&](auto... v) { f(std::false_type{}, v...); }, rest...);
+}
 
 enum class K1Variant { Direct = 1, March = 2, March2 = 3 };
 

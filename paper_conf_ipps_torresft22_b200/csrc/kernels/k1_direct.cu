@@ -14,7 +14,7 @@ namespace {
 
 constexpr int kBX = 32, kBY = 8;
 
-template <bool kUnitMass>
+template <bool kUnitMass, bool kFma>
 __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
     __shared__ WarpStats scratch[kBX * kBY / 32];
     const SlabGeom& g = a.g;
@@ -34,17 +34,17 @@ __global__ void __launch_bounds__(kBX* kBY) k1_direct_kernel(StepArgs a) {
         const bool interior = j >= 1 && j < g.n1 - 1 && k >= 1 && k < g.n2 - 1;
         if (interior) {
             auto ld3 = [&](const double* q) { return Vec3{q[0], q[cs], q[2 * cs]}; };
-            const Vec3 gmi = spring_force(xp, ld3(xc - ps), a.K, a.L);
-            const Vec3 gpi = spring_force(xp, ld3(xc + ps), a.K, a.L);
-            const Vec3 gmj = spring_force(xp, ld3(xc - g.ld), a.K, a.L);
-            const Vec3 gpj = spring_force(xp, ld3(xc + g.ld), a.K, a.L);
-            const Vec3 gmk = spring_force(xp, ld3(xc - 1), a.K, a.L);
-            const Vec3 gpk = spring_force(xp, ld3(xc + 1), a.K, a.L);
+            const Vec3 gmi = spring_force<false, kFma>(xp, ld3(xc - ps), a.K, a.L);
+            const Vec3 gpi = spring_force<false, kFma>(xp, ld3(xc + ps), a.K, a.L);
+            const Vec3 gmj = spring_force<false, kFma>(xp, ld3(xc - g.ld), a.K, a.L);
+            const Vec3 gpj = spring_force<false, kFma>(xp, ld3(xc + g.ld), a.K, a.L);
+            const Vec3 gmk = spring_force<false, kFma>(xp, ld3(xc - 1), a.K, a.L);
+            const Vec3 gpk = spring_force<false, kFma>(xp, ld3(xc + 1), a.K, a.L);
             const Vec3 F = sum_forces(gmi, gpi, gmj, gpj, gmk, gpk);
             double* vp = a.v + p * ps + off;
             Vec3 v{vp[0], vp[cs], vp[2 * cs]};
             Vec3 xn;
-            kick_drift<kUnitMass>(F, a.M, a.dt, v, xp, xn);
+            kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v, xp, xn);
             vp[0] = v.x;
             vp[cs] = v.y;
             vp[2 * cs] = v.z;
@@ -86,10 +86,9 @@ cudaError_t launch_k1_direct(const StepArgs& a, bool unit_mass, cudaStream_t str
     dim3 grid((unsigned)((a.g.n2 + kBX - 1) / kBX), (unsigned)((a.g.n1 + kBY - 1) / kBY), (unsigned)a.g.size);
     StepArgs b = a;
     b.lo_ctas = b.hi_ctas = grid.x * grid.y;  // one plane per grid z: the first / last plane's CTAs
-    if (unit_mass)
-        k1_direct_kernel<true><<<grid, block, 0, stream>>>(b);
-    else
-        k1_direct_kernel<false><<<grid, block, 0, stream>>>(b);
+    auto* kern = unit_mass ? (a.fma ? k1_direct_kernel<true, true> : k1_direct_kernel<true, false>)
+                           : (a.fma ? k1_direct_kernel<false, true> : k1_direct_kernel<false, false>);
+    kern<<<grid, block, 0, stream>>>(b);
     return cudaGetLastError();
 }
 

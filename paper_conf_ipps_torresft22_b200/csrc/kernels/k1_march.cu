@@ -122,7 +122,7 @@ __device__ __forceinline__ Vec3 shfl_up(const Vec3& v) {
 #endif
 constexpr int kUnroll = K1_UNROLL;
 
-template <bool kUnitMass, bool kPosK>
+template <bool kUnitMass, bool kPosK, bool kFma>
 __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     k1_march_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                     const MarchParams mp) {
@@ -183,7 +183,7 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
     // prologue: the -i spring of plane pb is the +i spring of plane pb-1 (negated)
     wait(q0);
     wait(pb);
-    Vec3 carry = spring_force<kPosK>(ld3(stage_x(0) + xo_own), ld3(stage_x(1) + xo_own), a.K, a.L);
+    Vec3 carry = spring_force<kPosK, kFma>(ld3(stage_x(0) + xo_own), ld3(stage_x(1) + xo_own), a.K, a.L);
     Vec3 xc = ld3(stage_x(1) + xo_own);
     __syncthreads();
     if (tid == 0 && q0 + kStages <= qlast) {
@@ -205,16 +205,16 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
         const double* Xn = stage_x(s_nxt);
         const double* me = Xc + xo_own;
         // ---- phase 1: the three "+" springs of every node, plus tile borders
-        const Vec3 gpk = spring_force<kPosK>(xc, ld3(me + 1), a.K, a.L);
+        const Vec3 gpk = spring_force<kPosK, kFma>(xc, ld3(me + 1), a.K, a.L);
         const Vec3 xni = ld3(Xn + xo_own);
-        const Vec3 gpi = spring_force<kPosK>(xc, xni, a.K, a.L);
-        const Vec3 gpj = spring_force<kPosK>(xc, ld3(me + kBK), a.K, a.L);
+        const Vec3 gpi = spring_force<kPosK, kFma>(xc, xni, a.K, a.L);
+        const Vec3 gpj = spring_force<kPosK, kFma>(xc, ld3(me + kBK), a.K, a.L);
         sm.gj[par][w][lane] = gpj;
         if (w == 0) {
-            sm.gbj[par][lane] = spring_force<kPosK>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
+            sm.gbj[par][lane] = spring_force<kPosK, kFma>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
         } else if (w == 1 && lane < kTJ) {
             const double* b = Xc + (lane + 1) * kBK + kCol0;
-            sm.gbk[par][lane] = spring_force<kPosK>(ld3(b - 1), ld3(b), a.K, a.L);
+            sm.gbk[par][lane] = spring_force<kPosK, kFma>(ld3(b - 1), ld3(b), a.K, a.L);
         }
         const Vec3 up = shfl_up(gpk);
         __syncthreads();
@@ -233,7 +233,7 @@ __global__ void __launch_bounds__(kThreads, K1_MIN_BLOCKS)
             const double* Vb = reinterpret_cast<const double*>(smem_raw + s_nxt * kStageBytes + kXSlot) + vo_own;
             Vec3 v{Vb[0], Vb[kVComp], Vb[2 * kVComp]};
             Vec3 xn;
-            kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
+            kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v, xc, xn);
             vo[0] = v.x;
             vo[cs] = v.y;
             vo[2 * cs] = v.z;
@@ -301,10 +301,9 @@ cudaError_t launch_k1_march(const StepArgs& a, bool unit_mass, cudaStream_t stre
         kernel<<<grid, block, smem, stream>>>(mx, mv, mp);
     };
     const bool pos_k = a.K > 0.0;
-    if (unit_mass)
-        pos_k ? launch(k1_march_kernel<true, true>) : launch(k1_march_kernel<true, false>);
-    else
-        pos_k ? launch(k1_march_kernel<false, true>) : launch(k1_march_kernel<false, false>);
+    dispatch_bools([&](auto um, auto pk, auto fm) {
+        launch(k1_march_kernel<decltype(um)::value, decltype(pk)::value, decltype(fm)::value>);
+    }, unit_mass, pos_k, a.fma != 0);
     return cudaGetLastError();
 }
 

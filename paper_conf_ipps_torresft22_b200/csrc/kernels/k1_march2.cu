@@ -92,7 +92,7 @@ __device__ __forceinline__ void st_out(double* p, double v, uint64_t pol) {
         *p = v;
 }
 
-template <bool kUnitMass, bool kPosK>
+template <bool kUnitMass, bool kPosK, bool kFma>
 __device__ __forceinline__ void update_node(bool interior, bool valid, bool write_fixed, const Vec3& F, const double* vb,
                                             const Vec3& xc, double* vo, double* xo, int64_t cs, double* lo_dst,
                                             double* hi_dst, int64_t off, const StepArgs& a, NodeStats& st,
@@ -100,7 +100,7 @@ __device__ __forceinline__ void update_node(bool interior, bool valid, bool writ
     if (interior) {
         Vec3 v{vb[0], vb[kVComp], vb[2 * kVComp]};
         Vec3 xn;
-        kick_drift<kUnitMass>(F, a.M, a.dt, v, xc, xn);
+        kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v, xc, xn);
         st_out(vo, v.x, pol);
         st_out(vo + cs, v.y, pol);
         st_out(vo + 2 * cs, v.z, pol);
@@ -129,7 +129,7 @@ __device__ __forceinline__ void update_node(bool interior, bool valid, bool writ
     }
 }
 
-template <bool kUnitMass, bool kPosK>
+template <bool kUnitMass, bool kPosK, bool kFma>
 __global__ void __launch_bounds__(kThreads, 2)
     k1_march2_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                      const March2Params mp) {
@@ -224,8 +224,8 @@ __global__ void __launch_bounds__(kThreads, 2)
         mbar_wait(&sm.full[s0], 0);
         mbar_wait(&sm.full[s1], 0);
     }
-    Vec3 carryA = spring_force<kPosK>(ld3(stage_x(0) + xA), ld3(stage_x(1) + xA), a.K, a.L);
-    Vec3 carryB = spring_force<kPosK>(ld3(stage_x(0) + xB), ld3(stage_x(1) + xB), a.K, a.L);
+    Vec3 carryA = spring_force<kPosK, kFma>(ld3(stage_x(0) + xA), ld3(stage_x(1) + xA), a.K, a.L);
+    Vec3 carryB = spring_force<kPosK, kFma>(ld3(stage_x(0) + xB), ld3(stage_x(1) + xB), a.K, a.L);
     Vec3 xcA = ld3(stage_x(1) + xA), xcB = ld3(stage_x(1) + xB);
     __syncthreads();
     if (tid == 0 && q0 + kStages <= qlast) {
@@ -247,19 +247,19 @@ __global__ void __launch_bounds__(kThreads, 2)
         const double* Xc = stage_x(s_cur);
         const double* Xn = stage_x(s_nxt);
         // ---- phase 1: "+" springs of both rows (+j of row A uses row B's position)
-        const Vec3 gpkA = spring_force<kPosK>(xcA, ld3(Xc + xA + 1), a.K, a.L);
-        const Vec3 gpkB = spring_force<kPosK>(xcB, ld3(Xc + xB + 1), a.K, a.L);
-        const Vec3 gpjA = spring_force<kPosK>(xcA, xcB, a.K, a.L);
-        const Vec3 gpjB = spring_force<kPosK>(xcB, ld3(Xc + xB + kBK), a.K, a.L);
+        const Vec3 gpkA = spring_force<kPosK, kFma>(xcA, ld3(Xc + xA + 1), a.K, a.L);
+        const Vec3 gpkB = spring_force<kPosK, kFma>(xcB, ld3(Xc + xB + 1), a.K, a.L);
+        const Vec3 gpjA = spring_force<kPosK, kFma>(xcA, xcB, a.K, a.L);
+        const Vec3 gpjB = spring_force<kPosK, kFma>(xcB, ld3(Xc + xB + kBK), a.K, a.L);
         sm.gj[par][w][lane] = gpjB;
         const Vec3 niA = ld3(Xn + xA), niB = ld3(Xn + xB);
-        const Vec3 gpiA = spring_force<kPosK>(xcA, niA, a.K, a.L);
-        const Vec3 gpiB = spring_force<kPosK>(xcB, niB, a.K, a.L);
+        const Vec3 gpiA = spring_force<kPosK, kFma>(xcA, niA, a.K, a.L);
+        const Vec3 gpiB = spring_force<kPosK, kFma>(xcB, niB, a.K, a.L);
         if (w == 0) {
-            sm.gbj[par][lane] = spring_force<kPosK>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
+            sm.gbj[par][lane] = spring_force<kPosK, kFma>(ld3(Xc + ck), ld3(Xc + kBK + ck), a.K, a.L);
         } else if (w == 1 && lane < kTJ) {
             const double* b = Xc + (lane + 1) * kBK + kCol0;
-            sm.gbk[par][lane] = spring_force<kPosK>(ld3(b - 1), ld3(b), a.K, a.L);
+            sm.gbk[par][lane] = spring_force<kPosK, kFma>(ld3(b - 1), ld3(b), a.K, a.L);
         }
         const Vec3 upA = shfl_up1(gpkA), upB = shfl_up1(gpkB);
         __syncthreads();
@@ -277,14 +277,14 @@ __global__ void __launch_bounds__(kThreads, 2)
             const Vec3 gmj = neg(w == 0 ? sm.gbj[par][lane] : sm.gj[par][w - 1][lane]);
             const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w] : upA);
             const Vec3 F = sum_forces(neg(carryA), gpiA, gmj, gpjA, gmk, gpkA);
-            update_node<kUnitMass, kPosK>(intA, validA, a.write_fixed, F, Vb + vA, xcA, vo, xo, cs,
+            update_node<kUnitMass, kPosK, kFma>(intA, validA, a.write_fixed, F, Vb + vA, xcA, vo, xo, cs,
                                           (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offA,
                                           a, st, pol_st);
         }
         {
             const Vec3 gmk = neg(lane == 0 ? sm.gbk[par][2 * w + 1] : upB);
             const Vec3 F = sum_forces(neg(carryB), gpiB, neg(gpjA), gpjB, gmk, gpkB);
-            update_node<kUnitMass, kPosK>(intB, validB, a.write_fixed, F, Vb + vB, xcB, vo + g.ld, xo + g.ld, cs,
+            update_node<kUnitMass, kPosK, kFma>(intB, validB, a.write_fixed, F, Vb + vB, xcB, vo + g.ld, xo + g.ld, cs,
                                           (p == 1) ? a.lo_dst : nullptr, (p == g.size) ? a.hi_dst : nullptr, offB,
                                           a, st, pol_st);
         }
@@ -363,10 +363,9 @@ cudaError_t launch_k1_march2(const StepArgs& a, bool unit_mass, cudaStream_t str
         cudaLaunchKernelEx(&cfg, kernel, mx, mv, mp);
     };
     const bool pos_k = a.K > 0.0;
-    if (unit_mass)
-        pos_k ? launch(k1_march2_kernel<true, true>) : launch(k1_march2_kernel<true, false>);
-    else
-        pos_k ? launch(k1_march2_kernel<false, true>) : launch(k1_march2_kernel<false, false>);
+    dispatch_bools([&](auto um, auto pk, auto fm) {
+        launch(k1_march2_kernel<decltype(um)::value, decltype(pk)::value, decltype(fm)::value>);
+    }, unit_mass, pos_k, a.fma != 0);
     return cudaGetLastError();
 }
 

@@ -126,7 +126,7 @@ __device__ __forceinline__ Vec3 ldb(const double* b, int off, int comp) {
 
 // kTwo: two steps per launch (else one: S1 only, its X_{t+1}, V_{t+1} written
 // for R2 -- the odd step of a TB2 handle, with the same halo layout).
-template <bool kUnitMass, bool kPosK, bool kTwo>
+template <bool kUnitMass, bool kPosK, bool kTwo, bool kFma>
 __global__ void __launch_bounds__(kThreads, 1)
     k1_tb2_kernel(const __grid_constant__ CUtensorMap tmap_x, const __grid_constant__ CUtensorMap tmap_v,
                   const Tb2Params tp) {
@@ -198,10 +198,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     auto border_springs = [&](int p) {
         const double* Xb = xbox(p);
         if (w == 0) {
-            sm.gbj[lane] = spring_force<kPosK>(ldb(Xb, lane + 2, kXComp), ldb(Xb, kBK + lane + 2, kXComp), a.K, a.L);
+            sm.gbj[lane] = spring_force<kPosK, kFma>(ldb(Xb, lane + 2, kXComp), ldb(Xb, kBK + lane + 2, kXComp), a.K, a.L);
         } else if (w == kW - 1 && lane < kRows) {
             const int r = (lane + 1) * kBK;
-            sm.gbk[lane] = spring_force<kPosK>(ldb(Xb, r + 1, kXComp), ldb(Xb, r + 2, kXComp), a.K, a.L);
+            sm.gbk[lane] = spring_force<kPosK, kFma>(ldb(Xb, r + 1, kXComp), ldb(Xb, r + 2, kXComp), a.K, a.L);
         }
     };
 
@@ -212,8 +212,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (ps0 >= 1) {
         border_springs(ps0);  // ps0 <= ilast always
         xwait(ps0 - 1);
-        carry1A = spring_force<kPosK>(ldb(xbox(ps0 - 1), xA, kXComp), xcA, a.K, a.L);
-        carry1B = spring_force<kPosK>(ldb(xbox(ps0 - 1), xB, kXComp), xcB, a.K, a.L);
+        carry1A = spring_force<kPosK, kFma>(ldb(xbox(ps0 - 1), xA, kXComp), xcA, a.K, a.L);
+        carry1B = spring_force<kPosK, kFma>(ldb(xbox(ps0 - 1), xB, kXComp), xcB, a.K, a.L);
         __syncthreads();
         if (tid == 0 && q0 + kStages <= qlast) {
             fence_proxy_async();
@@ -294,16 +294,16 @@ __global__ void __launch_bounds__(kThreads, 1)
         Vec3 gpi1A, gpi1B, gpj1A, gpj1B, gpk1A, gpk1B;
         const Vec3 niA = ldb(Xn, xA, kXComp), niB = ldb(Xn, xB, kXComp);
         if (has_next) {
-            gpi1A = spring_force<kPosK>(xcA, niA, a.K, a.L);
-            gpi1B = spring_force<kPosK>(xcB, niB, a.K, a.L);
+            gpi1A = spring_force<kPosK, kFma>(xcA, niA, a.K, a.L);
+            gpi1B = spring_force<kPosK, kFma>(xcB, niB, a.K, a.L);
         } else {
             gpi1A = gpi1B = Vec3{0.0, 0.0, 0.0};
         }
         if (upd1) {
-            gpk1A = spring_force<kPosK>(xcA, ldb(Xc, xA + 1, kXComp), a.K, a.L);
-            gpk1B = spring_force<kPosK>(xcB, ldb(Xc, xB + 1, kXComp), a.K, a.L);
-            gpj1A = spring_force<kPosK>(xcA, xcB, a.K, a.L);
-            gpj1B = spring_force<kPosK>(xcB, ldb(Xc, xB + kBK, kXComp), a.K, a.L);
+            gpk1A = spring_force<kPosK, kFma>(xcA, ldb(Xc, xA + 1, kXComp), a.K, a.L);
+            gpk1B = spring_force<kPosK, kFma>(xcB, ldb(Xc, xB + 1, kXComp), a.K, a.L);
+            gpj1A = spring_force<kPosK, kFma>(xcA, xcB, a.K, a.L);
+            gpj1B = spring_force<kPosK, kFma>(xcB, ldb(Xc, xB + kBK, kXComp), a.K, a.L);
             sm.g1j[w][lane] = gpj1B;
         } else {
             gpk1A = gpk1B = gpj1A = gpj1B = Vec3{0.0, 0.0, 0.0};
@@ -325,13 +325,13 @@ __global__ void __launch_bounds__(kThreads, 1)
                 const Vec3 gmk = neg(lane == 0 ? sm.gbk[rA] : up1A);
                 const Vec3 F = sum_forces(neg(carry1A), gpi1A, gmj, gpj1A, gmk, gpk1A);
                 v1A = ldb(Vb, vA, kVComp);
-                kick_drift<kUnitMass>(F, a.M, a.dt, v1A, xcA, x1A);
+                kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v1A, xcA, x1A);
             }
             if (intB) {
                 const Vec3 gmk = neg(lane == 0 ? sm.gbk[rB] : up1B);
                 const Vec3 F = sum_forces(neg(carry1B), gpi1B, neg(gpj1A), gpj1B, gmk, gpk1B);
                 v1B = ldb(Vb, vB, kVComp);
-                kick_drift<kUnitMass>(F, a.M, a.dt, v1B, xcB, x1B);
+                kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v1B, xcB, x1B);
             }
         }
         // step t+1's stats right where S1 produced them (plane p, if an output plane of this segment)
@@ -357,13 +357,13 @@ __global__ void __launch_bounds__(kThreads, 1)
             xqA = ldb(yq, yA, kYComp);
             xqB = ldb(yq, yB, kYComp);
             if (kTwo) {
-                gpi2A = spring_force<kPosK>(xqA, x1A, a.K, a.L);
-                gpi2B = spring_force<kPosK>(xqB, x1B, a.K, a.L);
+                gpi2A = spring_force<kPosK, kFma>(xqA, x1A, a.K, a.L);
+                gpi2B = spring_force<kPosK, kFma>(xqB, x1B, a.K, a.L);
                 if (out2) {
-                    gpk2A = spring_force<kPosK>(xqA, ldb(yq, yAk, kYComp), a.K, a.L);
-                    gpk2B = spring_force<kPosK>(xqB, ldb(yq, yBk, kYComp), a.K, a.L);
-                    gpj2A = spring_force<kPosK>(xqA, xqB, a.K, a.L);
-                    gpj2B = spring_force<kPosK>(xqB, ldb(yq, yBj, kYComp), a.K, a.L);
+                    gpk2A = spring_force<kPosK, kFma>(xqA, ldb(yq, yAk, kYComp), a.K, a.L);
+                    gpk2B = spring_force<kPosK, kFma>(xqB, ldb(yq, yBk, kYComp), a.K, a.L);
+                    gpj2A = spring_force<kPosK, kFma>(xqA, xqB, a.K, a.L);
+                    gpj2B = spring_force<kPosK, kFma>(xqB, ldb(yq, yBj, kYComp), a.K, a.L);
                     sm.g2j[w][lane] = gpj2B;
                 }
             }
@@ -383,7 +383,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                     if (kTwo) {
                         const Vec3 gmj = neg(sm.g2j[w > 0 ? w - 1 : 0][lane]);  // w == 0: row 0 is ring, not owned
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
-                        kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqA, x2);
+                        kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v2, xqA, x2);
                     }
                     store_out(q, offA, x2, v2);
                     if (sq) st_add(x2, v2, true);
@@ -396,7 +396,7 @@ __global__ void __launch_bounds__(kThreads, 1)
                     Vec3 v2 = v1pB, x2 = xqB;
                     if (kTwo) {
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
-                        kick_drift<kUnitMass>(F, a.M, a.dt, v2, xqB, x2);
+                        kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v2, xqB, x2);
                     }
                     store_out(q, offB, x2, v2);
                     if (sq) st_add(x2, v2, true);
@@ -541,17 +541,9 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
         kernel<<<grid, block, smem, stream>>>(mx, mv, tp);
     };
     const bool pos_k = a.K > 0.0;
-    if (o.two) {
-        if (unit_mass)
-            pos_k ? launch(k1_tb2_kernel<true, true, true>) : launch(k1_tb2_kernel<true, false, true>);
-        else
-            pos_k ? launch(k1_tb2_kernel<false, true, true>) : launch(k1_tb2_kernel<false, false, true>);
-    } else {
-        if (unit_mass)
-            pos_k ? launch(k1_tb2_kernel<true, true, false>) : launch(k1_tb2_kernel<true, false, false>);
-        else
-            pos_k ? launch(k1_tb2_kernel<false, true, false>) : launch(k1_tb2_kernel<false, false, false>);
-    }
+    dispatch_bools([&](auto um, auto pk, auto two, auto fm) {
+        launch(k1_tb2_kernel<decltype(um)::value, decltype(pk)::value, decltype(two)::value, decltype(fm)::value>);
+    }, unit_mass, pos_k, o.two, a.fma != 0);
     return cudaGetLastError();
 }
 

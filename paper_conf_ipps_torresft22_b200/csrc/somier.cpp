@@ -237,6 +237,9 @@ spread_status check_params(const somier_params* p) {
     if (p->exchange != SOMIER_EXCHANGE_FUSED && p->exchange != SOMIER_EXCHANGE_COPY &&
         p->exchange != SOMIER_EXCHANGE_NCCL)
         PAPER_FAIL(SPREAD_EINVAL, "somier: unknown exchange %d", p->exchange);
+    if (p->math != SOMIER_MATH_EXACT && p->math != SOMIER_MATH_FMA)
+        PAPER_FAIL(SPREAD_EINVAL, "somier: unknown math mode %d", p->math);
+    if (p->reserved != 0) PAPER_FAIL(SPREAD_EINVAL, "somier: reserved must be 0");
     const int64_t n0 = p->n[0], n1 = p->n[1], n2 = p->n[2];
     if (n1 > 65535LL * 8 || n0 > 65535 + 2)
         PAPER_FAIL(SPREAD_EINVAL, "somier: grid too large for the launch geometry");
@@ -1007,6 +1010,7 @@ spread_status enqueue_steps(somier_t h, int64_t nsteps) {
             }
             paper::StepArgs a;
             std::memset(&a, 0, sizeof a);
+            a.fma = h->p.math == SOMIER_MATH_FMA ? 1 : 0;
             a.x_cur = me.xs(cur);
             a.x_nxt = me.xs(nxt);
             a.v = me.vs(vb);
@@ -1101,6 +1105,7 @@ spread_status enqueue_tb2(somier_t h, bool two) {
         }
         paper::StepArgs a;
         std::memset(&a, 0, sizeof a);
+        a.fma = h->p.math == SOMIER_MATH_FMA ? 1 : 0;
         a.x_cur = me.x(cur);
         a.v = me.v(vb);
         a.g = h->geom_of(me);

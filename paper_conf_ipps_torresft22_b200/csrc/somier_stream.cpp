@@ -277,6 +277,7 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         }
         paper::StepArgs a;
         std::memset(&a, 0, sizeof a);
+        a.fma = h->p.math == SOMIER_MATH_FMA ? 1 : 0;
         a.x_cur = sl.x_in;
         a.x_nxt = sl.x_out;
         a.v = sl.v;
@@ -514,6 +515,7 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             if (st != SPREAD_OK) return st;
             paper::StepArgs a;
             std::memset(&a, 0, sizeof a);
+            a.fma = h->p.math == SOMIER_MATH_FMA ? 1 : 0;
             a.x_cur = xs;
             a.v = vs;
             a.g = gj;

@@ -28,7 +28,8 @@ class SomierParams:
     amplitude: float = 0.05
     seed: int = 42
     kernel: int = N.K1_AUTO
-    exchange: int = 0  # SOMIER_EXCHANGE_FUSED (0) or SOMIER_EXCHANGE_COPY (1)
+    exchange: int = 0  # somier_exchange: FUSED (0), COPY (1), NCCL (2)
+    math: int = 0  # somier_math: EXACT (0, bit-identical to the oracle) or FMA (1, reading S22)
 
     def c(self) -> N.somier_params:
         p = N.somier_params()
@@ -36,7 +37,7 @@ class SomierParams:
             p.n[d] = int(self.n[d])
         p.spacing, p.rest_len, p.k_spring, p.mass = self.spacing, self.rest_len, self.k_spring, self.mass
         p.dt, p.amplitude, p.seed, p.kernel = self.dt, self.amplitude, int(self.seed), int(self.kernel)
-        p.exchange = int(self.exchange)
+        p.exchange, p.math = int(self.exchange), int(self.math)
         return p
 
     @property

@@ -52,8 +52,8 @@ def test_status_strings_and_version():
 
 
 def test_struct_layouts():
-    # include/somier.h: somier_params = 3*8 + 7*8 + 2*4 bytes; somier_stats_t = 16*8
-    assert ctypes.sizeof(N.somier_params) == 88
+    # include/somier.h: somier_params = 3*8 + 7*8 + 4*4 bytes; somier_stats_t = 16*8
+    assert ctypes.sizeof(N.somier_params) == 96
     assert ctypes.sizeof(N.somier_stats_t) == 8 * (1 + 3 + 1 + 3 + 3 + 1 + 1)
 
 
@@ -114,3 +114,31 @@ def test_host_grid_size_is_checked():
         S._dptr(np.zeros(23), 24)
     with _pytest.raises(TypeError):
         S._dptr(np.zeros(24, dtype=np.float32), 24)
+
+
+def test_struct_layouts_match_the_c_header(tmp_path):
+    """The ctypes mirrors have the C compiler's sizes and field offsets."""
+    import shutil
+    import subprocess
+
+    cc = shutil.which("gcc") or shutil.which("cc")
+    if cc is None:
+        pytest.skip("no C compiler")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    structs = {"somier_params": N.somier_params, "somier_stats_t": N.somier_stats_t}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "somier.h"', "int main(void) {"]
+    for name, ct in structs.items():
+        lines.append('printf("%s %%zu\\n", sizeof(%s));' % (name, name))
+        for f in ct._fields_:
+            lines.append('printf("%s.%s %%zu\\n", offsetof(%s, %s));' % (name, f[0], name, f[0]))
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines) + "\n")
+    exe = tmp_path / "layout"
+    subprocess.run([cc, "-std=c99", "-I", os.path.join(root, "include"), str(src), "-o", str(exe)], check=True)
+    out = dict(l.rsplit(" ", 1) for l in subprocess.run([str(exe)], check=True, capture_output=True,
+                                                         text=True).stdout.splitlines())
+    for name, ct in structs.items():
+        assert int(out[name]) == ctypes.sizeof(ct), name
+        for f in ct._fields_:
+            assert int(out["%s.%s" % (name, f[0])]) == getattr(ct, f[0]).offset, (name, f[0])

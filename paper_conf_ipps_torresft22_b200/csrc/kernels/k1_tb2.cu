@@ -74,6 +74,11 @@ constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
 #ifndef TB2_MID_STATS
 #define TB2_MID_STATS 1
 #endif
+// TB2_ACC1_SEL=1: round-2's first placement of step t+1's accumulators (every
+// addend selected by ownership, (h, l) pairs as 128-bit slots) -- an A/B only.
+#ifndef TB2_ACC1_SEL
+#define TB2_ACC1_SEL 0
+#endif
 constexpr int kMinSegPlanes = 4, kMaxSegPlanes = 256;
 static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
 
@@ -89,8 +94,8 @@ struct __align__(16) Smem {
     unsigned long long vfull[kVStages];
     WarpStats scratch[kW];
     // step t+1's stats accumulators, thread-private (registers are full):
-    // [0..2] = (sum bits(hd), sum bits(ld)) of x, y, z; [3] = (max v.v, unused)
-    ulonglong2 acc1[4][kThreads];
+    // [0..2] = sum bits(hd) of x, y, z; [3..5] = sum bits(ld); [6] = max v.v
+    unsigned long long acc1[7][kThreads];
 };
 
 struct Tb2Params {
@@ -225,7 +230,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     NodeStats st;  // stats of the launch's last step (t+2, or t+1 in one-step mode); step t+1's: sm.acc1
     st.zero();
 #pragma unroll
-    for (int c = 0; c < 4; c++) sm.acc1[c][tid] = make_ulonglong2(0ull, 0ull);
+    for (int c = 0; c < 7; c++) sm.acc1[c][tid] = 0ull;
     const int border_last = min(pe, ilast);  // planes whose border springs S1 needs
     // X_{t+2} (X_{t+1}), V of an S2 output node: own slab, and the neighbours'
     // halo planes (2 planes of X, 1 of V per face: what their next launch reads)
@@ -242,35 +247,59 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
     };
 
-    // Step t+1's stats of the owned nodes of an output plane q: X_{t+1} from
-    // the ring, V_{t+1} from the register carry; read-modify-write of the
-    // thread's shared-memory accumulators, coordinate by coordinate. Branch-free
-    // (the addends of a node the thread does not own are selected to 0; a fixed
-    // node's V_{t+1} is 0): divergent code here makes ptxas wrap the march's
-    // warp shuffles in collective fix-up sequences.
+    // Step t+1's stats of an output plane from S1's registers (X_{t+1},
+    // V_{t+1}); read-modify-write of the thread's shared-memory accumulators.
+    // Counted rows are shifted by one against R2: a tile counts R1 rows
+    // 0 .. kRows-3 (global [jq - 1, jq + kOJ - 1)), which partition the j axis
+    // as R2's rows do (the launcher sizes tiles_j so the last row is covered) --
+    // so a whole warp (the last) skips, and no addend is selected per node: the
+    // threads of ring / k-face / out-of-grid COLUMNS (kown false) accumulate
+    // anyway and drop their sums at the end, and rows outside the grid add
+    // x = 0, v = 0 (the TMA zero fill, never updated), neutral once counted in
+    // n (set at the end: calls x 2).
+#if TB2_ACC1_SEL
     auto acc1_update = [&](const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb) {
         const double xsa[3] = {xa.x, xa.y, xa.z}, xsb[3] = {xb.x, xb.y, xb.z};
 #pragma unroll
         for (int c = 0; c < 3; c++) {
-            const double hda = __fma_rn(xsa[c], 0x1p28, kRoundC), hdb = __fma_rn(xsb[c], 0x1p28, kRoundC);
-            const double ra = __fma_rn(xsa[c], 0x1p28, -__dsub_rn(hda, kRoundC));
-            const double rb = __fma_rn(xsb[c], 0x1p28, -__dsub_rn(hdb, kRoundC));
-            const double lda = __fma_rn(ra, 0x1p32, kRoundC), ldb_ = __fma_rn(rb, 0x1p32, kRoundC);
+            double hda, lda, hdb, ldb_;
+            split_q(xsa[c], hda, lda);
+            split_q(xsb[c], hdb, ldb_);
             const unsigned long long ha = ownA ? (unsigned long long)__double_as_longlong(hda) : 0ull;
             const unsigned long long hb = ownB ? (unsigned long long)__double_as_longlong(hdb) : 0ull;
             const unsigned long long la = ownA ? (unsigned long long)__double_as_longlong(lda) : 0ull;
             const unsigned long long lb = ownB ? (unsigned long long)__double_as_longlong(ldb_) : 0ull;
-            ulonglong2 o = sm.acc1[c][tid];
-            o.x += ha + hb;
-            o.y += la + lb;
-            sm.acc1[c][tid] = o;
+            sm.acc1[c][tid] += ha + hb;
+            sm.acc1[3 + c][tid] += la + lb;
         }
         const double v2a = ownA ? dot_self(va) : 0.0, v2b = ownB ? dot_self(vb) : 0.0;
-        double vm = __longlong_as_double((long long)sm.acc1[3][tid].x);
+        double vm = __longlong_as_double((long long)sm.acc1[6][tid]);
         vm = (v2a > vm || v2a != v2a) ? v2a : vm;
         vm = (v2b > vm || v2b != v2b) ? v2b : vm;
-        sm.acc1[3][tid].x = (unsigned long long)__double_as_longlong(vm);
+        sm.acc1[6][tid] = (unsigned long long)__double_as_longlong(vm);
     };
+#else
+    auto acc1_update = [&](const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb) {
+        if (w == kW - 1) return;  // warp-uniform
+        auto coord = [&](int c, double a, double b) {
+            double hda, lda, hdb, ldb_;
+            split_q(a, hda, lda);
+            split_q(b, hdb, ldb_);
+            sm.acc1[c][tid] += (unsigned long long)__double_as_longlong(hda) +
+                               (unsigned long long)__double_as_longlong(hdb);
+            sm.acc1[3 + c][tid] += (unsigned long long)__double_as_longlong(lda) +
+                                   (unsigned long long)__double_as_longlong(ldb_);
+        };
+        coord(0, xa.x, xb.x);
+        coord(1, xa.y, xb.y);
+        coord(2, xa.z, xb.z);
+        const double v2a = dot_self(va), v2b = dot_self(vb);
+        double vm = __longlong_as_double((long long)sm.acc1[6][tid]);
+        vm = (v2a > vm || v2a != v2a) ? v2a : vm;
+        vm = (v2b > vm || v2b != v2b) ? v2b : vm;
+        sm.acc1[6][tid] = (unsigned long long)__double_as_longlong(vm);
+    };
+#endif
 
     // the last step's stats of one node (hasv: an interior node, v enters vmax)
     auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
@@ -385,8 +414,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                         const Vec3 F = sum_forces(neg(carry2A), gpi2A, gmj, gpj2A, neg(up2A), gpk2A);
                         kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v2, xqA, x2);
                     }
-                    store_out(q, offA, x2, v2);
+                    // stats first: v.v must not overwrite v2's registers before the stores read them
                     if (sq) st_add(x2, v2, true);
+                    store_out(q, offA, x2, v2);
                 } else if (sq) {
                     st_add(xqA, xqA, false);  // fixed face node
                 }
@@ -398,8 +428,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                         const Vec3 F = sum_forces(neg(carry2B), gpi2B, neg(gpj2A), gpj2B, neg(up2B), gpk2B);
                         kick_drift<kUnitMass, kFma>(F, a.M, a.dt, v2, xqB, x2);
                     }
-                    store_out(q, offB, x2, v2);
+                    // stats first: v.v must not overwrite v2's registers before the stores read them
                     if (sq) st_add(x2, v2, true);
+                    store_out(q, offB, x2, v2);
                 } else if (sq) {
                     st_add(xqB, xqB, false);
                 }
@@ -437,11 +468,19 @@ __global__ void __launch_bounds__(kThreads, 1)
 #ifndef STATS_FP64_ACC
         NodeStats st1;
         for (int c = 0; c < 3; c++) {
-            st1.hb[c] = sm.acc1[c][tid].x;
-            st1.lb[c] = sm.acc1[c][tid].y;
+            st1.hb[c] = sm.acc1[c][tid];
+            st1.lb[c] = sm.acc1[3 + c][tid];
         }
-        st1.vmax2 = __longlong_as_double((long long)sm.acc1[3][tid].x);
+        st1.vmax2 = __longlong_as_double((long long)sm.acc1[6][tid]);
+#if TB2_ACC1_SEL
         st1.copy_count(st);
+#else
+        {
+            const int calls = max(0, min(pe, tp.stats_hi) - max(pb, tp.stats_lo));
+            st1.n = (unsigned)(calls * 2);
+            if (!kown || w == kW - 1) st1.zero();
+        }
+#endif
         __syncthreads();  // scratch reuse
         block_accumulate(st1, sm.scratch, slots.mid);
 #else
@@ -480,7 +519,9 @@ cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cu
         tp.stats_hi = (int)(a.g.start + a.g.size);
     }
     tp.tiles_k = (int)((a.g.n2 - 2 + kOK - 1) / kOK);
-    tp.tiles_j = (int)((a.g.n1 + kOJ - 1) / kOJ);
+    // R2 rows [jq, jq + kOJ) cover [0, n1); step t+1's stats rows [jq - 1,
+    // jq + kOJ - 1) must too (one more tile when n1 is a multiple of kOJ)
+    tp.tiles_j = (int)((a.g.n1 + kOJ) / kOJ);
     const int tiles = tp.tiles_k * tp.tiles_j;
     // Segments per tile column: one CTA per SM (384 threads x 168 registers),
     // so the grid runs in waves of `sms` CTAs. Each segment pays ~3 planes of

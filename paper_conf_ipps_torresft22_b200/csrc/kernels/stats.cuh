@@ -24,14 +24,26 @@ namespace paper {
 
 constexpr int kMaxNodesPerThread = 128;  // STATS_FP64_ACC variant only
 constexpr double kRoundC = 6755399441055744.0;  // 1.5 * 2^52
+constexpr double kRoundK0 = kRoundC * 0x1p32 + kRoundC;  // 1.5 * 2^84 + 1.5 * 2^52, exact (34 significant bits)
+
+// The two words of q(x) = round_half_even(x 2^60) = h 2^32 + l as C + h and
+// C + l (|x| < 2^18), three fp64 operations; see NodeStats below.
+__device__ __forceinline__ void split_q(double x, double& hd, double& ld) {
+    hd = __fma_rn(x, 0x1p28, kRoundC);
+    ld = __fma_rn(x, 0x1p60, __fma_rn(-hd, 0x1p32, kRoundK0));
+}
 
 #ifndef STATS_FP64_ACC
 // Per thread, the exact sums are carried as the BIT PATTERNS of the rounded
-// doubles (fp64 work: 4 operations per coordinate, the accumulation on the
+// doubles (fp64 work: 3 operations per coordinate, the accumulation on the
 // integer pipe):
 //   hd = fma(x, 2^28, C)                   = C + h, h = round_half_even(x 2^28), |h| < 2^51
-//   r  = fma(x, 2^28, -(hd - C))           exact, |r| <= 1/2
-//   ld = fma(r, 2^32, C)                   = C + l, l = round_half_even(r 2^32)
+//   b  = fma(-hd, 2^32, C 2^32 + C)        = C - h 2^32 exactly (a multiple of 2^32 below 2^79
+//                                            in magnitude: 47 significant bits)
+//   ld = fma(x, 2^60, b)                   = RN(C + r 2^32), r = x 2^28 - h (|r| <= 1/2)
+//                                          = C + l, l = round_half_even(r 2^32)
+// (the same two words as the 4-operation form r = fma(x, 2^28, -(hd - C)),
+// ld = fma(r, 2^32, C): one rounding of the same exact value).
 // C + m with |m| < 2^51 lies in [2^52, 2^53), where one unit of the mantissa
 // is 1, so bits(C + m) = bits(C) + m: sum h = sum bits(hd) - n bits(C) and
 // sum l = sum bits(ld) - n bits(C), computed modulo 2^64, which is exact while
@@ -51,9 +63,8 @@ struct NodeStats {
         vmax2 = 0.0;
     }
     __device__ __forceinline__ void add_coord(int c, double x) {
-        const double hd = __fma_rn(x, 0x1p28, kRoundC);
-        const double r = __fma_rn(x, 0x1p28, -__dsub_rn(hd, kRoundC));
-        const double ld = __fma_rn(r, 0x1p32, kRoundC);
+        double hd, ld;
+        split_q(x, hd, ld);
         hb[c] += (unsigned long long)__double_as_longlong(hd);
         lb[c] += (unsigned long long)__double_as_longlong(ld);
     }

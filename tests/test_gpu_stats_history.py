@@ -125,3 +125,25 @@ def test_history_in_graph_replays():
         hist = s.stats_history(0, 42)
     for t in range(42):
         assert _same(hist[t], ref[t][1])
+
+
+@pytest.mark.parametrize("n1", [3, 21, 22, 23, 43, 44, 45, 66])
+@pytest.mark.parametrize("n2", [3, 31, 32, 33, 62])
+def test_tb2_tile_edges_every_step(n1, n2):
+    """K1_TB2 counts step t+1's nodes over R1 rows [jq - 1, jq + 21) (a
+    partition of the j axis shifted by one row against the owned tiles) and
+    drops ring / k-face columns per thread: cross-sections whose n1 is a
+    multiple of the 22-row tile (one more tile row), one below or above it, and
+    k extents around the 30-column tiles -- every step's stats and the state
+    bit for bit vs the oracle."""
+    n = (9, n1, n2)
+    sp = P.SomierParams(n=n, seed=11, kernel=P.K1_TB2)
+    ref = _oracle_history(sp, 6)
+    with P.Somier(P.Spread([0], 1, n[0] - 2), sp) as s:
+        assert s.kernel_in_use == P.K1_TB2
+        s.step(6)
+        hist = s.stats_history(0, 7)
+        X, V = s.read()
+    assert np.array_equal(X, ref[6][0].X) and np.array_equal(V, ref[6][0].V)
+    for t in range(7):
+        assert _same(hist[t], ref[t][1]), "step %d" % t

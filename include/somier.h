@@ -199,6 +199,14 @@ spread_status somier_sync(somier_t h);
  * the chunks THIS handle owns (plus the fixed end planes it holds as halos).
  * In single-process mode that is the whole grid. In multi-process mode combine
  * the per-process results with somier_stats_combine.
+ * Exact-stats domain (S18): the centre sums are exact while every
+ * position is finite with |x| < 2^23. Each state carries an upper bound on
+ * max |x| -- exact for an initialised / loaded (or, host-streamed, mapped-in)
+ * state, and (B + sqrt(vmax^2) |dt|) (1 + 2^-40) for the state a step produces
+ * (computed by the last CTA of each launch: no per-node cost). A state whose
+ * bound is not below 2^23 (or is NaN) reports centre[] = NaN (sum_lo / sum_hi
+ * are still exported; vmax is unaffected). somier_stats_combine propagates a
+ * NaN centre of any partial.
  */
 spread_status somier_stats(somier_t h, somier_stats_t* out);
 

@@ -16,7 +16,7 @@ spread_status check_somier_params(const somier_params* p);
 
 // centre = S * 2^-60 / (n0 n1 n2), vmax = sqrt(max v.v); fills every field.
 void finish_somier_stats(const somier_params* p, const __int128 sums[3], unsigned long long vmax2, int64_t nodes,
-                         int64_t step, somier_stats_t* out);
+                         int64_t step, somier_stats_t* out, bool in_domain = true);
 
 // cudaMemcpy3DAsync between `nplanes` planes of one component of a slab
 // (planes of 3 component blocks, row pitch g.ld) and a dense host grid of that

@@ -134,6 +134,11 @@ struct Tb2Out {
 };
 cudaError_t launch_k1_tb2(const StepArgs& a, const Tb2Out& o, bool unit_mass, cudaStream_t stream);
 cudaError_t launch_init(const InitArgs& a, cudaStream_t stream);
+// max |x| over planes [p0, p0+np) of an X slab (plane index inside the slab)
+// into acc->xmax (atomicMax of the IEEE bits): the exact-stats domain bound
+// of a mapped-in state (stats_layout.hpp, xbound_step)
+cudaError_t launch_xmax(const double* x_slab, const SlabGeom& g, int64_t p0, int64_t np, StatsAccum* acc,
+                        cudaStream_t stream);
 // Test hook (somier_stream_set_delay): one CTA that spins ~ns nanoseconds on the
 // stream, emulating a slower device.
 cudaError_t launch_delay(int64_t ns, cudaStream_t stream);

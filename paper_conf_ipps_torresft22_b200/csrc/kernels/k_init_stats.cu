@@ -61,16 +61,36 @@ __global__ void __launch_bounds__(kBX* kBY)
     const int64_t p = p0 + blockIdx.z;
     NodeStats st;
     st.zero();
+    unsigned long long xm = 0ull;  // max |x| bits (exact-stats domain bound)
     if (j < g.n1 && k < g.n2 && !(k_interior_only && (k == 0 || k == g.n2 - 1))) {
         const int64_t cs = g.comp_stride();
         const double* xp = x + p * g.plane_stride() + j * g.ld + k;
         st.add_position(Vec3{xp[0], xp[cs], xp[2 * cs]});
+        xm = max(abs_bits(xp[0]), max(abs_bits(xp[cs]), abs_bits(xp[2 * cs])));
         if (v) {
             const double* vp = v + (p - 1) * g.plane_stride() + j * g.ld + k;
             st.add_velocity(Vec3{vp[0], vp[cs], vp[2 * cs]});
         }
     }
     block_accumulate(st, scratch, acc);
+    warp_xmax(xm, acc);
+}
+
+// max |x| over the owned planes [p0, p0 + gridDim.z) of an X slab into
+// acc->xmax: the exact-stats domain bound of a state the host-streamed mode
+// maps in at the start of a run (its stats are not summed).
+__global__ void __launch_bounds__(kBX* kBY) xmax_kernel(const double* __restrict__ x, SlabGeom g, int64_t p0,
+                                                         StatsAccum* acc) {
+    const int64_t k = (int64_t)blockIdx.x * kBX + threadIdx.x;
+    const int64_t j = (int64_t)blockIdx.y * kBY + threadIdx.y;
+    const int64_t p = p0 + blockIdx.z;
+    unsigned long long xm = 0ull;
+    if (j < g.n1 && k < g.n2) {
+        const int64_t cs = g.comp_stride();
+        const double* xp = x + p * g.plane_stride() + j * g.ld + k;
+        xm = max(abs_bits(xp[0]), max(abs_bits(xp[cs]), abs_bits(xp[2 * cs])));
+    }
+    warp_xmax(xm, acc);
 }
 
 // Positions of the fixed k-face columns (k = 0 and k = n2-1, every j) of
@@ -82,14 +102,18 @@ __global__ void __launch_bounds__(256) kface_stats_kernel(const double* __restri
     const int64_t p = p0 + blockIdx.y;
     NodeStats st;
     st.zero();
+    unsigned long long xm = 0ull;
     if (j < g.n1) {
         const int64_t cs = g.comp_stride();
         const double* xp = x + p * g.plane_stride() + j * g.ld;
         st.add_position(Vec3{xp[0], xp[cs], xp[2 * cs]});
         const int64_t k1 = g.n2 - 1;
         st.add_position(Vec3{xp[k1], xp[cs + k1], xp[2 * cs + k1]});
+        xm = max(max(abs_bits(xp[0]), max(abs_bits(xp[cs]), abs_bits(xp[2 * cs]))),
+                 max(abs_bits(xp[k1]), max(abs_bits(xp[cs + k1]), abs_bits(xp[2 * cs + k1]))));
     }
     block_accumulate(st, scratch, acc);
+    warp_xmax(xm, acc);
 }
 
 }  // namespace
@@ -99,6 +123,15 @@ cudaError_t launch_kface_stats(const double* x_slab, const SlabGeom& g, int64_t 
     if (np <= 0) return cudaSuccess;
     dim3 grid((unsigned)((g.n1 + 255) / 256), (unsigned)np);
     kface_stats_kernel<<<grid, 256, 0, stream>>>(x_slab, g, p0, acc);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_xmax(const double* x_slab, const SlabGeom& g, int64_t p0, int64_t np, StatsAccum* acc,
+                        cudaStream_t stream) {
+    if (np <= 0) return cudaSuccess;
+    dim3 block(kBX, kBY);
+    dim3 grid((unsigned)((g.n2 + kBX - 1) / kBX), (unsigned)((g.n1 + kBY - 1) / kBY), (unsigned)np);
+    xmax_kernel<<<grid, block, 0, stream>>>(x_slab, g, p0, acc);
     return cudaGetLastError();
 }
 

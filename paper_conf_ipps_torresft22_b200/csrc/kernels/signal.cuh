@@ -39,8 +39,20 @@ __device__ __forceinline__ void finish_launch(const StepArgs& a, unsigned long l
     }
     if (a.step_word) {
         const unsigned int nblocks = gridDim.x * gridDim.y * gridDim.z;
+        __threadfence();  // this CTA's stats atomics (block_accumulate, same thread) before its count
         if (atomicAdd(a.done_counter, 1u) == nblocks - 1) {
+            __threadfence();
             *a.done_counter = 0u;
+            // exact-stats domain bound of the states this launch produced
+            // (stats_layout.hpp): from the previous state's bound and each
+            // step's vmax, now complete
+            volatile StatsAccum* r = a.acc_ring;
+            double B = __longlong_as_double((long long)r[ring_slot(t)].xmax);
+            for (int s = 1; s <= nsteps; s++) {
+                volatile StatsAccum* q = r + ring_slot(t + (unsigned long long)s);
+                B = xbound_step(B, __longlong_as_double((long long)q->vmax2), a.dt);
+                q->xmax = (unsigned long long)__double_as_longlong(B);
+            }
             *a.step_word = t + (unsigned long long)nsteps;
         }
     }

@@ -208,6 +208,23 @@ __device__ __forceinline__ void atomic_add_i128(unsigned long long* lo_word, uns
     }
 }
 
+// max |x| of the nodes a warp's threads hold (IEEE bits of |x|: non-negative
+// doubles order as unsigned integers, NaN above inf) into acc->xmax -- the
+// exact-stats domain bound of a state the stats kernels sum (stats_layout.hpp).
+// All 32 lanes of the warp must call it.
+__device__ __forceinline__ unsigned long long abs_bits(double x) {
+    return (unsigned long long)__double_as_longlong(fabs(x));
+}
+__device__ __forceinline__ void warp_xmax(unsigned long long b, StatsAccum* acc) {
+#pragma unroll
+    for (int m = 16; m > 0; m >>= 1) {
+        const unsigned long long o = __shfl_xor_sync(0xffffffffu, b, m);
+        b = o > b ? o : b;
+    }
+    const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+    if ((tid & 31) == 0 && b) atomicMax(&acc->xmax, b);
+}
+
 struct WarpStats {
     unsigned long long lo[3], hi[3], vmax2, pad;
 };

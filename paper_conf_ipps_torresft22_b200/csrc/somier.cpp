@@ -594,13 +594,16 @@ int64_t owned_nodes(const somier_s* h, const Chunk& c) {
     return planes * h->p.n[1] * h->p.n[2];
 }
 
+// in_domain: the state's bound on max |x| is inside the exact-stats domain
+// (stats_layout.hpp, xbound_ok); else the sums need not be the exact centre
+// sums and the centre is reported as NaN (the sums are still exported).
 void finish_stats(const somier_params* p, __int128 sums[3], unsigned long long vmax2, int64_t nodes, int64_t step,
-                  somier_stats_t* out) {
+                  somier_stats_t* out, bool in_domain = true) {
     const double N = (double)(p->n[0] * p->n[1] * p->n[2]);
     for (int c = 0; c < 3; c++) {
         out->sum_lo[c] = (uint64_t)(unsigned __int128)sums[c];
         out->sum_hi[c] = (int64_t)(sums[c] >> 64);
-        out->centre[c] = std::ldexp((double)sums[c], -60) / N;
+        out->centre[c] = in_domain ? std::ldexp((double)sums[c], -60) / N : std::nan("");
     }
     double v2;
     std::memcpy(&v2, &vmax2, sizeof v2);
@@ -624,9 +627,9 @@ namespace paper {
 spread_status check_somier_params(const somier_params* p) { return check_params(p); }
 
 void finish_somier_stats(const somier_params* p, const __int128 sums[3], unsigned long long vmax2, int64_t nodes,
-                         int64_t step, somier_stats_t* out) {
+                         int64_t step, somier_stats_t* out, bool in_domain) {
     __int128 s[3] = {sums[0], sums[1], sums[2]};
-    finish_stats(p, s, vmax2, nodes, step, out);
+    finish_stats(p, s, vmax2, nodes, step, out, in_domain);
 }
 
 spread_status encode_slab_tmap(CUtensorMap* map, const SlabGeom& g, double* base, int64_t planes, uint32_t box_k,
@@ -1204,7 +1207,7 @@ spread_status somier_stats_history(somier_t h, int64_t first_step, int64_t count
     if (st != SPREAD_OK) return st;
     if (count == 0) return SPREAD_OK;
     std::vector<__int128> sums((size_t)count * 3, 0);
-    std::vector<unsigned long long> vmax2((size_t)count, 0ull);
+    std::vector<unsigned long long> vmax2((size_t)count, 0ull), xmax((size_t)count, 0ull);
     int64_t nodes = 0;
     std::vector<paper::StatsAccum> acc(paper::kStatsRing + 1);
     for (auto& c : h->chunks) {
@@ -1216,12 +1219,19 @@ spread_status somier_stats_history(somier_t h, int64_t first_step, int64_t count
                 for (int d = 0; d < 3; d++)
                     sums[(size_t)(3 * i + d)] += (__int128)(((unsigned __int128)acc[q].hi[d] << 64) | acc[q].lo[d]);
                 vmax2[(size_t)i] = std::max(vmax2[(size_t)i], (unsigned long long)acc[q].vmax2);
+                xmax[(size_t)i] = std::max(xmax[(size_t)i], (unsigned long long)acc[q].xmax);
             }
         }
         nodes += owned_nodes(h, c);
     }
     for (int64_t i = 0; i < count; i++)
-        finish_stats(&h->p, &sums[(size_t)(3 * i)], vmax2[(size_t)i], nodes, first_step + i, &out[i]);
+    {
+        double B;
+        const unsigned long long b = xmax[(size_t)i];
+        std::memcpy(&B, &b, sizeof B);  // the bound's IEEE bits (NaN bits order above inf)
+        finish_stats(&h->p, &sums[(size_t)(3 * i)], vmax2[(size_t)i], nodes, first_step + i, &out[i],
+                     paper::xbound_ok(B));
+    }
     return SPREAD_OK;
 }
 
@@ -1235,15 +1245,17 @@ spread_status somier_stats_combine(const somier_stats_t* parts, int n, const som
     __int128 sums[3] = {0, 0, 0};
     unsigned long long vmax2 = 0;
     int64_t nodes = 0;
+    bool in_domain = true;  // a partial outside the exact-stats domain reports a NaN centre
     for (int i = 0; i < n; i++) {
         if (parts[i].step != parts[0].step)
             PAPER_FAIL(SPREAD_EINVAL, "somier_stats_combine: partials of different steps");
+        for (int d = 0; d < 3; d++) in_domain = in_domain && !std::isnan(parts[i].centre[d]);
         for (int d = 0; d < 3; d++)
             sums[d] += (__int128)(((unsigned __int128)(uint64_t)parts[i].sum_hi[d] << 64) | parts[i].sum_lo[d]);
         vmax2 = std::max(vmax2, (unsigned long long)parts[i].vmax2_bits);
         nodes += parts[i].nodes;
     }
-    finish_stats(p, sums, vmax2, nodes, parts[0].step, out);
+    finish_stats(p, sums, vmax2, nodes, parts[0].step, out, in_domain);
     return SPREAD_OK;
 }
 

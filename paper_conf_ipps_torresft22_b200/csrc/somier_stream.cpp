@@ -274,6 +274,8 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
         if (t == 0) {  // the fixed end planes, once per run (they never move)
             if (first) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, 0, 1, d.acc_static(), d.s_comp));
             if (last) S_TRY(h, paper::launch_stats(sl.x_in, nullptr, g, ci.size + 1, 1, d.acc_static(), d.s_comp));
+            // max |x| of the input state (the exact-stats domain bound, stats_layout.hpp)
+            S_TRY(h, paper::launch_xmax(sl.x_in, g, 1, ci.size, d.acc_static(), d.s_comp));
         }
         paper::StepArgs a;
         std::memset(&a, 0, sizeof a);
@@ -328,6 +330,7 @@ spread_status enqueue_stream_step(somier_stream_t h, double* const X[3], double*
 spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, somier_stats_t* stats) {
     std::vector<__int128> sums((size_t)n * 3, 0);
     std::vector<unsigned long long> vmax2((size_t)n, 0);
+    unsigned long long xmax0 = 0;  // max |x| bits of the run's input state and the fixed nodes
     std::vector<paper::StatsAccum> acc((size_t)n + 1);
     for (auto& d : h->devs) {
         if (!d.active) continue;
@@ -340,10 +343,19 @@ spread_status gather_stats(somier_stream_t h, int64_t n, const int64_t* steps, s
                     sums[(size_t)(3 * t + k)] += (__int128)(((unsigned __int128)a.hi[k] << 64) | a.lo[k]);
                 vmax2[(size_t)t] = std::max(vmax2[(size_t)t], (unsigned long long)a.vmax2);
             }
+        xmax0 = std::max(xmax0, (unsigned long long)acc[0].xmax);
     }
-    for (int64_t t = 0; t < n; t++)
+    // exact-stats domain: the bound of each state from the input state's max |x|
+    // and every step's vmax (stats_layout.hpp)
+    double B;
+    std::memcpy(&B, &xmax0, sizeof B);
+    for (int64_t t = 0; t < n; t++) {
+        double v2;
+        std::memcpy(&v2, &vmax2[(size_t)t], sizeof v2);
+        B = paper::xbound_step(B, v2, h->p.dt);
         paper::finish_somier_stats(&h->p, &sums[(size_t)(3 * t)], vmax2[(size_t)t],
-                                   h->p.n[0] * h->p.n[1] * h->p.n[2], steps[t], &stats[t]);
+                                   h->p.n[0] * h->p.n[1] * h->p.n[2], steps[t], &stats[t], paper::xbound_ok(B));
+    }
     return SPREAD_OK;
 }
 
@@ -496,6 +508,8 @@ spread_status enqueue_stream_blocked(somier_stream_t h, double* const X[3], doub
             if (first) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, 0, 1, d.acc_static(), d.s_comp));
             if (last) S_TRY(h, paper::launch_stats(xv_one, nullptr, g, ci.size + 1, 1, d.acc_static(), d.s_comp));
             S_TRY(h, paper::launch_kface_stats(xv_one, g, 1, ci.size, d.acc_static(), d.s_comp));
+            // max |x| of the input state (the exact-stats domain bound, stats_layout.hpp)
+            S_TRY(h, paper::launch_xmax(xv_one, g, 1, ci.size, d.acc_static(), d.s_comp));
         }
         S_TRY(h, paper::launch_delay(d.delay_ns, d.s_comp));
         int64_t remaining = s, done = 0;

@@ -54,6 +54,12 @@ class Stats:
     vmax2_bits: int
     nodes: int
 
+    @property
+    def in_domain(self) -> bool:
+        """False when a node of the state lies outside the exact-stats domain
+        (|x| >= 2^23 or non-finite): the centre is then NaN (somier.h)."""
+        return not any(c != c for c in self.centre)
+
     @staticmethod
     def from_c(s: N.somier_stats_t) -> "Stats":
         sums = tuple((int(s.sum_hi[c]) << 64) | int(s.sum_lo[c]) for c in range(3))

@@ -74,11 +74,6 @@ constexpr int kStages = TB2_STAGES, kVStages = TB2_VSTAGES;
 #ifndef TB2_MID_STATS
 #define TB2_MID_STATS 1
 #endif
-// TB2_ACC1_SEL=1: round-2's first placement of step t+1's accumulators (every
-// addend selected by ownership, (h, l) pairs as 128-bit slots) -- an A/B only.
-#ifndef TB2_ACC1_SEL
-#define TB2_ACC1_SEL 0
-#endif
 constexpr int kMinSegPlanes = 4, kMaxSegPlanes = 256;
 static_assert(kRows <= 32, "the -k border springs are computed by one warp, one row per lane");
 
@@ -257,28 +252,6 @@ __global__ void __launch_bounds__(kThreads, 1)
     // anyway and drop their sums at the end, and rows outside the grid add
     // x = 0, v = 0 (the TMA zero fill, never updated), neutral once counted in
     // n (set at the end: calls x 2).
-#if TB2_ACC1_SEL
-    auto acc1_update = [&](const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb) {
-        const double xsa[3] = {xa.x, xa.y, xa.z}, xsb[3] = {xb.x, xb.y, xb.z};
-#pragma unroll
-        for (int c = 0; c < 3; c++) {
-            double hda, lda, hdb, ldb_;
-            split_q(xsa[c], hda, lda);
-            split_q(xsb[c], hdb, ldb_);
-            const unsigned long long ha = ownA ? (unsigned long long)__double_as_longlong(hda) : 0ull;
-            const unsigned long long hb = ownB ? (unsigned long long)__double_as_longlong(hdb) : 0ull;
-            const unsigned long long la = ownA ? (unsigned long long)__double_as_longlong(lda) : 0ull;
-            const unsigned long long lb = ownB ? (unsigned long long)__double_as_longlong(ldb_) : 0ull;
-            sm.acc1[c][tid] += ha + hb;
-            sm.acc1[3 + c][tid] += la + lb;
-        }
-        const double v2a = ownA ? dot_self(va) : 0.0, v2b = ownB ? dot_self(vb) : 0.0;
-        double vm = __longlong_as_double((long long)sm.acc1[6][tid]);
-        vm = (v2a > vm || v2a != v2a) ? v2a : vm;
-        vm = (v2b > vm || v2b != v2b) ? v2b : vm;
-        sm.acc1[6][tid] = (unsigned long long)__double_as_longlong(vm);
-    };
-#else
     auto acc1_update = [&](const Vec3& xa, const Vec3& xb, const Vec3& va, const Vec3& vb) {
         if (w == kW - 1) return;  // warp-uniform
         auto coord = [&](int c, double a, double b) {
@@ -299,7 +272,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         vm = (v2b > vm || v2b != v2b) ? v2b : vm;
         sm.acc1[6][tid] = (unsigned long long)__double_as_longlong(vm);
     };
-#endif
 
     // the last step's stats of one node (hasv: an interior node, v enters vmax)
     auto st_add = [&](const Vec3& x, const Vec3& v, bool hasv) {
@@ -472,15 +444,11 @@ __global__ void __launch_bounds__(kThreads, 1)
             st1.lb[c] = sm.acc1[3 + c][tid];
         }
         st1.vmax2 = __longlong_as_double((long long)sm.acc1[6][tid]);
-#if TB2_ACC1_SEL
-        st1.copy_count(st);
-#else
         {
             const int calls = max(0, min(pe, tp.stats_hi) - max(pb, tp.stats_lo));
             st1.n = (unsigned)(calls * 2);
             if (!kown || w == kW - 1) st1.zero();
         }
-#endif
         __syncthreads();  // scratch reuse
         block_accumulate(st1, sm.scratch, slots.mid);
 #else

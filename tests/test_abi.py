@@ -71,6 +71,21 @@ def test_stats_combine_is_exact_host_logic():
         P.combine_stats([a, P.Stats(4, (0.0,) * 3, 0.0, (0, 0, 0), 0, 0)], sp)
 
 
+def test_stats_combine_propagates_out_of_domain():
+    """A partial outside the exact-stats domain (NaN centre, include/somier.h)
+    makes the combined centre NaN; the sums and vmax still combine exactly."""
+    import math
+
+    sp = P.SomierParams(n=(4, 4, 4))
+    a = P.Stats(3, (1.0, 2.0, 3.0), 0.0, (5, 6, 7), 0x3FF0000000000000, 32)
+    b = P.Stats(3, (math.nan,) * 3, 0.0, (1, 1, 1), 0x4000000000000000, 32)
+    c = P.combine_stats([a, b], sp)
+    assert not c.in_domain and all(math.isnan(x) for x in c.centre)
+    assert c.sums == (6, 7, 8) and c.vmax == 2.0 ** 0.5
+    d = P.combine_stats([a, a], sp)
+    assert d.in_domain and d.centre[0] == (10 * 2.0 ** -60) / 64
+
+
 def test_somier_init_without_gpu_fails_loudly():
     import torch
     if torch.cuda.is_available():

@@ -89,12 +89,12 @@ def interior_of(n, size):
 
 
 # fp64 lane-instructions per node-update of node_math.cuh with each spring
-# evaluated once: 3 springs x 27 (3 sub, d^2 5, sqrt + 1/d 11,
-# d-L and K* 2, quotient 3, f*d 3) + force sum 15 + kick/drift 12 = 108, and the
-# fused stats of every step 15 (3 x 3 exact-split centre terms, v.v 5, max 1).
-# SOMIER_MATH_FMA: d^2 as an FMA chain (-2 per spring) and the kick/drift as 6
-# FMAs (-6): 96 per node-update.
-FP64_OPS_STEP, FP64_OPS_STEP_FMA, FP64_OPS_STATS = 108, 96, 15
+# evaluated once: 3 springs x 26 (3 sub, d^2 5, sqrt + 1/d 10 --
+# its y/2 is an integer exponent decrement --, d-L and K* 2, quotient 3, f*d 3)
+# + force sum 15 + kick/drift 12 = 105, and the fused stats of every step 15
+# (3 x 3 exact-split centre terms, v.v 5, max 1). SOMIER_MATH_FMA: d^2 as an
+# FMA chain (-2 per spring) and the kick/drift as 6 FMAs (-6): 93.
+FP64_OPS_STEP, FP64_OPS_STEP_FMA, FP64_OPS_STATS = 105, 93, 15
 
 
 def fp64_ops_per_node_update(math="exact"):

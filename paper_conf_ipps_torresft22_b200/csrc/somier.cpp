@@ -18,6 +18,7 @@
 #include <vector>
 
 #include "driver_util.hpp"
+#include "guard.hpp"
 #include "kernels.hpp"
 #include "nccl_api.hpp"
 #include "trace.hpp"
@@ -65,6 +66,8 @@ struct Chunk {
     void* base = nullptr;
     size_t bytes = 0;
     size_t off_x[2] = {0, 0}, off_v = 0, off_v1 = 0, off_acc = 0, off_flags = 0, off_counter = 0;
+    size_t xbytes = 0;  // one X buffer (without a guard zone)
+    paper::GuardLayout guard;  // SOMIER_GUARD zones (guard.hpp; none by default)
     int64_t view_off = 0;  // doubles from a raw slab to its one-halo view (one plane on K1_TB2 handles)
     // remote view (IPC-opened), for non-local neighbours
     void* remote_base = nullptr;
@@ -126,6 +129,7 @@ uint64_t spread_layout_hash(const spread_s& s) {
 }
 
 size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
 
 }  // namespace
 
@@ -340,18 +344,26 @@ spread_status allocate_chunk(somier_t h, Chunk& c) {
     const size_t xb = round_up(plane * (size_t)(c.size + 2 + 2 * deep), 4096);
     const size_t vb = round_up(plane * (size_t)(c.size + 2 * deep), 4096);
     c.view_off = deep * g.plane_stride();
-    c.off_x[0] = 0;
-    c.off_x[1] = xb;
-    c.off_v = 2 * xb;
-    c.off_v1 = h->tb2 ? c.off_v + vb : c.off_v;
-    c.off_acc = c.off_v + (h->tb2 ? 2 : 1) * vb;
-    c.off_flags = c.off_acc + (paper::kStatsRing + 2) * sizeof(paper::StatsAccum);
+    c.xbytes = xb;
+    // [guard] X_0 [guard] X_1 [guard] V ([guard] V') [guard] stats ring + flags + counters [guard]
+    const size_t accb = (paper::kStatsRing + 2) * sizeof(paper::StatsAccum);
+    std::vector<std::pair<size_t, const char*>> regions = {{xb, "X_0"}, {xb, "X_1"}, {vb, "V"}};
+    if (h->tb2) regions.push_back({vb, "V'"});
+    regions.push_back({accb + 2 * sizeof(unsigned long long) + 64, "stats"});
+    c.guard.plan(paper::guard_bytes(plane), regions);  // no zones unless SOMIER_GUARD is set
+    c.off_x[0] = c.guard.off[0];
+    c.off_x[1] = c.guard.off[1];
+    c.off_v = c.guard.off[2];
+    c.off_v1 = h->tb2 ? c.guard.off[3] : c.off_v;
+    c.off_acc = c.guard.off.back();
+    c.off_flags = c.off_acc + accb;
     c.off_counter = c.off_flags + 2 * sizeof(unsigned long long);  // counter (4 B, padded to 8), step word, side counters[2]
-    c.bytes = round_up(c.off_counter + 64, 4096);
+    c.bytes = c.guard.bytes;
     CUDA_TRY(h, cudaSetDevice(c.device));
     CUDA_TRY(h, cudaMalloc(&c.base, c.bytes));
     cudaStream_t s = h->stream_of(c);
     CUDA_TRY(h, cudaMemsetAsync(c.base, 0, c.bytes, s));
+    CUDA_TRY(h, paper::guard_fill(c.guard, c.base, s));
     paper::InitArgs ia;
     ia.x0 = c.x(0);
     ia.x1 = c.x(1);
@@ -392,6 +404,19 @@ spread_status sync_all(somier_t h) {
         if (e != cudaSuccess) return cuda_fail(h, e, "somier_sync");
     }
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    for (size_t ci = 0; ci < h->chunks.size(); ci++) {  // SOMIER_GUARD zones (guard.hpp)
+        const Chunk& c = h->chunks[ci];
+        if (!c.local || !c.guard.G) continue;
+        std::string msg;
+        cudaError_t e = cudaSetDevice(c.device);
+        if (e != cudaSuccess) return cuda_fail(h, e, "somier guard check");
+        const std::string what = "chunk " + std::to_string(ci);
+        if (!paper::guard_check(c.guard, c.base, what.c_str(), msg, e)) {
+            if (e != cudaSuccess) return cuda_fail(h, e, "somier guard check");
+            if (h->sticky.empty()) h->sticky = msg;
+            PAPER_FAIL(SPREAD_ECUDA, "%s", msg.c_str());
+        }
+    }
     return SPREAD_OK;
 }
 
@@ -1348,7 +1373,7 @@ spread_status somier_load(somier_t h, const double* x, const double* y, const do
             }
         }
         // the X_{t+1} buffer must hold the same fixed nodes (never written by a step)
-        CUDA_TRY(h, cudaMemcpyAsync(c.x(cur ^ 1), c.x(cur), c.off_x[1] - c.off_x[0], cudaMemcpyDeviceToDevice, s));
+        CUDA_TRY(h, cudaMemcpyAsync(c.x(cur ^ 1), c.x(cur), c.xbytes, cudaMemcpyDeviceToDevice, s));
         spread_status st = reset_stats(h, c);
         if (st != SPREAD_OK) return st;
     }

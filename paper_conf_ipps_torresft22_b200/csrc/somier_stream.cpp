@@ -19,6 +19,7 @@
 #include <vector>
 
 #include "driver_util.hpp"
+#include "guard.hpp"
 #include "kernels.hpp"
 #include "somier.h"
 #include "spread_impl.hpp"
@@ -34,6 +35,7 @@ struct Slot {
     double* x_in = nullptr;   // X_t of the chunk, size+2 planes (halo planes included)
     double* x_out = nullptr;  // X_{t+1}, planes 1..size written by K1
     double* v = nullptr;      // V of the chunk, size planes
+    paper::GuardLayout guard; // SOMIER_GUARD zones (guard.hpp; none by default)
     alignas(64) CUtensorMap tmap_x;
     alignas(64) CUtensorMap tmap_v;
     alignas(64) CUtensorMap tmap_x2;
@@ -88,6 +90,7 @@ bool slot_free(const SlotT& sl) {
 struct DeepSlot {
     void* base = nullptr;
     double *xa = nullptr, *xb = nullptr, *va = nullptr, *vb = nullptr;
+    paper::GuardLayout guard;
     int64_t planes = 0;  // X planes per buffer (V: planes - 2)
     cudaEvent_t comp_done = nullptr, d2h_done = nullptr;
     bool used = false;
@@ -220,6 +223,27 @@ spread_status sync_devs(somier_stream_t h) {
         if (e != cudaSuccess) return sfail(h, e, "somier_stream: synchronize");
     }
     if (!h->sticky.empty()) PAPER_FAIL(SPREAD_ECUDA, "%s", h->sticky.c_str());
+    for (auto& d : h->devs) {  // SOMIER_GUARD zones (guard.hpp)
+        auto check = [&](const paper::GuardLayout& L, const void* base, const char* kind, size_t i) -> spread_status {
+            if (!L.G || !base) return SPREAD_OK;
+            std::string msg;
+            cudaError_t e = cudaSetDevice(d.device);
+            const std::string what = std::string(kind) + " " + std::to_string(i) + " of list position " +
+                                     std::to_string(d.pos);
+            if (e == cudaSuccess && paper::guard_check(L, base, what.c_str(), msg, e)) return SPREAD_OK;
+            if (e != cudaSuccess) return sfail(h, e, "somier_stream guard check");
+            if (h->sticky.empty()) h->sticky = msg;
+            PAPER_FAIL(SPREAD_ECUDA, "%s", msg.c_str());
+        };
+        for (size_t i = 0; i < d.slots.size(); i++) {
+            spread_status st = check(d.slots[i].guard, d.slots[i].base, "slot", i);
+            if (st != SPREAD_OK) return st;
+        }
+        for (size_t i = 0; i < d.deep.size(); i++) {
+            spread_status st = check(d.deep[i].guard, d.deep[i].base, "deep slot", i);
+            if (st != SPREAD_OK) return st;
+        }
+    }
     return SPREAD_OK;
 }
 
@@ -384,10 +408,15 @@ spread_status ensure_flat(somier_stream_t h) {
         release_deep(d);
         for (auto& sl : d.slots) {
             if (sl.base) continue;
-            S_TRY(h, cudaMalloc(&sl.base, 2 * xb + vb));
-            sl.x_in = (double*)sl.base;
-            sl.x_out = (double*)((char*)sl.base + xb);
-            sl.v = (double*)((char*)sl.base + 2 * xb);
+            sl.guard.plan(paper::guard_bytes(plane), {{xb, "X in"}, {xb, "X out"}, {vb, "V"}});
+            S_TRY(h, cudaMalloc(&sl.base, sl.guard.bytes));
+            sl.x_in = (double*)((char*)sl.base + sl.guard.off[0]);
+            sl.x_out = (double*)((char*)sl.base + sl.guard.off[1]);
+            sl.v = (double*)((char*)sl.base + sl.guard.off[2]);
+            if (sl.guard.G) {  // cudaMemset* on the legacy stream: finished before the handle's streams start
+                S_TRY(h, paper::guard_fill(sl.guard, sl.base, 0));
+                S_TRY(h, cudaDeviceSynchronize());
+            }
             sl.used = false;
             const paper::SlabGeom g = h->geom;
             spread_status st = paper::encode_slab_tmap(&sl.tmap_x, g, sl.x_in, h->max_chunk + 2, paper::kXBoxK,
@@ -424,13 +453,15 @@ spread_status ensure_deep(somier_stream_t h, int64_t planes) {
         const size_t xb = round_up(plane * (size_t)planes, 4096), vb = round_up(plane * (size_t)(planes - 2), 4096);
         for (auto& sl : d.deep) {
             sl.base = nullptr;
-            S_TRY(h, cudaMalloc(&sl.base, 2 * xb + 2 * vb));
+            sl.guard.plan(paper::guard_bytes(plane), {{xb, "X a"}, {xb, "X b"}, {vb, "V a"}, {vb, "V b"}});
+            S_TRY(h, cudaMalloc(&sl.base, sl.guard.bytes));
             // zeroed once: the fixed face nodes of V are never written by K1_TB2
-            S_TRY(h, cudaMemset(sl.base, 0, 2 * xb + 2 * vb));
-            sl.xa = (double*)sl.base;
-            sl.xb = (double*)((char*)sl.base + xb);
-            sl.va = (double*)((char*)sl.base + 2 * xb);
-            sl.vb = (double*)((char*)sl.base + 2 * xb + vb);
+            S_TRY(h, cudaMemset(sl.base, 0, sl.guard.bytes));
+            S_TRY(h, paper::guard_fill(sl.guard, sl.base, 0));
+            sl.xa = (double*)((char*)sl.base + sl.guard.off[0]);
+            sl.xb = (double*)((char*)sl.base + sl.guard.off[1]);
+            sl.va = (double*)((char*)sl.base + sl.guard.off[2]);
+            sl.vb = (double*)((char*)sl.base + sl.guard.off[3]);
             sl.planes = planes;
             sl.used = false;
             for (cudaEvent_t* pe : {&sl.comp_done, &sl.d2h_done})
